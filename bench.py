@@ -1,0 +1,335 @@
+#!/usr/bin/env python
+"""bench.py — GSNP hot path on B200: genome sites/s (device-timed) + HBM roofline.
+
+One step = the whole hot path over one shard of synthetic input:
+calibration count (GPU histogram) -> [N>1: NCCL all-reduce of the 2 MiB counts] -> finalize
+(host p matrix + score table, upload) -> gsnp_call over every site of the shard.  Inputs are
+resident in HBM before timing.  N=1 workload: BASELINE.json configs[1] (C2, chr21-like 48 Mb,
+20X).  Multi-GPU: weak scaling, each rank a contiguous C2-sized shard of a larger genome.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl reference]
+
+--impl reference times the CPU oracle (the reference arm of this tier) on a bounded sample.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "genome sites/sec at 1/2/4/8 B200 (device-timed) + % of HBM roofline"
+UNIT = "sites/s"
+
+
+def _peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.rows = []
+        self.stop = threading.Event()
+        self.th = threading.Thread(target=self._run, daemon=True)
+
+    def _run(self):
+        while not self.stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True,
+                                     text=True, timeout=5).stdout.strip()
+                if out:
+                    self.rows.append([x.strip() for x in out.split(",")])
+            except Exception:
+                pass
+            self.stop.wait(0.1)
+
+    def __enter__(self):
+        self.th.start()
+        return self
+
+    def __exit__(self, *a):
+        self.stop.set()
+        self.th.join(timeout=10)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4)
+                          if len(r) > 2 + i and r[2 + i].lower() == "active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": reasons,
+                "samples": len(self.rows)}
+
+
+def _dist():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def make_shard(cfg_name: str, rank: int, ws: int):
+    import synth
+    base = synth.CONFIGS[cfg_name]
+    # weak scaling: rank r holds sites [r*n, (r+1)*n) of a genome of ws*n sites
+    cfg = base.scaled(seed=base.seed + 1000 * rank, origin=rank * base.n_sites)
+    return synth.generate(cfg)
+
+
+def input_bytes(w) -> int:
+    return sum(int(np.asarray(w[k]).nbytes) for k in ("pos", "len", "off", "bases", "quals",
+                                                      "strand", "hits"))
+
+
+def cpu_oracle_rate(w, budget_s: float = 15.0, max_sites: int | None = None):
+    """Oracle (as it stands) on a bounded sample of the shard: calibration + call over the
+    first S non-trivial sites; returns (sites/s, description)."""
+    import oracle
+    import synth
+    P = oracle.Params()
+    origin = int(w["origin"])
+    ref = w["ref"]
+    nz = np.nonzero(ref != 4)[0]
+    s0 = origin + int(nz[0]) if len(nz) else origin
+    S = 50_000
+    rate = None
+    desc = ""
+    spent = 0.0
+    while True:
+        s1 = min(s0 + S, origin + len(ref))
+        ra, rb = synth.read_range(w, s0, s1)
+        sub = synth.slice_reads(w, ra, rb)
+        t = time.perf_counter()
+        C = oracle.calib_counts(P, sub)
+        p = oracle.p_matrix(P, C)
+        oracle.call_window(P, sub, p, s0, s1)
+        dt = time.perf_counter() - t
+        spent += dt
+        rate = (s1 - s0) / dt
+        desc = (f"oracle calibrate+call over {s1 - s0} sites [{s0},{s1}) of the shard "
+                f"({rb - ra} reads), single thread, {dt:.2f} s")
+        if spent > budget_s * 0.4 or s1 - s0 >= (max_sites or 1 << 62) or s1 >= origin + len(ref):
+            break
+        S = int(min(max(S * 2, budget_s * 0.6 * rate), 5_000_000))
+    return rate, desc
+
+
+def run_reference(args):
+    ws, rank, _ = _dist()
+    if rank != 0:
+        return 0
+    w = make_shard(args.config, 0, 1)
+    for _ in range(args.warmup):
+        cpu_oracle_rate(w, budget_s=1.0, max_sites=20_000)
+    vals = []
+    desc = ""
+    for _ in range(args.steps):
+        v, desc = cpu_oracle_rate(w, budget_s=args.ref_budget)
+        vals.append(v)
+    v = float(np.median(vals))
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": None,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": args.config, "sample": desc},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": desc},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def run_gpu(args):
+    import torch
+    from paper_conf_icpp_luzlwfl11_b200 import gsnp
+    ws, rank, local = _dist()
+    if ws != args.gpus:
+        args.gpus = ws
+    torch.cuda.set_device(local)
+    dist = None
+    if ws > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    w = make_shard(args.config, rank, ws)
+    S = len(w["ref"])
+    w0, w1 = int(w["origin"]), int(w["origin"]) + S
+    stream = torch.cuda.current_stream()
+    keys = ("pos", "len", "off", "bases", "quals", "strand", "hits")
+    host = {k: torch.from_numpy(np.ascontiguousarray(w[k])) for k in keys}
+    dev = {k: v.cuda() for k, v in host.items()}
+    torch.cuda.synchronize()
+    ctx = gsnp.Context.from_workload(w, device=local, stream=stream,
+                                     flags=gsnp.GSNP_RANK_SUM | gsnp.GSNP_TIMING)
+    counts = torch.zeros(64 * 256 * 16, dtype=torch.uint64, device="cuda")
+    out = torch.empty(40 * S, dtype=torch.uint8, device="cuda")
+    rd = gsnp.make_reads(dev)
+
+    def step():
+        ctx.calibrate_count(rd_dict, counts)
+        if dist is not None:
+            c64 = counts.view(torch.int64)
+            dist.all_reduce(c64)
+        ctx.calibrate_finalize(counts)
+        ctx.call_reads(rd, w0, w1, out)
+
+    rd_dict = dev
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    ctx.stage_times(reset=True)
+    l0 = ctx.launch_count()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    if dist is not None:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        ev0.record(stream)
+        for _ in range(args.steps):
+            step()
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    if dist is not None:
+        dist.barrier()
+    ms_total = ev0.elapsed_time(ev1)
+    launches = ctx.launch_count() - l0
+    st = ctx.stage_times(reset=True)
+    t = torch.tensor([ms_total], dtype=torch.float64, device="cuda")
+    if dist is not None:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_max = float(t.item())
+    ms_step = ms_max / args.steps
+    total_sites = S * ws
+    value = total_sites / (ms_step / 1e3)
+
+    # ---- e2e: same metric through the public API with host (pinned) inputs and outputs
+    pinned = {k: v.pin_memory() for k, v in host.items()}
+    out_h = torch.empty(40 * S, dtype=torch.uint8).pin_memory()
+    dev2 = {k: torch.empty_like(v, device="cuda") for k, v in host.items()}
+    rd2 = gsnp.make_reads(dev2)
+    h2d = sum(v.numel() * v.element_size() for v in pinned.values())
+    d2h = out_h.numel()
+
+    def e2e_step():
+        for k in keys:
+            dev2[k].copy_(pinned[k], non_blocking=True)
+        ctx.calibrate_count(dev2, counts)
+        if dist is not None:
+            dist.all_reduce(counts.view(torch.int64))
+        ctx.calibrate_finalize(counts)
+        ctx.call_reads(rd2, w0, w1, out)
+        out_h.copy_(out, non_blocking=True)
+
+    for _ in range(max(1, args.warmup // 2)):
+        e2e_step()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    n_e2e = max(2, min(args.steps, 5))
+    e0.record(stream)
+    for _ in range(n_e2e):
+        e2e_step()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    te = torch.tensor([e0.elapsed_time(e1) / n_e2e], dtype=torch.float64, device="cuda")
+    if dist is not None:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e_val = total_sites / (float(te.item()) / 1e3)
+    ok = bytes(out_h[:40 * 1000].numpy()) == bytes(out[:40 * 1000].cpu().numpy())
+
+    if rank != 0:
+        if dist is not None:
+            dist.destroy_process_group()
+        return 0
+    # ---- roofline of the dominant kernel (k_call_tile)
+    peak, peak_kind = _peaks()
+    call_ms, call_n = st["call_tile"]
+    nreads = int(len(w["pos"]))
+    nbases = int(w["off"][-1] - w["off"][0])
+    # algorithmic HBM bytes of one k_call_tile launch: read bases+quals (2 B/base), read metadata
+    # (pos 8 + len 2 + off 8 + strand 1 + hits 2 = 21 B/read), reference (1 B/site), records
+    # (40 B/site).  DESIGN.md §6.
+    alg_bytes = 2 * nbases + 21 * nreads + 1 * S + 40 * S
+    call_avg_ms = call_ms / max(call_n, 1)
+    achieved = alg_bytes / (call_avg_ms / 1e3) / 1e9
+    stage_share = {k: round(v[0] / max(ms_total, 1e-9), 4) for k, v in st.items()}
+    traffic = None
+    tr_path = os.path.join(ROOT, "profiles", "latest_call_tile_dram_bytes.json")
+    if os.path.exists(tr_path):
+        try:
+            traffic = json.load(open(tr_path)).get("bytes_per_launch")
+        except Exception:
+            traffic = None
+    cpu_v, cpu_desc = (None, None)
+    if not args.no_cpu:
+        cpu_v, cpu_desc = cpu_oracle_rate(w, budget_s=args.ref_budget)
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": args.config, "sites_per_gpu": S, "reads_per_gpu": nreads,
+                   "bases_per_gpu": nbases, "depth": synth_depth(args.config),
+                   "read_len": 100, "l2": "inputs (%.2f GB/GPU) > L2 126 MB; no flush" %
+                   (input_bytes(w) / 1e9), "parallelism": f"shard{ws}",
+                   "stage_ms_per_step": {k: round(v[0] / args.steps, 4) for k, v in st.items()},
+                   "stage_share": stage_share},
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
+                     "kernel": "k_call_tile", "alg_bytes_per_launch": alg_bytes,
+                     "launch_ms": call_avg_ms},
+        "cpu_baseline": ({"value": cpu_v, "unit": UNIT, "cores": 1, "kind": "oracle",
+                          "sample": cpu_desc} if cpu_v else None),
+        "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": h2d,
+                "d2h_bytes_per_step": d2h, "ms_per_step": float(te.item()), "check": ok},
+        "gpu_launches": launches,
+        "clocks": clk.summary(),
+    }
+    print(json.dumps(line), flush=True)
+    ctx.close()
+    if dist is not None:
+        dist.destroy_process_group()
+    return 0
+
+
+def synth_depth(name):
+    import synth
+    return synth.CONFIGS[name].depth
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--impl", default="gsnp", choices=["gsnp", "reference"])
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--ref-budget", type=float, default=15.0)
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_gpu(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

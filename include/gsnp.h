@@ -1,0 +1,177 @@
+/*
+ * gsnp.h — C ABI of libgsnp, the B200 (sm_100a) GSNP hot path.
+ *
+ * GSNP (Lu et al., ICPP 2011; /root/reference/PAPER.md, cited "P:L<line>") detects SNPs with the
+ * SOAPsnp Bayesian model: a calibration pass over all aligned reads (cal_p_matrix, P:L193-196,
+ * P:L714-727), then per window of sites (read_site): counting (§IV-B),
+ * likelihood = sort + comp (Alg. 4), posterior and output.  This
+ * library computes that path on one GPU; every step runs in its CUDA kernels.  Readings of what
+ * the paper leaves silent (R1..R15) are listed in DESIGN.md §3.
+ *
+ * Conventions for every call:
+ *  - Status: 0 = GSNP_OK, negative = error (below); never exit()/abort().  After an error the
+ *    context stays usable; gsnp_last_error() holds a one-line description.
+ *  - Ownership: every input pointer is borrowed for the duration of the call only.  The context
+ *    copies what it keeps (reference codes, known-SNP list, tables).  Outputs go to caller-owned
+ *    buffers, which may be host memory or device memory (detected per pointer).
+ *  - Concurrency: one context per device per process; a context is not thread-safe.  Work is
+ *    enqueued on params.stream (NULL = the legacy default stream); calls that return results to
+ *    the host synchronise that stream before returning.
+ *  - Base codes 0=A 1=C 2=T 3=G 4=N; genotype n = 0..9 is AA AC AT AG CC CT CG TT TG GG
+ *    (Alg. 4 lines 13-17).
+ */
+#ifndef GSNP_H
+#define GSNP_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define GSNP_ABI_VERSION 1u
+
+typedef int32_t gsnp_status;
+#define GSNP_OK 0
+#define GSNP_E_INVAL (-1)     /* NULL/invalid argument or parameter */
+#define GSNP_E_RANGE (-2)     /* value out of range: len > max_read_len, qual > q_max, base > 4,
+                                 strand > 1, hits == 0, read/window outside the reference */
+#define GSNP_E_UNSORTED (-3)  /* read positions decrease (input must be sorted) */
+#define GSNP_E_STATE (-4)     /* call order violated (gsnp_call before calibration) */
+#define GSNP_E_NOMEM (-5)     /* host or device allocation failed */
+#define GSNP_E_CUDA (-6)      /* CUDA runtime error (message in gsnp_last_error) */
+#define GSNP_E_CAPACITY (-7)  /* output buffer too small; *n_out holds the required count */
+
+#define GSNP_RANK_SUM 0x1u    /* apply the rank-sum test to heterozygous calls (reading R8) */
+#define GSNP_TIMING 0x2u      /* record per-stage device times with CUDA events (see below) */
+
+/* stages reported by gsnp_stage_times */
+#define GSNP_STAGE_VALIDATE 0     /* k_validate_reads */
+#define GSNP_STAGE_CALIB 1        /* k_calib_count (a1) */
+#define GSNP_STAGE_RANGES 2       /* k_tile_ranges (a3) */
+#define GSNP_STAGE_CALL 3         /* k_call_tile (a4..a8) */
+#define GSNP_STAGE_FINALIZE 4     /* host tables + upload (a2), wall time on the host */
+#define GSNP_N_STAGES 5
+
+typedef struct gsnp_ctx gsnp_ctx;  /* opaque; owned by the library until gsnp_destroy */
+
+typedef struct {
+    uint32_t abi_version;     /* must be GSNP_ABI_VERSION */
+    uint32_t max_read_len;    /* L, 1..256 (8-bit coord field); default 100 */
+    uint32_t q_max;           /* highest quality, <= 63 (6-bit score field); default 40 */
+    uint32_t calib_min_count; /* tau of the calibration estimator (R1); default 10 */
+    double het_novel;         /* novel heterozygote prior (R6); default 1e-3 */
+    double althom_novel;      /* novel alt-homozygote prior (R6); default 5e-4 */
+    double global_dep;        /* global dependency coefficient in (0,1] (R3); default 0.9 */
+    double pcr_dep;           /* PCR dependency coefficient in (0,1] (R3); default 0.5 */
+    uint32_t flags;           /* GSNP_RANK_SUM (default set) */
+    int32_t device;           /* CUDA device ordinal; default 0 */
+    void* stream;             /* cudaStream_t to enqueue on, or NULL; e.g. a torch stream */
+} gsnp_params;
+
+typedef struct {              /* the reference sequence (input file 2) */
+    const uint8_t* code;      /* n_sites codes 0..4, host memory */
+    uint64_t n_sites;
+    uint64_t origin;          /* global coordinate of code[0] (a shard's offset) */
+} gsnp_reference;
+
+typedef struct {              /* known SNPs with priors (input file 3) */
+    uint64_t n;
+    const uint64_t* pos;      /* strictly increasing global coordinates, host memory */
+    const double* prior10;    /* n x 10 linear priors (> 0), genotype order n = 0..9 */
+} gsnp_priors;
+
+typedef struct {              /* aligned reads sorted by position (input file 1) */
+    uint64_t n_reads;
+    const uint64_t* pos;      /* leftmost global coordinate, non-decreasing */
+    const uint16_t* len;      /* 1..max_read_len */
+    const uint64_t* off;      /* n_reads+1 offsets into bases/quals (base i of read r at off[r]+i);
+                                 off[0] need not be 0 */
+    const uint8_t* bases;     /* 0..4, reference-forward orientation (R11) */
+    const uint8_t* quals;     /* 0..q_max */
+    const uint8_t* strand;    /* 0 '+', 1 '-' */
+    const uint16_t* hits;     /* >= 1; 1 = uniquely aligned */
+    int32_t on_device;        /* 0: host arrays (copied by the library); 1: device arrays on the
+                                 context's device (e.g. torch CUDA tensors), used in place */
+} gsnp_reads;
+
+typedef struct {              /* 40 bytes: one output row (fields R9) */
+    uint64_t pos;             /* global coordinate */
+    uint8_t ref;              /* reference code */
+    uint8_t genotype;         /* 0..9, 255 = no call (ref N and depth 0) */
+    uint8_t quality;          /* consensus quality 0..99 (R9) */
+    uint8_t base1, base2;     /* best / second base, 4 = none (R9) */
+    uint8_t avgq1, avgq2;     /* mean quality of the unique base1/base2 observations */
+    uint8_t known;            /* 1 if the site is in the known-SNP list */
+    uint16_t cnt_uni1, cnt_all1, cnt_uni2, cnt_all2;  /* unique / all counts (saturating) */
+    uint32_t depth;           /* non-N aligned bases (all hits) */
+    float rank_p;             /* rank-sum p-value of het calls, else 1 (R8) */
+    float copy_num;           /* sum(hits) / depth (R9) */
+    float post1;              /* posterior probability of the called genotype (R7) */
+} gsnp_record;
+
+/* Fill *out with the defaults listed above. */
+gsnp_status gsnp_params_default(gsnp_params* out);
+
+/* Create a context on params->device: copies the reference and known-SNP list to the device and
+ * builds the adjust table (R3) on the host.  priors may be NULL (no known SNPs). */
+gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
+                        const gsnp_params* params, gsnp_ctx** out);
+
+/* Calibration = count (GPU histogram, a1) + finalize (host tables, a2).  Needs all reads before
+ * any window is called.  Reads must lie inside the reference. */
+gsnp_status gsnp_calibrate(gsnp_ctx* ctx, const gsnp_reads* reads);
+
+/* Multi-process split of gsnp_calibrate.  _count writes this shard's counts
+ * C[q][cyc][t][o] (uint64[64][256][4][4], index q<<12|cyc<<4|t<<2|o; host or device buffer).
+ * Count each read on exactly one rank.  The caller sums the buffers across ranks (e.g.
+ * torch.distributed.all_reduce) and passes the sum to _finalize, which builds the p matrix, the
+ * score table T (Alg. 3) and the priors on the host and uploads them. */
+gsnp_status gsnp_calibrate_count(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t* counts);
+gsnp_status gsnp_calibrate_finalize(gsnp_ctx* ctx, const uint64_t* counts);
+
+/* Call sites [w0, w1) (global coordinates inside the reference): one gsnp_record per site,
+ * written to out[0 .. w1-w0).  reads must include every read overlapping the window (the
+ * read-length halo: pos in [w0-L+1, w1)); bases outside [w0, w1) are ignored.  out may be host or
+ * device memory.  out_cap < w1-w0 -> GSNP_E_CAPACITY with *n_out = w1-w0. */
+gsnp_status gsnp_call(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1,
+                      gsnp_record* out, uint64_t out_cap, uint64_t* n_out);
+
+/* Debug dump of the same pipeline for [w0, w1) into HOST buffers (any may be NULL):
+ *   off[S+1]        u32 CSR offsets of each site's unique keys (S = w1-w0)
+ *   keys_built      u32 keys as the builder scattered them (per-site order unspecified)
+ *   keys_sorted     u32 keys after the sort (ascending)  — both sized off[S]
+ *   site_counters   u32[S][15] = depth, dep_uni, repeat, count_all[4], count_uni[4], q_sum[4]
+ *   L10, post10     f64[S][10] log10 likelihoods and posteriors
+ *   records         gsnp_record[S]
+ * Buffers for keys must hold at least the number of bases in reads. */
+gsnp_status gsnp_debug_window(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1,
+                              uint32_t* off, uint32_t* keys_built, uint32_t* keys_sorted,
+                              uint32_t* site_counters, double* L10, double* post10,
+                              gsnp_record* records);
+
+/* Copy the context's tables to host buffers (any may be NULL):
+ *   counts u64[64*256*16]; p_matrix f64[64*256*16] (index q<<12|coord<<4|allele<<2|base);
+ *   T f64[64*L*4*10] (index ((q*L+coord)*4+base)*10+n, Alg. 3); adj u8[64*adj_pcr*adj_g].
+ * dims (may be NULL) receives {L, adj_pcr, adj_g}. */
+gsnp_status gsnp_get_tables(gsnp_ctx* ctx, uint64_t* counts, double* p_matrix, double* T,
+                            uint8_t* adj, uint32_t* dims);
+
+/* Number of kernel launches this context has issued so far (for bench accounting). */
+uint64_t gsnp_launch_count(const gsnp_ctx* ctx);
+
+/* With GSNP_TIMING set in params.flags: accumulated milliseconds and launch counts per stage
+ * (GSNP_STAGE_*), measured with CUDA events recorded on params.stream around each launch
+ * (finalize: host wall time).  ms/launches may be NULL; n_stages <= GSNP_N_STAGES entries are
+ * written; reset != 0 clears the accumulators after reading. */
+gsnp_status gsnp_stage_times(gsnp_ctx* ctx, double* ms, uint64_t* launches, int n_stages,
+                             int reset);
+
+const char* gsnp_strerror(gsnp_status s);
+const char* gsnp_last_error(const gsnp_ctx* ctx);
+void gsnp_destroy(gsnp_ctx* ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GSNP_H */

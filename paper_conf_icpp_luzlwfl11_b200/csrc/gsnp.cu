@@ -1,0 +1,748 @@
+// gsnp.cu — libgsnp: the C ABI of include/gsnp.h (host orchestration + table builders) and the
+// sm_100a kernels of gsnp_kernels.cuh.  See DESIGN.md for the path, readings and roofline.
+//
+// Host arithmetic that feeds integer decisions (the adjust table, R3) or the score table T
+// (Alg. 3; built on the CPU for CPU/GPU consistency, §IV-G) is compiled
+// with -ffp-contract=off and uses glibc log10/pow.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "gsnp.h"
+#include "gsnp_kernels.cuh"
+
+using namespace gsnp_dev;
+
+namespace {
+
+template <typename T>
+struct DevBuf {  // grow-only device buffer
+    T* p = nullptr;
+    size_t n = 0;
+    cudaError_t ensure(size_t want) {
+        if (want <= n && p) return cudaSuccess;
+        if (p) cudaFree(p);
+        p = nullptr;
+        n = 0;
+        cudaError_t e = cudaMalloc(&p, std::max<size_t>(want, 1) * sizeof(T));
+        if (e == cudaSuccess) n = std::max<size_t>(want, 1);
+        return e;
+    }
+    void release() {
+        if (p) cudaFree(p);
+        p = nullptr;
+        n = 0;
+    }
+};
+
+const double kLog10Zero = 0.0;
+
+}  // namespace
+
+struct gsnp_ctx {
+    gsnp_params prm{};
+    cudaStream_t stream = nullptr;
+    std::string err;
+    // reference + known SNPs
+    uint64_t n_sites = 0, origin = 0;
+    DevBuf<uint8_t> ref;
+    DevBuf<uint32_t> known_bits;
+    DevBuf<uint64_t> known_pos;
+    DevBuf<double> known_lp;
+    uint64_t n_known = 0;
+    std::vector<uint64_t> h_known_pos;
+    // tables
+    std::vector<uint8_t> h_adj;
+    int adjP = 1, adjG = 1;
+    DevBuf<uint8_t> adj;
+    DevBuf<double> LP;
+    std::vector<uint64_t> h_counts;
+    std::vector<double> h_p;   // [64][256][4][4]
+    std::vector<double> h_T;   // [64][L][4][10]
+    DevBuf<double> T;
+    bool calibrated = false;
+    // scratch
+    DevBuf<int> d_err;
+    DevBuf<unsigned long long> d_counts;
+    DevBuf<uint64_t> tile_ra, tile_rb;
+    DevBuf<gsnp_record> rec;
+    // staged host reads
+    DevBuf<uint64_t> r_pos, r_off;
+    DevBuf<uint16_t> r_len, r_hits;
+    DevBuf<uint8_t> r_bases, r_quals, r_strand;
+    // debug
+    DevBuf<uint32_t> dbg_u32a, dbg_u32b, dbg_u32c, dbg_u32d, dbg_u32e;
+    DevBuf<double> dbg_f64a, dbg_f64b;
+    uint64_t launches = 0;
+    // per-stage timing (GSNP_TIMING)
+    struct Pending { int stage; cudaEvent_t a, b; };
+    std::vector<cudaEvent_t> ev_pool;
+    std::vector<Pending> pending;
+    double stage_ms[GSNP_N_STAGES] = {0, 0, 0, 0, 0};
+    uint64_t stage_n[GSNP_N_STAGES] = {0, 0, 0, 0, 0};
+    bool timing() const { return (prm.flags & GSNP_TIMING) != 0; }
+    cudaEvent_t ev() {
+        if (ev_pool.empty()) {
+            cudaEvent_t e;
+            cudaEventCreate(&e);
+            return e;
+        }
+        cudaEvent_t e = ev_pool.back();
+        ev_pool.pop_back();
+        return e;
+    }
+    // bracket one launch of a stage: call begin() before and end() after the launch
+    cudaEvent_t cur_a = nullptr;
+    void begin() {
+        if (!timing()) return;
+        cur_a = ev();
+        cudaEventRecord(cur_a, stream);
+    }
+    void end(int stage) {
+        if (!timing()) return;
+        cudaEvent_t b = ev();
+        cudaEventRecord(b, stream);
+        pending.push_back({stage, cur_a, b});
+        cur_a = nullptr;
+    }
+    // after a stream sync: fold completed pairs into the accumulators
+    void flush() {
+        for (auto& p : pending) {
+            float ms = 0;
+            if (cudaEventElapsedTime(&ms, p.a, p.b) == cudaSuccess) {
+                stage_ms[p.stage] += ms;
+                stage_n[p.stage] += 1;
+            } else {
+                cudaGetLastError();
+            }
+            ev_pool.push_back(p.a);
+            ev_pool.push_back(p.b);
+        }
+        pending.clear();
+    }
+};
+
+namespace {
+
+gsnp_status fail(gsnp_ctx* c, gsnp_status s, const char* fmt, ...) {
+    if (c) {
+        char buf[512];
+        va_list ap;
+        va_start(ap, fmt);
+        vsnprintf(buf, sizeof buf, fmt, ap);
+        va_end(ap);
+        c->err = buf;
+    }
+    return s;
+}
+
+#define CK(call)                                                                              \
+    do {                                                                                      \
+        cudaError_t e_ = (call);                                                              \
+        if (e_ != cudaSuccess)                                                                \
+            return fail(ctx, e_ == cudaErrorMemoryAllocation ? GSNP_E_NOMEM : GSNP_E_CUDA,    \
+                        "%s: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__); \
+    } while (0)
+
+bool is_device_ptr(const void* p) {
+    if (!p) return false;
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+// R3: q_adj = max(1, (int)(10^(log10 q + (pcr-1) log10 pcr_dep + g log10 global_dep) + 0.5))
+int adjust_expr(double lpd, double lgd, int q, int pcr, int g) {
+    double lq = log10((double)q);
+    double e = lq + (double)(pcr - 1) * lpd + (double)g * lgd;
+    int qa = (int)(pow(10.0, e) + 0.5);
+    return qa < 1 ? 1 : qa;
+}
+
+// Build adj[64][P][G].  The expression is non-increasing in pcr and g (coefficients <= 1), so
+// P = first pcr with adjust(63, P, 0) == 1 and G = first g with adjust(63, 1, G) == 1 bound
+// where it saturates at 1; beyond them every cell is 1 and indices clamp.
+gsnp_status build_adj(gsnp_ctx* ctx) {
+    const double lpd = log10(ctx->prm.pcr_dep), lgd = log10(ctx->prm.global_dep);
+    int P = 1, G = 1;
+    if (ctx->prm.pcr_dep < 1.0) {
+        while (adjust_expr(lpd, lgd, 63, P, 0) > 1) {
+            if (++P > 255) return fail(ctx, GSNP_E_INVAL, "pcr_dep too close to 1 (table > 255)");
+        }
+    }
+    if (ctx->prm.global_dep < 1.0) {
+        while (adjust_expr(lpd, lgd, 63, 1, G - 1) > 1) {
+            if (++G > 4096) return fail(ctx, GSNP_E_INVAL, "global_dep too close to 1");
+        }
+    } else {
+        G = 1;
+    }
+    // with global_dep == 1, g has no effect (G = 1); with pcr_dep == 1, P = 1.
+    ctx->adjP = P;
+    ctx->adjG = G;
+    ctx->h_adj.assign((size_t)64 * P * G, 1);
+    for (int q = 0; q < 64; ++q)
+        for (int p = 1; p <= P; ++p)
+            for (int g = 0; g < G; ++g)
+                ctx->h_adj[((size_t)q * P + (p - 1)) * G + g] = (uint8_t)adjust_expr(lpd, lgd, q, p, g);
+    return GSNP_OK;
+}
+
+// R1 estimator (host): p[q][c][t][o], index q<<12 | c<<4 | t<<2 | o.
+void estimate_p(const gsnp_params& prm, const uint64_t* C, std::vector<double>& p) {
+    const int L = (int)prm.max_read_len;
+    const double tau = (double)prm.calib_min_count;
+    p.assign((size_t)64 * 256 * 16, 0.0);
+    for (int q = 0; q < 64; ++q) {
+        double tot = 0, mm = 0;
+        for (int c = 0; c < L; ++c)
+            for (int t = 0; t < 4; ++t)
+                for (int o = 0; o < 4; ++o) {
+                    double v = (double)C[q << 12 | c << 4 | t << 2 | o];
+                    tot += v;
+                    if (t != o) mm += v;
+                }
+        for (int t = 0; t < 4; ++t) {
+            double npool[4] = {0, 0, 0, 0}, Npool = 0;
+            for (int c = 0; c < L; ++c)
+                for (int o = 0; o < 4; ++o) {
+                    double v = (double)C[q << 12 | c << 4 | t << 2 | o];
+                    npool[o] += v;
+                    Npool += v;
+                }
+            for (int c = 0; c < L; ++c) {
+                double Nct = 0;
+                for (int o = 0; o < 4; ++o) Nct += (double)C[q << 12 | c << 4 | t << 2 | o];
+                for (int o = 0; o < 4; ++o) {
+                    double n = (double)C[q << 12 | c << 4 | t << 2 | o], v;
+                    if (n > tau) v = n / Nct;
+                    else if (npool[o] > tau) v = npool[o] / Npool;
+                    else if (mm > 0 && mm < tot) v = (o == t) ? (tot - mm) / tot : mm / (3.0 * tot);
+                    else {
+                        double e = pow(10.0, -(double)q / 10.0);
+                        if (e > 0.75) e = 0.75;
+                        v = (o == t) ? 1.0 - e : e / 3.0;
+                    }
+                    p[q << 12 | c << 4 | t << 2 | o] = v;
+                }
+            }
+        }
+    }
+}
+
+// Alg. 3 score table: T[qa][c][b][n] = log10(0.5 p[qa][c][a1][b] + 0.5 p[qa][c][a2][b]),
+// the value Alg. 2 returns; built once on the CPU (§IV-G).  Rows qa = 1..63 (adjust >= 1).
+void build_T(int L, const std::vector<double>& p, std::vector<double>& T) {
+    static const int A1[10] = {0, 0, 0, 0, 1, 1, 1, 2, 2, 3};
+    static const int A2[10] = {0, 1, 2, 3, 1, 2, 3, 2, 3, 3};
+    T.assign((size_t)64 * L * 4 * 10, 0.0);
+    auto work = [&](int q0, int q1) {
+        for (int qa = q0; qa < q1; ++qa)
+            for (int c = 0; c < L; ++c)
+                for (int b = 0; b < 4; ++b)
+                    for (int n = 0; n < 10; ++n) {
+                        int p1 = qa << 12 | c << 4 | A1[n] << 2 | b;
+                        int p2 = qa << 12 | c << 4 | A2[n] << 2 | b;
+                        T[(((size_t)qa * L + c) * 4 + b) * 10 + n] = log10(0.5 * p[p1] + 0.5 * p[p2]);
+                    }
+    };
+    unsigned nt = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+    std::vector<std::thread> th;
+    int per = (64 + (int)nt - 1) / (int)nt;
+    for (unsigned i = 0; i < nt; ++i) {
+        int q0 = (int)i * per, q1 = std::min(64, q0 + per);
+        if (q0 < q1) th.emplace_back(work, q0, q1);
+    }
+    for (auto& t : th) t.join();
+}
+
+gsnp_status check_params(gsnp_ctx* ctx, const gsnp_params* p) {
+    if (!p || p->abi_version != GSNP_ABI_VERSION) return fail(ctx, GSNP_E_INVAL, "bad params/abi");
+    if (p->max_read_len < 1 || p->max_read_len > 256) return fail(ctx, GSNP_E_INVAL, "max_read_len");
+    if (p->q_max > 63) return fail(ctx, GSNP_E_INVAL, "q_max > 63");
+    if (!(p->global_dep > 0 && p->global_dep <= 1) || !(p->pcr_dep > 0 && p->pcr_dep <= 1))
+        return fail(ctx, GSNP_E_INVAL, "dependency coefficients must be in (0,1]");
+    if (!(p->het_novel > 0) || !(p->althom_novel > 0)) return fail(ctx, GSNP_E_INVAL, "priors");
+    return GSNP_OK;
+}
+
+// Stage reads on the device (host arrays are copied; device arrays used in place).
+gsnp_status stage_reads(gsnp_ctx* ctx, const gsnp_reads* r, DevReads& d) {
+    if (!r) return fail(ctx, GSNP_E_INVAL, "reads == NULL");
+    d.n = r->n_reads;
+    if (r->n_reads == 0) {
+        d.pos = nullptr; d.len = nullptr; d.off = nullptr; d.bases = nullptr; d.quals = nullptr;
+        d.strand = nullptr; d.hits = nullptr; d.off0 = 0;
+        return GSNP_OK;
+    }
+    if (!r->pos || !r->len || !r->off || !r->bases || !r->quals || !r->strand || !r->hits)
+        return fail(ctx, GSNP_E_INVAL, "NULL read array");
+    if (r->on_device) {
+        d.pos = r->pos; d.len = r->len; d.off = r->off; d.bases = r->bases; d.quals = r->quals;
+        d.strand = r->strand; d.hits = r->hits; d.off0 = 0;
+        return GSNP_OK;
+    }
+    const uint64_t n = r->n_reads;
+    const uint64_t o0 = r->off[0], o1 = r->off[n];
+    if (o1 < o0) return fail(ctx, GSNP_E_RANGE, "off[n] < off[0]");
+    const uint64_t nb = o1 - o0;
+    cudaStream_t s = ctx->stream;
+    CK(ctx->r_pos.ensure(n));
+    CK(ctx->r_off.ensure(n + 1));
+    CK(ctx->r_len.ensure(n));
+    CK(ctx->r_hits.ensure(n));
+    CK(ctx->r_strand.ensure(n));
+    CK(ctx->r_bases.ensure(nb));
+    CK(ctx->r_quals.ensure(nb));
+    CK(cudaMemcpyAsync(ctx->r_pos.p, r->pos, n * 8, cudaMemcpyHostToDevice, s));
+    CK(cudaMemcpyAsync(ctx->r_off.p, r->off, (n + 1) * 8, cudaMemcpyHostToDevice, s));
+    CK(cudaMemcpyAsync(ctx->r_len.p, r->len, n * 2, cudaMemcpyHostToDevice, s));
+    CK(cudaMemcpyAsync(ctx->r_hits.p, r->hits, n * 2, cudaMemcpyHostToDevice, s));
+    CK(cudaMemcpyAsync(ctx->r_strand.p, r->strand, n, cudaMemcpyHostToDevice, s));
+    CK(cudaMemcpyAsync(ctx->r_bases.p, r->bases + o0, nb, cudaMemcpyHostToDevice, s));
+    CK(cudaMemcpyAsync(ctx->r_quals.p, r->quals + o0, nb, cudaMemcpyHostToDevice, s));
+    d.pos = ctx->r_pos.p; d.len = ctx->r_len.p; d.off = ctx->r_off.p; d.bases = ctx->r_bases.p;
+    d.quals = ctx->r_quals.p; d.strand = ctx->r_strand.p; d.hits = ctx->r_hits.p; d.off0 = o0;
+    return GSNP_OK;
+}
+
+gsnp_status map_err(gsnp_ctx* ctx, int e) {
+    if (!e) return GSNP_OK;
+    if (e & ERR_UNSORTED) return fail(ctx, GSNP_E_UNSORTED, "read positions decrease");
+    if (e & (ERR_RANGE | ERR_QUAL))
+        return fail(ctx, GSNP_E_RANGE, "read value out of range (len/base/qual/strand/hits/pos)");
+    if (e & ERR_DEEP)
+        return fail(ctx, GSNP_E_CAPACITY, "a site's unique depth exceeds the shared-memory key buffer");
+    return fail(ctx, GSNP_E_CUDA, "device error flag %d", e);
+}
+
+gsnp_status launch_validate(gsnp_ctx* ctx, const DevReads& d) {
+    if (d.n == 0) return GSNP_OK;
+    unsigned blocks = (unsigned)((d.n + 255) / 256);
+    ctx->begin();
+    k_validate_reads<<<blocks, 256, 0, ctx->stream>>>(d, ctx->origin, ctx->n_sites,
+                                                      (int)ctx->prm.max_read_len, ctx->d_err.p);
+    ctx->end(GSNP_STAGE_VALIDATE);
+    ctx->launches++;
+    CK(cudaGetLastError());
+    return GSNP_OK;
+}
+
+int g_num_sms = 0;
+
+gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w1,
+                       gsnp_record* d_out, CallArgs& A) {
+    cudaStream_t s = ctx->stream;
+    const uint64_t n_tiles = (w1 - w0 + TS - 1) / TS;
+    const uint64_t n_groups = (w1 - w0 + 31) / 32;
+    if (n_tiles == 0) return GSNP_OK;
+    CK(ctx->tile_ra.ensure(n_groups));
+    CK(ctx->tile_rb.ensure(n_groups));
+    if (d.n) {
+        ctx->begin();
+        k_tile_ranges<<<(unsigned)((n_groups + 255) / 256), 256, 0, s>>>(
+            d.pos, d.n, w0, w1, (int)ctx->prm.max_read_len, n_groups, ctx->tile_ra.p,
+            ctx->tile_rb.p);
+        ctx->end(GSNP_STAGE_RANGES);
+        ctx->launches++;
+    } else {
+        CK(cudaMemsetAsync(ctx->tile_ra.p, 0, n_groups * 8, s));
+        CK(cudaMemsetAsync(ctx->tile_rb.p, 0, n_groups * 8, s));
+    }
+    A.R = d;
+    A.ref = ctx->ref.p;
+    A.origin = ctx->origin;
+    A.n_sites = ctx->n_sites;
+    A.known_bits = ctx->known_bits.p;
+    A.known_pos = ctx->known_pos.p;
+    A.known_lp = ctx->known_lp.p;
+    A.n_known = ctx->n_known;
+    A.LP = ctx->LP.p;
+    A.T = ctx->T.p;
+    A.adj = ctx->adj.p;
+    A.adjP = ctx->adjP;
+    A.adjG = ctx->adjG;
+    A.L = (int)ctx->prm.max_read_len;
+    A.q_max = (int)ctx->prm.q_max;
+    A.flags = ctx->prm.flags;
+    A.w0 = w0;
+    A.w1 = w1;
+    A.tile_ra = ctx->tile_ra.p;
+    A.tile_rb = ctx->tile_rb.p;
+    A.out = d_out;
+    A.err = ctx->d_err.p;
+    const size_t smem = call_smem_bytes(A.L, nullptr, nullptr);
+    CK(cudaFuncSetAttribute(k_call_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    ctx->begin();
+    k_call_tile<<<(unsigned)n_tiles, NT, smem, s>>>(A);
+    ctx->end(GSNP_STAGE_CALL);
+    ctx->launches++;
+    CK(cudaGetLastError());
+    return GSNP_OK;
+}
+
+gsnp_status read_err(gsnp_ctx* ctx) {
+    int h = 0;
+    CK(cudaMemcpyAsync(&h, ctx->d_err.p, sizeof(int), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    ctx->flush();
+    return map_err(ctx, h);
+}
+
+gsnp_status count_impl(gsnp_ctx* ctx, const gsnp_reads* reads) {
+    DevReads d;
+    gsnp_status st = stage_reads(ctx, reads, d);
+    if (st) return st;
+    cudaStream_t s = ctx->stream;
+    CK(ctx->d_counts.ensure(64 * 256 * 16));
+    CK(cudaMemsetAsync(ctx->d_counts.p, 0, 64 * 256 * 16 * 8, s));
+    CK(cudaMemsetAsync(ctx->d_err.p, 0, sizeof(int), s));
+    if ((st = launch_validate(ctx, d))) return st;
+    if (d.n) {
+        CalibArgs A;
+        A.R = d;
+        A.ref = ctx->ref.p;
+        A.origin = ctx->origin;
+        A.n_sites = ctx->n_sites;
+        A.known_bits = ctx->known_bits.p;
+        A.L = (int)ctx->prm.max_read_len;
+        A.q_max = (int)ctx->prm.q_max;
+        A.C = ctx->d_counts.p;
+        A.err = ctx->d_err.p;
+        size_t diag = (size_t)(A.q_max + 1) * A.L * 4 * 4;
+        A.smem_diag = diag <= 160 * 1024;
+        size_t smem = A.smem_diag ? diag : 0;
+        int per_sm = smem <= 72 * 1024 ? 3 : smem <= 110 * 1024 ? 2 : 1;
+        unsigned grid = (unsigned)std::min<uint64_t>((uint64_t)g_num_sms * per_sm, (d.n + 63) / 64);
+        grid = std::max(grid, 1u);
+        CK(cudaFuncSetAttribute(k_calib_count, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        ctx->begin();
+        k_calib_count<<<grid, NT, smem, s>>>(A);
+        ctx->end(GSNP_STAGE_CALIB);
+        ctx->launches++;
+        CK(cudaGetLastError());
+    }
+    return GSNP_OK;
+}
+
+gsnp_status finalize_impl(gsnp_ctx* ctx, const uint64_t* counts_host) {
+    auto t0 = std::chrono::steady_clock::now();
+    ctx->h_counts.assign(counts_host, counts_host + 64 * 256 * 16);
+    estimate_p(ctx->prm, ctx->h_counts.data(), ctx->h_p);
+    build_T((int)ctx->prm.max_read_len, ctx->h_p, ctx->h_T);
+    CK(ctx->T.ensure(ctx->h_T.size()));
+    CK(cudaMemcpyAsync(ctx->T.p, ctx->h_T.data(), ctx->h_T.size() * 8, cudaMemcpyHostToDevice,
+                       ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    ctx->calibrated = true;
+    if (ctx->timing()) {
+        ctx->stage_ms[GSNP_STAGE_FINALIZE] +=
+            std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+        ctx->stage_n[GSNP_STAGE_FINALIZE] += 1;
+    }
+    return GSNP_OK;
+}
+
+}  // namespace
+
+// ============================================================================ public ABI
+extern "C" {
+
+gsnp_status gsnp_params_default(gsnp_params* out) {
+    if (!out) return GSNP_E_INVAL;
+    memset(out, 0, sizeof *out);
+    out->abi_version = GSNP_ABI_VERSION;
+    out->max_read_len = 100;
+    out->q_max = 40;
+    out->calib_min_count = 10;
+    out->het_novel = 1e-3;
+    out->althom_novel = 5e-4;
+    out->global_dep = 0.9;
+    out->pcr_dep = 0.5;
+    out->flags = GSNP_RANK_SUM;
+    out->device = 0;
+    out->stream = nullptr;
+    return GSNP_OK;
+}
+
+gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
+                        const gsnp_params* params, gsnp_ctx** out) {
+    if (!out) return GSNP_E_INVAL;
+    *out = nullptr;
+    if (!ref || !ref->code || ref->n_sites == 0) return GSNP_E_INVAL;
+    gsnp_ctx* ctx = new (std::nothrow) gsnp_ctx();
+    if (!ctx) return GSNP_E_NOMEM;
+    gsnp_status st = check_params(ctx, params);
+    if (st) { delete ctx; return st; }
+    ctx->prm = *params;
+    ctx->stream = (cudaStream_t)params->stream;
+    auto bail = [&](gsnp_status s) { gsnp_destroy(ctx); return s; };
+    if (cudaSetDevice(params->device) != cudaSuccess) { cudaGetLastError(); return bail(GSNP_E_CUDA); }
+    if (!g_num_sms) {
+        cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, params->device);
+        if (g_num_sms <= 0) g_num_sms = 148;
+    }
+    ctx->n_sites = ref->n_sites;
+    ctx->origin = ref->origin;
+    for (uint64_t i = 0; i < ref->n_sites; ++i)
+        if (ref->code[i] > 4) return bail(GSNP_E_RANGE);
+    // known SNPs: sorted positions, log10 prior rows (C6), site bitmap
+    uint64_t nk = priors ? priors->n : 0;
+    std::vector<double> lp(std::max<uint64_t>(nk, 1) * 10);
+    std::vector<uint32_t> bits((ref->n_sites + 31) / 32 + 1, 0u);
+    ctx->h_known_pos.assign(nk, 0);
+    for (uint64_t k = 0; k < nk; ++k) {
+        uint64_t p = priors->pos[k];
+        if (k && p <= priors->pos[k - 1]) return bail(GSNP_E_UNSORTED);
+        if (p < ref->origin || p >= ref->origin + ref->n_sites) return bail(GSNP_E_RANGE);
+        for (int n = 0; n < 10; ++n) {
+            double v = priors->prior10[k * 10 + n];
+            if (!(v > 0)) return bail(GSNP_E_RANGE);
+            lp[k * 10 + n] = log10(v);
+        }
+        uint64_t rs = p - ref->origin;
+        bits[rs >> 5] |= 1u << (rs & 31);
+        ctx->h_known_pos[k] = p;
+    }
+    ctx->n_known = nk;
+    // novel log10 priors per reference code (R6); ref N: flat
+    double LP[50];
+    static const int A1[10] = {0, 0, 0, 0, 1, 1, 1, 2, 2, 3};
+    static const int A2[10] = {0, 1, 2, 3, 1, 2, 3, 2, 3, 3};
+    for (int r = 0; r < 5; ++r)
+        for (int n = 0; n < 10; ++n) {
+            double v;
+            if (r == 4) { LP[r * 10 + n] = kLog10Zero; continue; }
+            if (A1[n] == r && A2[n] == r) v = 1.0;
+            else if (A1[n] == r || A2[n] == r) v = params->het_novel;
+            else if (A1[n] == A2[n]) v = params->althom_novel;
+            else v = params->het_novel * params->althom_novel;
+            LP[r * 10 + n] = log10(v);
+        }
+    if ((st = build_adj(ctx))) return bail(st);
+    gsnp_ctx* c = ctx;
+#define CKC(x) do { if ((x) != cudaSuccess) { cudaGetLastError(); return bail(fail(c, GSNP_E_CUDA, "%s", #x)); } } while (0)
+    CKC(ctx->ref.ensure(ref->n_sites));
+    CKC(cudaMemcpy(ctx->ref.p, ref->code, ref->n_sites, cudaMemcpyHostToDevice));
+    CKC(ctx->known_bits.ensure(bits.size()));
+    CKC(cudaMemcpy(ctx->known_bits.p, bits.data(), bits.size() * 4, cudaMemcpyHostToDevice));
+    CKC(ctx->known_pos.ensure(std::max<uint64_t>(nk, 1)));
+    if (nk) CKC(cudaMemcpy(ctx->known_pos.p, ctx->h_known_pos.data(), nk * 8, cudaMemcpyHostToDevice));
+    CKC(ctx->known_lp.ensure(lp.size()));
+    CKC(cudaMemcpy(ctx->known_lp.p, lp.data(), lp.size() * 8, cudaMemcpyHostToDevice));
+    CKC(ctx->LP.ensure(50));
+    CKC(cudaMemcpy(ctx->LP.p, LP, sizeof LP, cudaMemcpyHostToDevice));
+    CKC(ctx->adj.ensure(ctx->h_adj.size()));
+    CKC(cudaMemcpy(ctx->adj.p, ctx->h_adj.data(), ctx->h_adj.size(), cudaMemcpyHostToDevice));
+    CKC(ctx->d_err.ensure(1));
+#undef CKC
+    *out = ctx;
+    return GSNP_OK;
+}
+
+gsnp_status gsnp_calibrate_count(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t* counts) {
+    if (!ctx || !counts) return GSNP_E_INVAL;
+    if (cudaSetDevice(ctx->prm.device) != cudaSuccess) return fail(ctx, GSNP_E_CUDA, "set device");
+    gsnp_status st = count_impl(ctx, reads);
+    if (st) return st;
+    if ((st = read_err(ctx))) return st;
+    cudaMemcpyKind kind = is_device_ptr(counts) ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost;
+    CK(cudaMemcpyAsync(counts, ctx->d_counts.p, 64 * 256 * 16 * 8, kind, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    return GSNP_OK;
+}
+
+gsnp_status gsnp_calibrate_finalize(gsnp_ctx* ctx, const uint64_t* counts) {
+    if (!ctx || !counts) return GSNP_E_INVAL;
+    if (cudaSetDevice(ctx->prm.device) != cudaSuccess) return fail(ctx, GSNP_E_CUDA, "set device");
+    std::vector<uint64_t> h(64 * 256 * 16);
+    if (is_device_ptr(counts)) {
+        CK(cudaMemcpyAsync(h.data(), counts, h.size() * 8, cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+    } else {
+        memcpy(h.data(), counts, h.size() * 8);
+    }
+    return finalize_impl(ctx, h.data());
+}
+
+gsnp_status gsnp_calibrate(gsnp_ctx* ctx, const gsnp_reads* reads) {
+    if (!ctx) return GSNP_E_INVAL;
+    if (cudaSetDevice(ctx->prm.device) != cudaSuccess) return fail(ctx, GSNP_E_CUDA, "set device");
+    gsnp_status st = count_impl(ctx, reads);
+    if (st) return st;
+    if ((st = read_err(ctx))) return st;
+    std::vector<uint64_t> h(64 * 256 * 16);
+    CK(cudaMemcpyAsync(h.data(), ctx->d_counts.p, h.size() * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    return finalize_impl(ctx, h.data());
+}
+
+static gsnp_status check_window(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1) {
+    if (!ctx->calibrated) return fail(ctx, GSNP_E_STATE, "gsnp_call before calibration");
+    if (!reads) return fail(ctx, GSNP_E_INVAL, "reads == NULL");
+    if (w1 < w0 || w0 < ctx->origin || w1 > ctx->origin + ctx->n_sites)
+        return fail(ctx, GSNP_E_RANGE, "window outside the reference");
+    return GSNP_OK;
+}
+
+gsnp_status gsnp_call(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1,
+                      gsnp_record* out, uint64_t out_cap, uint64_t* n_out) {
+    if (!ctx) return GSNP_E_INVAL;
+    if (cudaSetDevice(ctx->prm.device) != cudaSuccess) return fail(ctx, GSNP_E_CUDA, "set device");
+    gsnp_status st = check_window(ctx, reads, w0, w1);
+    if (st) return st;
+    const uint64_t S = w1 - w0;
+    if (n_out) *n_out = S;
+    if (out_cap < S) return fail(ctx, GSNP_E_CAPACITY, "out_cap %llu < %llu", (unsigned long long)out_cap,
+                                 (unsigned long long)S);
+    if (S && !out) return fail(ctx, GSNP_E_INVAL, "out == NULL");
+    if (S == 0) return GSNP_OK;
+    DevReads d;
+    if ((st = stage_reads(ctx, reads, d))) return st;
+    CK(cudaMemsetAsync(ctx->d_err.p, 0, sizeof(int), ctx->stream));
+    if ((st = launch_validate(ctx, d))) return st;
+    const bool dev_out = is_device_ptr(out);
+    gsnp_record* d_out = out;
+    if (!dev_out) {
+        CK(ctx->rec.ensure(S));
+        d_out = ctx->rec.p;
+    }
+    CallArgs A;
+    memset(&A, 0, sizeof A);
+    if ((st = run_window(ctx, d, w0, w1, d_out, A))) return st;
+    if (!dev_out)
+        CK(cudaMemcpyAsync(out, d_out, S * sizeof(gsnp_record), cudaMemcpyDeviceToHost, ctx->stream));
+    return read_err(ctx);
+}
+
+gsnp_status gsnp_debug_window(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1,
+                              uint32_t* off, uint32_t* keys_built, uint32_t* keys_sorted,
+                              uint32_t* site_counters, double* L10, double* post10,
+                              gsnp_record* records) {
+    if (!ctx) return GSNP_E_INVAL;
+    if (cudaSetDevice(ctx->prm.device) != cudaSuccess) return fail(ctx, GSNP_E_CUDA, "set device");
+    gsnp_status st = check_window(ctx, reads, w0, w1);
+    if (st) return st;
+    const uint64_t S = w1 - w0;
+    if (S == 0) return GSNP_OK;
+    cudaStream_t s = ctx->stream;
+    DevReads d;
+    if ((st = stage_reads(ctx, reads, d))) return st;
+    CK(cudaMemsetAsync(ctx->d_err.p, 0, sizeof(int), s));
+    if ((st = launch_validate(ctx, d))) return st;
+    // pass 1: unique keys per site -> CSR offsets (host scan)
+    CK(ctx->dbg_u32a.ensure(S));
+    CK(ctx->rec.ensure(S));
+    CallArgs A;
+    memset(&A, 0, sizeof A);
+    A.count_only = 1;
+    A.dbg_nuni = ctx->dbg_u32a.p;
+    if ((st = run_window(ctx, d, w0, w1, ctx->rec.p, A))) return st;
+    std::vector<uint32_t> nuni(S), hoff(S + 1);
+    CK(cudaMemcpyAsync(nuni.data(), ctx->dbg_u32a.p, S * 4, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if ((st = read_err(ctx))) return st;
+    hoff[0] = 0;
+    for (uint64_t i = 0; i < S; ++i) hoff[i + 1] = hoff[i] + nuni[i];
+    const uint64_t K = hoff[S];
+    CK(ctx->dbg_u32b.ensure(S + 1));
+    CK(ctx->dbg_u32c.ensure(std::max<uint64_t>(K, 1)));
+    CK(ctx->dbg_u32d.ensure(std::max<uint64_t>(K, 1)));
+    CK(ctx->dbg_u32e.ensure(S * 15));
+    CK(ctx->dbg_f64a.ensure(S * 10));
+    CK(ctx->dbg_f64b.ensure(S * 10));
+    CK(cudaMemcpyAsync(ctx->dbg_u32b.p, hoff.data(), (S + 1) * 4, cudaMemcpyHostToDevice, s));
+    memset(&A, 0, sizeof A);
+    A.dbg_off = ctx->dbg_u32b.p;
+    A.dbg_keys_built = ctx->dbg_u32c.p;
+    A.dbg_keys_sorted = ctx->dbg_u32d.p;
+    A.dbg_counters = ctx->dbg_u32e.p;
+    A.dbg_L10 = ctx->dbg_f64a.p;
+    A.dbg_post10 = ctx->dbg_f64b.p;
+    if ((st = run_window(ctx, d, w0, w1, ctx->rec.p, A))) return st;
+    if ((st = read_err(ctx))) return st;
+    if (off) memcpy(off, hoff.data(), (S + 1) * 4);
+    if (keys_built && K) CK(cudaMemcpyAsync(keys_built, ctx->dbg_u32c.p, K * 4, cudaMemcpyDeviceToHost, s));
+    if (keys_sorted && K) CK(cudaMemcpyAsync(keys_sorted, ctx->dbg_u32d.p, K * 4, cudaMemcpyDeviceToHost, s));
+    if (site_counters) CK(cudaMemcpyAsync(site_counters, ctx->dbg_u32e.p, S * 60, cudaMemcpyDeviceToHost, s));
+    if (L10) CK(cudaMemcpyAsync(L10, ctx->dbg_f64a.p, S * 80, cudaMemcpyDeviceToHost, s));
+    if (post10) CK(cudaMemcpyAsync(post10, ctx->dbg_f64b.p, S * 80, cudaMemcpyDeviceToHost, s));
+    if (records) CK(cudaMemcpyAsync(records, ctx->rec.p, S * sizeof(gsnp_record), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    return GSNP_OK;
+}
+
+gsnp_status gsnp_get_tables(gsnp_ctx* ctx, uint64_t* counts, double* p_matrix, double* T,
+                            uint8_t* adj, uint32_t* dims) {
+    if (!ctx) return GSNP_E_INVAL;
+    if (dims) {
+        dims[0] = ctx->prm.max_read_len;
+        dims[1] = (uint32_t)ctx->adjP;
+        dims[2] = (uint32_t)ctx->adjG;
+    }
+    if (adj) memcpy(adj, ctx->h_adj.data(), ctx->h_adj.size());
+    if ((counts || p_matrix || T) && !ctx->calibrated) return fail(ctx, GSNP_E_STATE, "not calibrated");
+    if (counts) memcpy(counts, ctx->h_counts.data(), ctx->h_counts.size() * 8);
+    if (p_matrix) memcpy(p_matrix, ctx->h_p.data(), ctx->h_p.size() * 8);
+    if (T) memcpy(T, ctx->h_T.data(), ctx->h_T.size() * 8);
+    return GSNP_OK;
+}
+
+uint64_t gsnp_launch_count(const gsnp_ctx* ctx) { return ctx ? ctx->launches : 0; }
+
+gsnp_status gsnp_stage_times(gsnp_ctx* ctx, double* ms, uint64_t* launches, int n_stages,
+                             int reset) {
+    if (!ctx || n_stages < 0) return GSNP_E_INVAL;
+    ctx->flush();
+    for (int i = 0; i < n_stages && i < GSNP_N_STAGES; ++i) {
+        if (ms) ms[i] = ctx->stage_ms[i];
+        if (launches) launches[i] = ctx->stage_n[i];
+    }
+    if (reset)
+        for (int i = 0; i < GSNP_N_STAGES; ++i) { ctx->stage_ms[i] = 0; ctx->stage_n[i] = 0; }
+    return GSNP_OK;
+}
+
+const char* gsnp_strerror(gsnp_status s) {
+    switch (s) {
+        case GSNP_OK: return "ok";
+        case GSNP_E_INVAL: return "invalid argument";
+        case GSNP_E_RANGE: return "value out of range";
+        case GSNP_E_UNSORTED: return "reads not sorted by position";
+        case GSNP_E_STATE: return "call order violated";
+        case GSNP_E_NOMEM: return "out of memory";
+        case GSNP_E_CUDA: return "CUDA error";
+        case GSNP_E_CAPACITY: return "capacity exceeded";
+        default: return "unknown status";
+    }
+}
+
+const char* gsnp_last_error(const gsnp_ctx* ctx) { return ctx ? ctx->err.c_str() : ""; }
+
+void gsnp_destroy(gsnp_ctx* ctx) {
+    if (!ctx) return;
+    cudaSetDevice(ctx->prm.device);
+    ctx->ref.release(); ctx->known_bits.release(); ctx->known_pos.release(); ctx->known_lp.release();
+    ctx->adj.release(); ctx->LP.release(); ctx->T.release(); ctx->d_err.release();
+    ctx->d_counts.release(); ctx->tile_ra.release(); ctx->tile_rb.release(); ctx->rec.release();
+    ctx->r_pos.release(); ctx->r_off.release(); ctx->r_len.release(); ctx->r_hits.release();
+    ctx->r_bases.release(); ctx->r_quals.release(); ctx->r_strand.release();
+    ctx->dbg_u32a.release(); ctx->dbg_u32b.release(); ctx->dbg_u32c.release();
+    ctx->dbg_u32d.release(); ctx->dbg_u32e.release(); ctx->dbg_f64a.release(); ctx->dbg_f64b.release();
+    for (auto& p : ctx->pending) { cudaEventDestroy(p.a); cudaEventDestroy(p.b); }
+    for (auto e : ctx->ev_pool) cudaEventDestroy(e);
+    delete ctx;
+}
+
+}  // extern "C"

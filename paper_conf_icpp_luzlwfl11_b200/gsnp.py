@@ -1,0 +1,318 @@
+"""Thin ctypes binding of libgsnp (include/gsnp.h).  Argument marshalling only: every step of the
+hot path runs in the library's CUDA kernels.  Arrays may be numpy (host) or torch tensors
+(host or CUDA; CUDA tensors are used in place).  There is no fallback: if ``libgsnp.so`` is
+missing the import fails (run ``__graft_entry__.build()``).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libgsnp.so")
+
+GSNP_ABI_VERSION = 1
+GSNP_RANK_SUM = 0x1
+GSNP_TIMING = 0x2
+STAGES = ("validate", "calib_count", "tile_ranges", "call_tile", "finalize")
+STATUS = {0: "GSNP_OK", -1: "GSNP_E_INVAL", -2: "GSNP_E_RANGE", -3: "GSNP_E_UNSORTED",
+          -4: "GSNP_E_STATE", -5: "GSNP_E_NOMEM", -6: "GSNP_E_CUDA", -7: "GSNP_E_CAPACITY"}
+
+# exported symbols declared in include/gsnp.h
+SYMBOLS = ("gsnp_params_default", "gsnp_create", "gsnp_calibrate", "gsnp_calibrate_count",
+           "gsnp_calibrate_finalize", "gsnp_call", "gsnp_debug_window", "gsnp_get_tables",
+           "gsnp_launch_count", "gsnp_stage_times", "gsnp_strerror", "gsnp_last_error",
+           "gsnp_destroy")
+
+
+class GsnpError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class gsnp_params(ctypes.Structure):
+    _fields_ = [("abi_version", ctypes.c_uint32), ("max_read_len", ctypes.c_uint32),
+                ("q_max", ctypes.c_uint32), ("calib_min_count", ctypes.c_uint32),
+                ("het_novel", ctypes.c_double), ("althom_novel", ctypes.c_double),
+                ("global_dep", ctypes.c_double), ("pcr_dep", ctypes.c_double),
+                ("flags", ctypes.c_uint32), ("device", ctypes.c_int32),
+                ("stream", ctypes.c_void_p)]
+
+
+class gsnp_reference(ctypes.Structure):
+    _fields_ = [("code", ctypes.c_void_p), ("n_sites", ctypes.c_uint64),
+                ("origin", ctypes.c_uint64)]
+
+
+class gsnp_priors(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_uint64), ("pos", ctypes.c_void_p), ("prior10", ctypes.c_void_p)]
+
+
+class gsnp_reads(ctypes.Structure):
+    _fields_ = [("n_reads", ctypes.c_uint64), ("pos", ctypes.c_void_p), ("len", ctypes.c_void_p),
+                ("off", ctypes.c_void_p), ("bases", ctypes.c_void_p), ("quals", ctypes.c_void_p),
+                ("strand", ctypes.c_void_p), ("hits", ctypes.c_void_p),
+                ("on_device", ctypes.c_int32)]
+
+
+RECORD_DTYPE = np.dtype([("pos", "<u8"), ("ref", "u1"), ("genotype", "u1"), ("quality", "u1"),
+                         ("base1", "u1"), ("base2", "u1"), ("avgq1", "u1"), ("avgq2", "u1"),
+                         ("known", "u1"), ("cnt_uni1", "<u2"), ("cnt_all1", "<u2"),
+                         ("cnt_uni2", "<u2"), ("cnt_all2", "<u2"), ("depth", "<u4"),
+                         ("rank_p", "<f4"), ("copy_num", "<f4"), ("post1", "<f4")])
+assert RECORD_DTYPE.itemsize == 40
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing: build it with __graft_entry__.build()")
+        L = ctypes.CDLL(LIB_PATH)
+        P = ctypes.c_void_p
+        S = ctypes.c_int32
+        u64 = ctypes.c_uint64
+        L.gsnp_params_default.restype = S
+        L.gsnp_params_default.argtypes = [ctypes.POINTER(gsnp_params)]
+        L.gsnp_create.restype = S
+        L.gsnp_create.argtypes = [ctypes.POINTER(gsnp_reference), ctypes.POINTER(gsnp_priors),
+                                  ctypes.POINTER(gsnp_params), ctypes.POINTER(P)]
+        L.gsnp_calibrate.restype = S
+        L.gsnp_calibrate.argtypes = [P, ctypes.POINTER(gsnp_reads)]
+        L.gsnp_calibrate_count.restype = S
+        L.gsnp_calibrate_count.argtypes = [P, ctypes.POINTER(gsnp_reads), P]
+        L.gsnp_calibrate_finalize.restype = S
+        L.gsnp_calibrate_finalize.argtypes = [P, P]
+        L.gsnp_call.restype = S
+        L.gsnp_call.argtypes = [P, ctypes.POINTER(gsnp_reads), u64, u64, P, u64,
+                                ctypes.POINTER(u64)]
+        L.gsnp_debug_window.restype = S
+        L.gsnp_debug_window.argtypes = [P, ctypes.POINTER(gsnp_reads), u64, u64] + [P] * 7
+        L.gsnp_get_tables.restype = S
+        L.gsnp_get_tables.argtypes = [P, P, P, P, P, P]
+        L.gsnp_launch_count.restype = u64
+        L.gsnp_launch_count.argtypes = [P]
+        L.gsnp_stage_times.restype = S
+        L.gsnp_stage_times.argtypes = [P, P, P, ctypes.c_int, ctypes.c_int]
+        L.gsnp_strerror.restype = ctypes.c_char_p
+        L.gsnp_strerror.argtypes = [S]
+        L.gsnp_last_error.restype = ctypes.c_char_p
+        L.gsnp_last_error.argtypes = [P]
+        L.gsnp_destroy.restype = None
+        L.gsnp_destroy.argtypes = [P]
+        _lib = L
+    return _lib
+
+
+def _ptr(a):
+    """Data pointer of a numpy array or torch tensor (host or CUDA)."""
+    if a is None:
+        return None
+    if hasattr(a, "data_ptr"):
+        return ctypes.c_void_p(a.data_ptr())
+    return a.ctypes.data_as(ctypes.c_void_p)
+
+
+def _on_device(a) -> bool:
+    return bool(getattr(a, "is_cuda", False))
+
+
+def _contig(a, dtype):
+    if hasattr(a, "data_ptr"):
+        import torch
+        tmap = {np.uint8: torch.uint8, np.uint16: torch.uint16, np.uint64: torch.uint64,
+                np.float64: torch.float64}
+        t = a.contiguous()
+        assert t.dtype == tmap[dtype], f"expected {tmap[dtype]}, got {t.dtype}"
+        return t
+    return np.ascontiguousarray(a, dtype)
+
+
+def make_reads(w: dict):
+    """gsnp_reads from a dict with pos/len/off/bases/quals/strand/hits (numpy or torch)."""
+    arrs = dict(pos=_contig(w["pos"], np.uint64), len=_contig(w["len"], np.uint16),
+                off=_contig(w["off"], np.uint64), bases=_contig(w["bases"], np.uint8),
+                quals=_contig(w["quals"], np.uint8), strand=_contig(w["strand"], np.uint8),
+                hits=_contig(w["hits"], np.uint16))
+    dev = _on_device(arrs["pos"])
+    n = int(arrs["pos"].shape[0])
+    r = gsnp_reads(n, *[_ptr(arrs[k]) for k in ("pos", "len", "off", "bases", "quals",
+                                                "strand", "hits")], int(dev))
+    r._keep = arrs
+    return r
+
+
+def params_default(**kw) -> gsnp_params:
+    p = gsnp_params()
+    _check(lib().gsnp_params_default(ctypes.byref(p)), None)
+    for k, v in kw.items():
+        if k == "stream" and v is not None and not isinstance(v, int):
+            v = int(getattr(v, "cuda_stream", v))
+        setattr(p, k, v)
+    return p
+
+
+def _check(st: int, ctx):
+    if st != 0:
+        msg = lib().gsnp_last_error(ctx).decode() if ctx else lib().gsnp_strerror(st).decode()
+        raise GsnpError(st, msg)
+
+
+class Context:
+    """RAII wrapper over gsnp_ctx*.  Methods mirror the ABI calls."""
+
+    def __init__(self, ref, origin: int = 0, known_pos=None, known_prior10=None, **params):
+        self.params = params_default(**params)
+        ref = np.ascontiguousarray(ref, np.uint8)
+        self._ref = ref
+        r = gsnp_reference(_ptr(ref), len(ref), int(origin))
+        kp = np.ascontiguousarray(known_pos if known_pos is not None else [], np.uint64)
+        kpr = np.ascontiguousarray(known_prior10 if known_prior10 is not None else
+                                   np.zeros((0, 10)), np.float64)
+        pri = gsnp_priors(len(kp), _ptr(kp), _ptr(kpr))
+        h = ctypes.c_void_p()
+        st = lib().gsnp_create(ctypes.byref(r), ctypes.byref(pri), ctypes.byref(self.params),
+                               ctypes.byref(h))
+        if st != 0:
+            raise GsnpError(st, lib().gsnp_strerror(st).decode())
+        self.h = h
+        self.origin = int(origin)
+        self.n_sites = len(ref)
+
+    @classmethod
+    def from_workload(cls, w: dict, **params):
+        return cls(w["ref"], w["origin"], w["known_pos"], w["known_prior10"], **params)
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().gsnp_destroy(self.h)
+            self.h = None
+
+    __del__ = close
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def calibrate(self, reads: dict):
+        r = make_reads(reads)
+        _check(lib().gsnp_calibrate(self.h, ctypes.byref(r)), self.h)
+
+    def calibrate_count(self, reads: dict, counts=None):
+        """Returns (or fills) this shard's counts, uint64[64*256*16] (numpy or CUDA tensor)."""
+        if counts is None:
+            counts = np.zeros(64 * 256 * 16, np.uint64)
+        r = make_reads(reads)
+        _check(lib().gsnp_calibrate_count(self.h, ctypes.byref(r), _ptr(counts)), self.h)
+        return counts
+
+    def calibrate_finalize(self, counts):
+        _check(lib().gsnp_calibrate_finalize(self.h, _ptr(counts)), self.h)
+
+    def call(self, reads: dict, w0: int, w1: int, out=None):
+        """Records for sites [w0, w1).  out: None (numpy result), a numpy RECORD_DTYPE array,
+        or a CUDA uint8 tensor of >= 40*(w1-w0) bytes (device output)."""
+        S = w1 - w0
+        if out is None:
+            out = np.zeros(S, RECORD_DTYPE)
+        cap = (out.numel() // 40) if hasattr(out, "numel") else len(out)
+        r = make_reads(reads)
+        n = ctypes.c_uint64(0)
+        _check(lib().gsnp_call(self.h, ctypes.byref(r), w0, w1, _ptr(out), cap, ctypes.byref(n)),
+               self.h)
+        return out
+
+    def call_reads(self, r: gsnp_reads, w0: int, w1: int, out):
+        """Low-overhead variant with prebuilt gsnp_reads (bench loop)."""
+        cap = (out.numel() // 40) if hasattr(out, "numel") else len(out)
+        n = ctypes.c_uint64(0)
+        _check(lib().gsnp_call(self.h, ctypes.byref(r), w0, w1, _ptr(out), cap, ctypes.byref(n)),
+               self.h)
+        return out
+
+    def debug_window(self, reads: dict, w0: int, w1: int):
+        S = w1 - w0
+        nb = int(np.asarray(reads["off"][-1]) - np.asarray(reads["off"][0])) \
+            if len(reads["off"]) else 0
+        out = dict(off=np.zeros(S + 1, np.uint32), keys_built=np.zeros(max(nb, 1), np.uint32),
+                   keys_sorted=np.zeros(max(nb, 1), np.uint32),
+                   counters=np.zeros((S, 15), np.uint32), L10=np.zeros((S, 10)),
+                   post10=np.zeros((S, 10)), records=np.zeros(S, RECORD_DTYPE))
+        r = make_reads(reads)
+        _check(lib().gsnp_debug_window(self.h, ctypes.byref(r), w0, w1, _ptr(out["off"]),
+                                       _ptr(out["keys_built"]), _ptr(out["keys_sorted"]),
+                                       _ptr(out["counters"]), _ptr(out["L10"]),
+                                       _ptr(out["post10"]), _ptr(out["records"])), self.h)
+        K = int(out["off"][-1])
+        out["keys_built"] = out["keys_built"][:K]
+        out["keys_sorted"] = out["keys_sorted"][:K]
+        return out
+
+    def get_tables(self, calibrated: bool = True):
+        dims = np.zeros(3, np.uint32)
+        _check(lib().gsnp_get_tables(self.h, None, None, None, None, _ptr(dims)), self.h)
+        L, P, G = (int(x) for x in dims)
+        adj = np.zeros(64 * P * G, np.uint8)
+        out = dict(L=L, adjP=P, adjG=G)
+        if calibrated:
+            counts = np.zeros(64 * 256 * 16, np.uint64)
+            p = np.zeros(64 * 256 * 16)
+            T = np.zeros(64 * L * 40)
+            _check(lib().gsnp_get_tables(self.h, _ptr(counts), _ptr(p), _ptr(T), _ptr(adj), None),
+                   self.h)
+            out.update(counts=counts.reshape(64, 256, 4, 4), p=p.reshape(64, 256, 4, 4),
+                       T=T.reshape(64, L, 4, 10))
+        else:
+            _check(lib().gsnp_get_tables(self.h, None, None, None, _ptr(adj), None), self.h)
+        out["adj"] = adj.reshape(64, P, G)
+        return out
+
+    def launch_count(self) -> int:
+        return int(lib().gsnp_launch_count(self.h))
+
+    def stage_times(self, reset: bool = False) -> dict:
+        """{stage: (ms, launches)} accumulated with GSNP_TIMING (CUDA events in the library)."""
+        ms = np.zeros(len(STAGES))
+        n = np.zeros(len(STAGES), np.uint64)
+        _check(lib().gsnp_stage_times(self.h, _ptr(ms), _ptr(n), len(STAGES), int(reset)), self.h)
+        return {k: (float(ms[i]), int(n[i])) for i, k in enumerate(STAGES)}
+
+
+# ABI-named free functions (thin aliases)
+def gsnp_create(ref, origin=0, known_pos=None, known_prior10=None, **params) -> Context:
+    return Context(ref, origin, known_pos, known_prior10, **params)
+
+
+def gsnp_calibrate(ctx: Context, reads):
+    return ctx.calibrate(reads)
+
+
+def gsnp_calibrate_count(ctx: Context, reads, counts=None):
+    return ctx.calibrate_count(reads, counts)
+
+
+def gsnp_calibrate_finalize(ctx: Context, counts):
+    return ctx.calibrate_finalize(counts)
+
+
+def gsnp_call(ctx: Context, reads, w0, w1, out=None):
+    return ctx.call(reads, w0, w1, out)
+
+
+def gsnp_debug_window(ctx: Context, reads, w0, w1):
+    return ctx.debug_window(reads, w0, w1)
+
+
+def gsnp_get_tables(ctx: Context):
+    return ctx.get_tables()
+
+
+def gsnp_destroy(ctx: Context):
+    ctx.close()
