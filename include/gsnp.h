@@ -51,7 +51,8 @@ typedef int32_t gsnp_status;
 #define GSNP_STAGE_RANGES 2       /* k_tile_ranges (a3) */
 #define GSNP_STAGE_CALL 3         /* k_call_tile (a4..a8) */
 #define GSNP_STAGE_FINALIZE 4     /* host tables + upload (a2), wall time on the host */
-#define GSNP_N_STAGES 5
+#define GSNP_STAGE_BIG 5          /* k_big_sites (sites with > 1024 unique keys) */
+#define GSNP_N_STAGES 6
 
 typedef struct gsnp_ctx gsnp_ctx;  /* opaque; owned by the library until gsnp_destroy */
 

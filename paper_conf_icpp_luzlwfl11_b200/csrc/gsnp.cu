@@ -53,8 +53,7 @@ struct gsnp_ctx {
     std::string err;
     // reference + known SNPs
     uint64_t n_sites = 0, origin = 0;
-    DevBuf<uint8_t> ref;
-    DevBuf<uint32_t> known_bits;
+    DevBuf<uint8_t> ref;           // code | known << 3
     DevBuf<uint64_t> known_pos;
     DevBuf<double> known_lp;
     uint64_t n_known = 0;
@@ -74,6 +73,8 @@ struct gsnp_ctx {
     DevBuf<unsigned long long> d_counts;
     DevBuf<uint64_t> tile_ra, tile_rb;
     DevBuf<gsnp_record> rec;
+    DevBuf<BigSite> big;
+    DevBuf<uint32_t> big_n;
     // staged host reads
     DevBuf<uint64_t> r_pos, r_off;
     DevBuf<uint16_t> r_len, r_hits;
@@ -86,8 +87,8 @@ struct gsnp_ctx {
     struct Pending { int stage; cudaEvent_t a, b; };
     std::vector<cudaEvent_t> ev_pool;
     std::vector<Pending> pending;
-    double stage_ms[GSNP_N_STAGES] = {0, 0, 0, 0, 0};
-    uint64_t stage_n[GSNP_N_STAGES] = {0, 0, 0, 0, 0};
+    double stage_ms[GSNP_N_STAGES] = {};
+    uint64_t stage_n[GSNP_N_STAGES] = {};
     bool timing() const { return (prm.flags & GSNP_TIMING) != 0; }
     cudaEvent_t ev() {
         if (ev_pool.empty()) {
@@ -364,7 +365,6 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
     A.ref = ctx->ref.p;
     A.origin = ctx->origin;
     A.n_sites = ctx->n_sites;
-    A.known_bits = ctx->known_bits.p;
     A.known_pos = ctx->known_pos.p;
     A.known_lp = ctx->known_lp.p;
     A.n_known = ctx->n_known;
@@ -383,12 +383,27 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
     A.out = d_out;
     A.err = ctx->d_err.p;
     const size_t smem = call_smem_bytes(A.L, nullptr, nullptr);
+    const uint32_t big_cap = (uint32_t)std::min<uint64_t>(w1 - w0, 1u << 22);
+    CK(ctx->big.ensure(big_cap));
+    CK(ctx->big_n.ensure(1));
+    CK(cudaMemsetAsync(ctx->big_n.p, 0, 4, s));
     CK(cudaFuncSetAttribute(k_call_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     ctx->begin();
-    k_call_tile<<<(unsigned)n_tiles, NT, smem, s>>>(A);
+    k_call_tile<<<(unsigned)n_tiles, NT, smem, s>>>(A, ctx->big.p, ctx->big_n.p, big_cap);
     ctx->end(GSNP_STAGE_CALL);
     ctx->launches++;
     CK(cudaGetLastError());
+    if (!A.count_only) {
+        // sites beyond 1024 unique keys: one CTA each, shared buffer of up to ~200 KB
+        const uint32_t cap = (uint32_t)((200 * 1024 - (size_t)8 * A.L) / 4);
+        const size_t bsm = 4 * (size_t)cap + (size_t)8 * A.L;
+        CK(cudaFuncSetAttribute(k_big_sites, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bsm));
+        ctx->begin();
+        k_big_sites<<<(unsigned)g_num_sms, NT, bsm, s>>>(A, ctx->big.p, ctx->big_n.p, cap);
+        ctx->end(GSNP_STAGE_BIG);
+        ctx->launches++;
+        CK(cudaGetLastError());
+    }
     return GSNP_OK;
 }
 
@@ -415,20 +430,20 @@ gsnp_status count_impl(gsnp_ctx* ctx, const gsnp_reads* reads) {
         A.ref = ctx->ref.p;
         A.origin = ctx->origin;
         A.n_sites = ctx->n_sites;
-        A.known_bits = ctx->known_bits.p;
         A.L = (int)ctx->prm.max_read_len;
         A.q_max = (int)ctx->prm.q_max;
+        A.CT = (A.L + 31) / 32 * 32;
+        A.SB = 12 * 1024;                              // bases (and quals) per stage
+        A.CB = std::max(1, std::min<int>(CAL_MAXB, (int)(A.SB - 32) / A.L));
         A.C = ctx->d_counts.p;
         A.err = ctx->d_err.p;
-        size_t diag = (size_t)(A.q_max + 1) * A.L * 4 * 4;
-        A.smem_diag = diag <= 160 * 1024;
-        size_t smem = A.smem_diag ? diag : 0;
-        int per_sm = smem <= 72 * 1024 ? 3 : smem <= 110 * 1024 ? 2 : 1;
-        unsigned grid = (unsigned)std::min<uint64_t>((uint64_t)g_num_sms * per_sm, (d.n + 63) / 64);
+        const size_t smem = align16((size_t)(A.q_max + 1) * 4 * A.CT * 2) + 4 * (size_t)A.SB;
+        const int per_sm = (int)std::max<size_t>(1, std::min<size_t>(4, (227 * 1024) / (smem + 10 * 1024)));
+        unsigned grid = (unsigned)std::min<uint64_t>((uint64_t)g_num_sms * per_sm, (d.n + A.CB - 1) / A.CB);
         grid = std::max(grid, 1u);
         CK(cudaFuncSetAttribute(k_calib_count, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         ctx->begin();
-        k_calib_count<<<grid, NT, smem, s>>>(A);
+        k_calib_count<<<grid, A.CT, smem, s>>>(A);
         ctx->end(GSNP_STAGE_CALIB);
         ctx->launches++;
         CK(cudaGetLastError());
@@ -481,6 +496,7 @@ gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
     if (!out) return GSNP_E_INVAL;
     *out = nullptr;
     if (!ref || !ref->code || ref->n_sites == 0) return GSNP_E_INVAL;
+    if (ref->n_sites >= (1ull << 32)) return GSNP_E_RANGE;   // per-context shard < 4 Gb
     gsnp_ctx* ctx = new (std::nothrow) gsnp_ctx();
     if (!ctx) return GSNP_E_NOMEM;
     gsnp_status st = check_params(ctx, params);
@@ -500,7 +516,7 @@ gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
     // known SNPs: sorted positions, log10 prior rows (C6), site bitmap
     uint64_t nk = priors ? priors->n : 0;
     std::vector<double> lp(std::max<uint64_t>(nk, 1) * 10);
-    std::vector<uint32_t> bits((ref->n_sites + 31) / 32 + 1, 0u);
+    std::vector<uint8_t> code(ref->code, ref->code + ref->n_sites);
     ctx->h_known_pos.assign(nk, 0);
     for (uint64_t k = 0; k < nk; ++k) {
         uint64_t p = priors->pos[k];
@@ -511,8 +527,7 @@ gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
             if (!(v > 0)) return bail(GSNP_E_RANGE);
             lp[k * 10 + n] = log10(v);
         }
-        uint64_t rs = p - ref->origin;
-        bits[rs >> 5] |= 1u << (rs & 31);
+        code[p - ref->origin] |= 8u;                     // known-SNP flag rides on the code
         ctx->h_known_pos[k] = p;
     }
     ctx->n_known = nk;
@@ -534,9 +549,7 @@ gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
     gsnp_ctx* c = ctx;
 #define CKC(x) do { if ((x) != cudaSuccess) { cudaGetLastError(); return bail(fail(c, GSNP_E_CUDA, "%s", #x)); } } while (0)
     CKC(ctx->ref.ensure(ref->n_sites));
-    CKC(cudaMemcpy(ctx->ref.p, ref->code, ref->n_sites, cudaMemcpyHostToDevice));
-    CKC(ctx->known_bits.ensure(bits.size()));
-    CKC(cudaMemcpy(ctx->known_bits.p, bits.data(), bits.size() * 4, cudaMemcpyHostToDevice));
+    CKC(cudaMemcpy(ctx->ref.p, code.data(), ref->n_sites, cudaMemcpyHostToDevice));
     CKC(ctx->known_pos.ensure(std::max<uint64_t>(nk, 1)));
     if (nk) CKC(cudaMemcpy(ctx->known_pos.p, ctx->h_known_pos.data(), nk * 8, cudaMemcpyHostToDevice));
     CKC(ctx->known_lp.ensure(lp.size()));
@@ -733,9 +746,10 @@ const char* gsnp_last_error(const gsnp_ctx* ctx) { return ctx ? ctx->err.c_str()
 void gsnp_destroy(gsnp_ctx* ctx) {
     if (!ctx) return;
     cudaSetDevice(ctx->prm.device);
-    ctx->ref.release(); ctx->known_bits.release(); ctx->known_pos.release(); ctx->known_lp.release();
+    ctx->ref.release(); ctx->known_pos.release(); ctx->known_lp.release();
     ctx->adj.release(); ctx->LP.release(); ctx->T.release(); ctx->d_err.release();
     ctx->d_counts.release(); ctx->tile_ra.release(); ctx->tile_rb.release(); ctx->rec.release();
+    ctx->big.release(); ctx->big_n.release();
     ctx->r_pos.release(); ctx->r_off.release(); ctx->r_len.release(); ctx->r_hits.release();
     ctx->r_bases.release(); ctx->r_quals.release(); ctx->r_strand.release();
     ctx->dbg_u32a.release(); ctx->dbg_u32b.release(); ctx->dbg_u32c.release();

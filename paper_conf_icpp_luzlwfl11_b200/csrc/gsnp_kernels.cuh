@@ -38,9 +38,8 @@ struct DevReads {
 
 struct CallArgs {
     DevReads R;
-    const uint8_t* ref;               // reference codes, ref[site - origin]
+    const uint8_t* ref;               // ref[site - origin] = code | known << 3 (known SNP)
     uint64_t origin, n_sites;
-    const uint32_t* known_bits;       // bit (site - origin): site is a known SNP
     const uint64_t* known_pos;        // sorted
     const double* known_lp;           // n_known x 10 log10 priors (host-built)
     uint64_t n_known;
@@ -145,56 +144,165 @@ __device__ __forceinline__ void for_each_base(const DevReads& R, uint64_t ra, ui
 }
 
 // ------------------------------------------------------------------------------------------
-// a1: calibration histogram.  Diagonal cells (t == o, ~98% of bases) go to a shared
-// [q][cyc][t] u32 histogram flushed once per CTA; mismatches go straight to global u64 REDs.
+// TMA (1-D bulk copy) + mbarrier helpers (sm_90+; SASS UBLKCP / SYNCS).
+__host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+                 "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n .reg .pred P1;\n"
+        "WAIT_%=:\n"
+        " mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+        " @!P1 bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)), "r"(parity) : "memory");
+}
+// global -> shared bulk copy of `bytes` (multiple of 16, both addresses 16-byte aligned)
+__device__ __forceinline__ void tma_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+        ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+// ------------------------------------------------------------------------------------------
+// a1: calibration histogram C[q][cyc][t][o] (cal_p_matrix).
+// The CTA streams its share of the reads in batches: the batch's bases and qualities (one
+// contiguous byte range) arrive in shared memory by TMA bulk copies, double-buffered and
+// completed on an mbarrier, while the previous batch is counted.  Cycle-major counting: thread
+// c owns sequencing cycle c, so the diagonal cells (t == o, ~98% of bases) accumulate in a
+// shared [q][t][cycle] u16 histogram with plain read-modify-writes (flushed to the global u64
+// counts before any cell can overflow); mismatches go straight to global u64 REDs.
 struct CalibArgs {
     DevReads R;
-    const uint8_t* ref;
+    const uint8_t* ref;               // code | known << 3, indexed by site - origin
     uint64_t origin, n_sites;
-    const uint32_t* known_bits;
     int L, q_max;
+    int CT;                           // threads per CTA = L rounded up to a multiple of 32
+    int CB;                           // reads per batch
+    uint32_t SB;                      // bytes per stage buffer (bases; quals the same)
     unsigned long long* C;            // [64][256][4][4]
     int* err;
-    int smem_diag;                    // 1 if the diagonal histogram lives in shared memory
 };
 
-__global__ void __launch_bounds__(NT) k_calib_count(CalibArgs A) {
-    extern __shared__ __align__(16) unsigned char smem[];
-    __shared__ WarpMeta wm[NW];
-    uint32_t* diag = reinterpret_cast<uint32_t*>(smem);
-    const int nd = (A.q_max + 1) * A.L * 4;
-    if (A.smem_diag)
-        for (int i = threadIdx.x; i < nd; i += NT) diag[i] = 0;
-    __syncthreads();
-    const int warp = threadIdx.x >> 5;
-    // this CTA's share of the reads
-    uint64_t per = (A.R.n + gridDim.x - 1) / gridDim.x;
-    uint64_t ra = min(A.R.n, (uint64_t)blockIdx.x * per), rb = min(A.R.n, ra + per);
-    for_each_base(A.R, ra, rb, wm[warp], warp, NW, [&](int k, uint32_t i, WarpMeta& m) {
-        if (m.hits[k] != 1) return;
-        uint64_t site = m.pos[k] + i;
-        uint64_t bi = m.off[k] + i;
-        uint32_t o = A.R.bases[bi], q = A.R.quals[bi];
-        if (o > 4) { atomicOr(A.err, ERR_RANGE); return; }
-        if (q > (uint32_t)A.q_max) { atomicOr(A.err, ERR_QUAL); return; }
-        if (site < A.origin || site >= A.origin + A.n_sites) return;   // flagged by validate
-        uint64_t rs = site - A.origin;
-        uint32_t t = A.ref[rs];
-        if (t == 4 || o == 4) return;
-        if ((A.known_bits[rs >> 5] >> (rs & 31)) & 1u) return;
-        uint32_t cyc = m.strand[k] ? m.len[k] - 1 - i : i;
-        if (t == o && A.smem_diag) atomicAdd(&diag[(q * A.L + cyc) * 4 + t], 1u);
-        else atomicAdd(&A.C[q << 12 | cyc << 4 | t << 2 | o], 1ull);
-    });
-    __syncthreads();
-    if (A.smem_diag)
-        for (int i = threadIdx.x; i < nd; i += NT) {
-            uint32_t v = diag[i];
-            if (v) {
-                int t = i & 3, cyc = (i >> 2) % A.L, q = (i >> 2) / A.L;
-                atomicAdd(&A.C[q << 12 | cyc << 4 | t << 2 | t], (unsigned long long)v);
-            }
+constexpr int CAL_MAXB = 512;         // max reads per batch (metadata arrays)
+
+__device__ __forceinline__ void calib_flush(const CalibArgs& A, uint16_t* h, int nbins) {
+    const int c = threadIdx.x;
+    if (c >= A.L) return;
+    for (int k = 0; k < nbins; ++k) {                 // k = q*4 + t
+        uint16_t* cell = h + (size_t)k * A.CT + c;
+        const uint32_t v = *cell;
+        if (v) {
+            const uint32_t q = k >> 2, t = k & 3;
+            atomicAdd(&A.C[q << 12 | (uint32_t)c << 4 | t << 2 | t], (unsigned long long)v);
+            *cell = 0;
         }
+    }
+}
+
+__global__ void __launch_bounds__(256) k_calib_count(CalibArgs A) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    __shared__ uint32_t m_rs[CAL_MAXB];               // read start - origin
+    __shared__ uint32_t m_off[CAL_MAXB];              // byte offset within the stage buffer
+    __shared__ uint32_t m_lhs[CAL_MAXB];              // len | strand << 16 | counted << 17
+    __shared__ __align__(8) uint64_t bar[2];
+    __shared__ uint64_t st_base[2];                   // global byte index of each stage's start
+    __shared__ int st_direct[2];                      // batch too wide for the stage: read global
+    const int nbins = (A.q_max + 1) * 4;
+    uint16_t* h = reinterpret_cast<uint16_t*>(smem);
+    unsigned char* stage = smem + align16((size_t)nbins * A.CT * 2);
+    const int c = threadIdx.x;
+    for (int i = c; i < nbins * A.CT; i += blockDim.x) h[i] = 0;
+    const uint64_t per = (A.R.n + gridDim.x - 1) / gridDim.x;
+    const uint64_t ra = min(A.R.n, (uint64_t)blockIdx.x * per), rb = min(A.R.n, ra + per);
+    const uint64_t nbatch = (rb - ra + A.CB - 1) / A.CB;
+    if (c == 0) { mbar_init(&bar[0], 1); mbar_init(&bar[1], 1); }
+    __syncthreads();
+    // issue the bulk copies of batch k into stage k & 1 (thread 0)
+    auto issue = [&](uint64_t k) {
+        const uint64_t b0 = ra + k * A.CB, b1 = min(rb, b0 + A.CB);
+        const uint64_t o0 = A.R.off[b0] - A.R.off0, o1 = A.R.off[b1] - A.R.off0;
+        const uint64_t a0 = o0 & ~15ull, a1 = (o1 + 15) & ~15ull;
+        const int sidx = (int)(k & 1);
+        st_base[sidx] = a0;
+        if (a1 - a0 > A.SB) { st_direct[sidx] = 1; return; }
+        st_direct[sidx] = 0;
+        unsigned char* sb = stage + (size_t)sidx * 2 * A.SB;
+        const uint32_t bytes = (uint32_t)(a1 - a0);
+        fence_proxy_async_smem();
+        mbar_arrive_expect_tx(&bar[sidx], 2 * bytes);
+        tma_g2s(sb, A.R.bases + a0, bytes, &bar[sidx]);
+        tma_g2s(sb + A.SB, A.R.quals + a0, bytes, &bar[sidx]);
+    };
+    if (c == 0 && nbatch > 0) issue(0);
+    int err = 0;
+    uint32_t since_flush = 0;
+    // count cycle c of reads [0, nr) of the current batch from byte arrays sb/sq
+    auto count = [&](const unsigned char* __restrict__ sb, const unsigned char* __restrict__ sq,
+                     uint32_t nr) {
+#pragma unroll 4
+        for (uint32_t j = 0; j < nr; ++j) {
+            const uint32_t lhs = m_lhs[j], l = lhs & 0xFFFFu, st = (lhs >> 16) & 1u;
+            const bool take = (lhs >> 17) && (uint32_t)c < l;       // counted read, cycle exists
+            const uint32_t i = st ? l - 1 - c : c;                 // read position of cycle c
+            const uint32_t bi = m_off[j] + (take ? i : 0u);
+            const uint32_t o = sb[bi], q = sq[bi];
+            const uint32_t rt = A.ref[take ? m_rs[j] + i : 0u];     // code | known << 3
+            const uint32_t t = rt & 7u;
+            err |= (take && o > 4) ? ERR_RANGE : 0;
+            err |= (take && q > (uint32_t)A.q_max) ? ERR_QUAL : 0;
+            const bool cnt = take && t < 4 && o < 4 && q <= (uint32_t)A.q_max && !(rt & 8u);
+            if (cnt && t == o) h[(q * 4 + t) * A.CT + c] += 1;
+            else if (cnt) atomicAdd(&A.C[q << 12 | (uint32_t)c << 4 | t << 2 | o], 1ull);
+        }
+    };
+    for (uint64_t k = 0; k < nbatch; ++k) {
+        const int sidx = (int)(k & 1);
+        const uint64_t b0 = ra + k * A.CB, b1 = min(rb, b0 + A.CB);
+        const uint32_t nr = (uint32_t)(b1 - b0);
+        __syncthreads();                               // stage (k+1)&1 and metadata free
+        if (c == 0 && k + 1 < nbatch) issue(k + 1);
+        for (uint32_t j = c; j < nr; j += blockDim.x) {
+            const uint64_t r = b0 + j;
+            const uint64_t p = A.R.pos[r];
+            const uint32_t l = A.R.len[r];
+            // unique reads inside the reference are counted (others are flagged by validate)
+            const bool in = p >= A.origin && p + l <= A.origin + A.n_sites;
+            m_rs[j] = in ? (uint32_t)(p - A.origin) : 0u;
+            m_off[j] = (uint32_t)(A.R.off[r] - A.R.off0 - st_base[sidx]);
+            m_lhs[j] = l | (uint32_t)A.R.strand[r] << 16 | ((A.R.hits[r] == 1 && in) ? 1u << 17 : 0u);
+        }
+        if (since_flush + nr > 65535u) {               // u16 cells could overflow: flush
+            __syncthreads();
+            calib_flush(A, h, nbins);
+            since_flush = 0;
+        }
+        since_flush += nr;
+        __syncthreads();
+        if (c < A.L) {
+            if (st_direct[sidx]) {
+                count(A.R.bases + st_base[sidx], A.R.quals + st_base[sidx], nr);
+            } else {
+                mbar_wait(&bar[sidx], (uint32_t)((k >> 1) & 1));
+                const unsigned char* sb = stage + (size_t)sidx * 2 * A.SB;
+                count(sb, sb + A.SB, nr);
+            }
+        } else if (!st_direct[sidx]) {
+            mbar_wait(&bar[sidx], (uint32_t)((k >> 1) & 1));
+        }
+    }
+    if (err) atomicOr(A.err, err);
+    __syncthreads();
+    calib_flush(A, h, nbins);
 }
 // ------------------------------------------------------------------------------------------
 // a3: read ranges.  For each group of 32 consecutive sites [s0, s0+32) (one warp of
@@ -215,39 +323,22 @@ __global__ void k_tile_ranges(const uint64_t* pos, uint64_t n, uint64_t w0, uint
 // parallelisation).  Shared-memory layout (host: call_smem_bytes()).
 constexpr int TS = NT;
 constexpr int COLS = 32;              // key slots per site on the thread-per-site path
-constexpr int WBUF = 256;             // per-warp key buffer of the warp path (n <= 256)
 
 struct TileSmem {
-    uint32_t* col;       // [COLS][TS] keys in gather order; reused as the CTA deep buffer
-    uint32_t* wbuf;      // [NW][WBUF]
+    uint32_t* col;       // [COLS][TS] keys: column of site t at col[j*TS + t]; a warp's 32
+                         // columns double as its 1024-key buffer on the warp paths
     uint8_t* slotcnt;    // [NW][4 * 2L] per-warp (base, strand, coord) counters
-    uint32_t* cnt_all;   // [4][TS]
-    uint32_t* rep;       // [TS]
-    uint32_t* nuni;      // [TS]
-    int deep_cap;        // keys the col region holds
 };
 
-__host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
-
 __host__ __device__ inline size_t call_smem_bytes(int L, TileSmem* s, unsigned char* base) {
-    size_t o = 0;
-    auto take = [&](size_t bytes) { size_t r = o; o = align16(o + bytes); return r; };
-    size_t o_col = take(4 * (size_t)COLS * TS);
-    size_t o_wbuf = take(4 * (size_t)NW * WBUF);
-    size_t o_slot = take((size_t)NW * 8 * L);
-    size_t o_cnt = take(16 * (size_t)TS);
-    size_t o_rep = take(4 * (size_t)TS);
-    size_t o_nuni = take(4 * (size_t)TS);
+    size_t o_col = 0;
+    size_t o_slot = align16(4 * (size_t)COLS * TS);
+    size_t total = align16(o_slot + (size_t)NW * 8 * L);
     if (s) {
         s->col = reinterpret_cast<uint32_t*>(base + o_col);
-        s->wbuf = reinterpret_cast<uint32_t*>(base + o_wbuf);
         s->slotcnt = base + o_slot;
-        s->cnt_all = reinterpret_cast<uint32_t*>(base + o_cnt);
-        s->rep = reinterpret_cast<uint32_t*>(base + o_rep);
-        s->nuni = reinterpret_cast<uint32_t*>(base + o_nuni);
-        s->deep_cap = COLS * TS;
     }
-    return o;
+    return total;
 }
 
 __device__ __forceinline__ uint32_t key_base(uint32_t k) { return (k >> 15) & 3u; }
@@ -295,10 +386,11 @@ __device__ __forceinline__ int geno_a2(int t) {
     return t < 4 ? t : t < 7 ? t - 3 : t < 9 ? t - 5 : 3;
 }
 
-// Known-SNP lookup of a site: the row index into known_lp, or -1 (novel prior, R6).
-__device__ __forceinline__ int64_t known_index(const CallArgs& A, uint64_t site) {
-    const uint64_t rs = site - A.origin;
-    if (!((__ldg(A.known_bits + (rs >> 5)) >> (rs & 31)) & 1u)) return -1;
+// Reference code and known-SNP row of a site (R6: -1 = novel prior).
+__device__ __forceinline__ int64_t site_ref(const CallArgs& A, uint64_t site, int& refb) {
+    const uint32_t rt = A.ref[site - A.origin];
+    refb = (int)(rt & 7u);
+    if (!(rt & 8u)) return -1;
     return (int64_t)lower_bound_u64(A.known_pos, 0, A.n_known, site);
 }
 
@@ -399,10 +491,11 @@ __device__ __noinline__ void site_record(const CallArgs& A, uint64_t site, int r
 }
 
 // ------------------------------------------------------------------------------------------
-// Thread-per-site likelihood for n <= N <= 32 keys (the common case).  Keys come from the
-// site's shared-memory column, are sorted by an in-register bitonic network (likelihood_sort),
-// then Alg. 4 runs sequentially in canonical order — the same terms in the same order as the
-// oracle — followed by C7 and the record.
+// Thread-per-site likelihood for n <= N <= 32 keys (the common case).  Each key was stored as
+// key << 8 | (pcr - 1) by the gather (pcr = occurrences of its (base, strand, coord) so far in
+// canonical order).  An in-register bitonic network sorts them (likelihood_sort; the pcr byte
+// only breaks ties between identical keys), then Alg. 4 runs sequentially in canonical order —
+// the same terms in the same order as the oracle — followed by C6-C9 and the record.
 template <int N>
 __device__ __forceinline__ void sort_net(uint32_t (&k)[N]) {
 #pragma unroll
@@ -421,74 +514,90 @@ __device__ __forceinline__ void sort_net(uint32_t (&k)[N]) {
             }
 }
 
+// Sort the first n (<= N) entries of this thread's column in registers and store them back.
 template <int N>
-__device__ __forceinline__ void thread_site(const CallArgs& A, const TileSmem& sm, uint64_t site,
-                                            uint32_t n, bool dup, uint32_t ca0, uint32_t ca1,
-                                            uint32_t ca2, uint32_t ca3, uint32_t rep,
-                                            const double* sLP) {
-    const int tid = threadIdx.x;
+__device__ __forceinline__ void sort_column(uint32_t* colp, uint32_t n) {
     uint32_t k[N];
 #pragma unroll
-    for (int j = 0; j < N; ++j) k[j] = (j < (int)n) ? sm.col[j * TS + tid] : KEY_INF;
+    for (int j = 0; j < N; ++j) k[j] = (j < (int)n) ? colp[j * TS] : KEY_INF;
     sort_net<N>(k);
+#pragma unroll
+    for (int j = 0; j < N; ++j) if (j < (int)n) colp[j * TS] = k[j];
+}
+
+__device__ __noinline__ void thread_site(const CallArgs& A, uint32_t* colp, uint64_t site,
+                                         uint32_t n, bool slow_pcr, uint32_t ca0, uint32_t ca1,
+                                         uint32_t ca2, uint32_t ca3, uint32_t rep) {
     if (A.dbg_keys_sorted) {
         const uint32_t o = A.dbg_off[site - A.w0];
-#pragma unroll
-        for (int j = 0; j < N; ++j) if (j < (int)n) A.dbg_keys_sorted[o + j] = k[j];
+        for (uint32_t j = 0; j < n; ++j) A.dbg_keys_sorted[o + j] = colp[j * TS] >> 8;
     }
-    // Alg. 4 lines 6-17: dep_count reset per base (l.8-11); pcr = occurrences of this
-    // (strand, coord) so far; g = distinct (strand, coord) so far - 1 (R3).  Without duplicate
-    // slots (checked during the gather) pcr == 1 and g = position within the base's run.
+    // Alg. 4 lines 6-17 in canonical order: dep_count reset per base (l.8-11); pcr from the
+    // gather, or recounted when '-' strand reads of unequal length can share a coordinate;
+    // g = distinct (strand, coord) so far in this base - 1 (R3).
     double acc[10];
 #pragma unroll
     for (int j = 0; j < 10; ++j) acc[j] = 0.0;
     uint64_t cu = 0, qs = 0;
     uint32_t prev_b = 4, distinct = 0;
-#pragma unroll
-    for (int j = 0; j < N; ++j) {
-        if (j < (int)n) {
-            const uint32_t kk = k[j], b = key_base(kk), q = key_q(kk);
-            uint32_t pcr = 1;
-            if (dup) {
-#pragma unroll
-                for (int i = 0; i < j; ++i) pcr += ((k[i] ^ kk) & KEY_BSLOT) == 0;
-            }
-            if (b != prev_b) { distinct = 0; prev_b = b; }
-            distinct += pcr == 1;
-            const int qa = adj_lookup(A, q, pcr, distinct - 1);
-            add_row(A.T, A.L, (uint32_t)qa, key_cyc(kk), b, acc);
-            cu += 1ull << (16 * b);
-            qs += (uint64_t)q << (16 * b);
+#pragma unroll 4
+    for (uint32_t j = 0; j < n; ++j) {
+        const uint32_t kw = colp[j * TS];
+        const uint32_t kk = kw >> 8, b = key_base(kk), q = key_q(kk);
+        uint32_t pcr = (kw & 255u) + 1u;
+        if (slow_pcr) {
+            pcr = 1;
+            for (uint32_t i = 0; i < j; ++i) pcr += (((colp[i * TS] >> 8) ^ kk) & KEY_BSLOT) == 0;
         }
+        if (b != prev_b) { distinct = 0; prev_b = b; }
+        distinct += pcr == 1;
+        const int qa = adj_lookup(A, q, pcr, distinct - 1);
+        add_row(A.T, A.L, (uint32_t)qa, key_cyc(kk), b, acc);
+        cu += 1ull << (16 * b);
+        qs += (uint64_t)q << (16 * b);
     }
     // C6/C7: priors, posterior, top-2
-    const int refb = A.ref[site - A.origin];
-    const int64_t kidx = known_index(A, site);
-    const double* prow = kidx >= 0 ? A.known_lp + kidx * 10 : sLP + refb * 10;
+    int refb;
+    const int64_t kidx = site_ref(A, site, refb);
+    const double* prow = kidx >= 0 ? A.known_lp + kidx * 10 : A.LP + refb * 10;
     double lp[10], m = -INFINITY;
 #pragma unroll
     for (int j = 0; j < 10; ++j) {
-        lp[j] = acc[j] + prow[j];
+        lp[j] = acc[j] + __ldg(prow + j);
         m = lp[j] > m ? lp[j] : m;
     }
     int t1, t2;
     top2(lp, t1, t2);
-    double esum = 0.0;
+    // posterior denominator in genotype order; a term below 1e-18 of the maximum cannot change
+    // the double sum (every term is <= 1 and the maximum's term is exactly 1), so it is skipped
+    // unless the debug dump wants every posterior
+    const bool all_terms = A.dbg_post10 != nullptr;
+    uint32_t need = 0;
 #pragma unroll
-    for (int j = 0; j < 10; ++j) esum += exp10(lp[j] - m);
+    for (int j = 0; j < 10; ++j) need |= (all_terms || lp[j] - m > -18.0) ? 1u << j : 0u;
+    double esum = 0.0;
+    const uint32_t am = __activemask();
+    while (__any_sync(am, need != 0)) {                // terms in genotype order, one per pass
+        if (need) {
+            const int jj = __ffs(need) - 1;
+            need &= need - 1;
+            double x = lp[0];
+#pragma unroll
+            for (int j = 1; j < 10; ++j) x = jj == j ? lp[j] : x;
+            esum += exp10(x - m);
+        }
+    }
     // C8 pieces: W = sum of pooled mid-ranks of allele-1 qualities; tie = sum(t^3 - t)
     const int a1 = geno_a1(t1), a2 = geno_a2(t1);
     double wsum = 0.0, tie = 0.0;
     if (a1 != a2 && (A.flags & GSNP_RANK_SUM) && f16(cu, a1) && f16(cu, a2)) {
-#pragma unroll 1
-        for (int x = 0; x < (int)n; ++x) {
-            uint32_t xk = sm.col[x * TS + tid];
+        for (uint32_t x = 0; x < n; ++x) {
+            const uint32_t xk = colp[x * TS] >> 8;
             const uint32_t xb = key_base(xk), xq = key_q(xk);
             if (xb != (uint32_t)a1 && xb != (uint32_t)a2) continue;
             uint32_t less = 0, eq = 0;
-#pragma unroll 1
-            for (int y = 0; y < (int)n; ++y) {
-                const uint32_t yk = sm.col[y * TS + tid], yb = key_base(yk), yq = key_q(yk);
+            for (uint32_t y = 0; y < n; ++y) {
+                const uint32_t yk = colp[y * TS] >> 8, yb = key_base(yk), yq = key_q(yk);
                 const bool yin = yb == (uint32_t)a1 || yb == (uint32_t)a2;
                 less += yin && yq < xq;
                 eq += yin && yq == xq;
@@ -510,18 +619,21 @@ __device__ __forceinline__ void thread_site(const CallArgs& A, const TileSmem& s
 }
 
 // ------------------------------------------------------------------------------------------
-// Warp path for 32 < n <= 256: the warp gathers the site's keys into its buffer, sorts them
-// with a K-per-lane bitonic network, and walks Alg. 4 chunk by chunk (32 keys per chunk) with
-// match_any for same-slot peers and per-warp shared counters across chunks.
+// Warp paths for n > 32.  The warp re-gathers the site's keys (plain 17-bit keys) into its
+// slice of the col region: element e lives at col[(e >> 5) * TS + warp * 32 + (e & 31)].
+__device__ __forceinline__ uint32_t wslot(int warp, uint32_t e) {
+    return (e >> 5) * TS + warp * 32 + (e & 31);
+}
+
 __device__ __forceinline__ void group_epilogue(const CallArgs& A, uint64_t site, int refb,
-                                               int64_t kidx, const double* sLP, const double* L10,
+                                               int64_t kidx, const double* L10,
                                                const uint32_t* cu, const uint32_t* qs,
                                                uint32_t ca0, uint32_t ca1, uint32_t ca2,
                                                uint32_t ca3, uint32_t rep, double wsum,
                                                double tie) {
     const int lane = threadIdx.x & 31;
     double lp[10], m = -INFINITY;
-    const double* prow = kidx >= 0 ? A.known_lp + kidx * 10 : sLP + refb * 10;
+    const double* prow = kidx >= 0 ? A.known_lp + kidx * 10 : A.LP + refb * 10;
 #pragma unroll
     for (int n = 0; n < 10; ++n) {
         lp[n] = L10[n] + prow[n];
@@ -545,22 +657,53 @@ __device__ __forceinline__ void group_epilogue(const CallArgs& A, uint64_t site,
     }
 }
 
+// Warp gather of one site's unique non-N keys from the reads [ra, rb) into the warp slice;
+// returns the count.
+__device__ __forceinline__ uint32_t warp_gather(const CallArgs& A, uint32_t* col, int warp,
+                                                uint64_t s, uint64_t ra, uint64_t rb) {
+    const int lane = threadIdx.x & 31;
+    uint32_t m = 0;
+    for (uint64_t r0 = ra; r0 < rb; r0 += 32) {
+        const uint64_t r = r0 + lane;
+        uint32_t key = KEY_INF;
+        if (r < rb && A.R.hits[r] == 1) {
+            const uint64_t i = s - A.R.pos[r];
+            const uint32_t l = A.R.len[r];
+            if (i < l) {
+                const uint64_t bi = A.R.off[r] - A.R.off0 + i;
+                const uint32_t b = A.R.bases[bi];
+                if (b < 4) {
+                    const uint32_t st = A.R.strand[r];
+                    const uint32_t cyc = st ? l - 1 - (uint32_t)i : (uint32_t)i;
+                    key = b << 15 | (63u - A.R.quals[bi]) << 9 | cyc << 1 | st;
+                }
+            }
+        }
+        const uint32_t v = __ballot_sync(FULL, key != KEY_INF);
+        if (key != KEY_INF) col[wslot(warp, m + __popc(v & lanemask_lt()))] = key;
+        m += __popc(v);
+    }
+    __syncwarp();
+    return m;
+}
+
+// 32 < n <= 256: K keys per lane in registers, bitonic network over N = 32K, Alg. 4 walked
+// chunk by chunk with match_any for same-slot peers and per-warp counters across chunks.
 template <int K>
-__device__ void warp_site(const CallArgs& A, const uint32_t* buf, uint32_t n, uint64_t site,
-                          uint32_t ca0, uint32_t ca1, uint32_t ca2, uint32_t ca3, uint32_t rep,
-                          const double* sLP, uint8_t* slotcnt) {
+__device__ void warp_site(const CallArgs& A, const uint32_t* col, int warp, uint32_t n,
+                          uint64_t site, uint32_t ca0, uint32_t ca1, uint32_t ca2, uint32_t ca3,
+                          uint32_t rep, uint8_t* slotcnt) {
     constexpr int N = 32 * K;
     const int lane = threadIdx.x & 31;
     const int L2 = 2 * A.L;
-    const int refb = A.ref[site - A.origin];
-    const int64_t kidx = known_index(A, site);
+    int refb;
+    const int64_t kidx = site_ref(A, site, refb);
     uint32_t key[K];
 #pragma unroll
     for (int k = 0; k < K; ++k) {
         uint32_t e = k * 32 + lane;
-        key[k] = (e < n) ? buf[e] : KEY_INF;
+        key[k] = (e < n) ? col[wslot(warp, e)] : KEY_INF;
     }
-    // bitonic network over N = 32*K elements (element e = k*32 + lane)
 #pragma unroll
     for (int size = 2; size <= N; size <<= 1) {
 #pragma unroll
@@ -647,7 +790,7 @@ __device__ void warp_site(const CallArgs& A, const uint32_t* buf, uint32_t n, ui
     }
     // rank-sum pieces for a heterozygous call (R8)
     double lp[10];
-    const double* prow = kidx >= 0 ? A.known_lp + kidx * 10 : sLP + refb * 10;
+    const double* prow = kidx >= 0 ? A.known_lp + kidx * 10 : A.LP + refb * 10;
 #pragma unroll
     for (int j = 0; j < 10; ++j) lp[j] = acc[j] + prow[j];
     int t1, t2;
@@ -664,7 +807,7 @@ __device__ void warp_site(const CallArgs& A, const uint32_t* buf, uint32_t n, ui
             uint32_t less = 0, eq = 0;
 #pragma unroll 1
             for (uint32_t e = 0; e < n; ++e) {
-                const uint32_t y = buf[e], yb = key_base(y), yq = key_q(y);
+                const uint32_t y = col[wslot(warp, e)], yb = key_base(y), yq = key_q(y);
                 const bool yin = yb == (uint32_t)a1 || yb == (uint32_t)a2;
                 less += yin && yq < xq;
                 eq += yin && yq == xq;
@@ -680,7 +823,140 @@ __device__ void warp_site(const CallArgs& A, const uint32_t* buf, uint32_t n, ui
             tie += __shfl_xor_sync(FULL, tie, d);
         }
     }
-    group_epilogue(A, site, refb, kidx, sLP, acc, cu, qs, ca0, ca1, ca2, ca3, rep, wsum, tie);
+    group_epilogue(A, site, refb, kidx, acc, cu, qs, ca0, ca1, ca2, ca3, rep, wsum, tie);
+}
+
+// Dependency walk over keys already in canonical order, one warp, 32 per chunk: stores q_adj
+// into bits 17..22 of each key (shared by the warp-deep and CTA paths).
+template <typename Idx>
+__device__ __forceinline__ void walk_chunks(const CallArgs& A, uint32_t* a, Idx idx, uint32_t n,
+                                            uint8_t* slotcnt) {
+    const int lane = threadIdx.x & 31;
+    const int L2 = 2 * A.L;
+    int d0 = 0, d1 = 0, d2 = 0, d3 = 0;
+    const uint32_t lt = lanemask_lt(), le = lt | (1u << lane);
+    for (uint32_t c0 = 0; c0 < n; c0 += 32) {
+        const uint32_t e = c0 + lane;
+        const bool valid = e < n;
+        const uint32_t kk = valid ? a[idx(e)] : KEY_INF;
+        const uint32_t b = key_base(kk), q = key_q(kk), slot = key_slot(kk);
+        const uint32_t peers = __match_any_sync(FULL, valid ? (b << 9 | slot) : (0x80000000u | lane));
+        uint32_t pcr = 1u + __popc(peers & lt) + (valid ? slotcnt[b * L2 + slot] : 0u);
+        const bool first = valid && pcr == 1u;
+        const uint32_t fb = __ballot_sync(FULL, first);
+        const uint32_t bmask = __match_any_sync(FULL, valid ? b : (0x80000000u | lane));
+        const int db = b == 0 ? d0 : b == 1 ? d1 : b == 2 ? d2 : d3;
+        const uint32_t g = (uint32_t)(db + __popc(fb & bmask & le) - 1);
+        if (valid && (peers >> lane) == 1u) slotcnt[b * L2 + slot] = (uint8_t)min(pcr, 255u);
+        d0 += __popc(fb & __ballot_sync(FULL, valid && b == 0));
+        d1 += __popc(fb & __ballot_sync(FULL, valid && b == 1));
+        d2 += __popc(fb & __ballot_sync(FULL, valid && b == 2));
+        d3 += __popc(fb & __ballot_sync(FULL, valid && b == 3));
+        __syncwarp();
+        if (valid) a[idx(e)] = (kk & 0x1FFFFu) | (uint32_t)adj_lookup(A, q, pcr, g) << 17;
+    }
+    __syncwarp();
+    for (uint32_t e = lane; e < n; e += 32) slotcnt[key_base(a[idx(e)]) * L2 + key_slot(a[idx(e)])] = 0;
+    __syncwarp();
+}
+
+// Rank-sum pieces over keys (bits 0..16 valid) by histogram over the 64 quality values.
+template <typename Idx>
+__device__ void hist_ranks(const uint32_t* a, Idx idx, uint32_t n, int a1, int a2, double& wsum,
+                           double& tie) {
+    uint32_t hx[64], hy[64];
+    for (int v = 0; v < 64; ++v) { hx[v] = 0; hy[v] = 0; }
+    for (uint32_t e = 0; e < n; ++e) {
+        uint32_t b = key_base(a[idx(e)]), q = key_q(a[idx(e)]);
+        if (b == (uint32_t)a1) hx[q]++;
+        else if (b == (uint32_t)a2) hy[q]++;
+    }
+    double less = 0.0;
+    wsum = 0.0;
+    tie = 0.0;
+    for (int v = 0; v < 64; ++v) {
+        double t = (double)hx[v] + (double)hy[v];
+        wsum += (double)hx[v] * (less + (t + 1.0) / 2.0);
+        tie += t * t * t - t;
+        less += t;
+    }
+}
+
+// 256 < n <= 1024: the warp sorts its slice in shared memory (bitonic, arbitrary n), walks the
+// chunks, then all lanes gather and reduce.
+__device__ __noinline__ void warp_deep_site(const CallArgs& A, uint32_t* col, int warp,
+                                            uint32_t n, uint64_t site, uint32_t ca0, uint32_t ca1,
+                                            uint32_t ca2, uint32_t ca3, uint32_t rep,
+                                            uint8_t* slotcnt) {
+    const int lane = threadIdx.x & 31;
+    auto idx = [warp](uint32_t e) { return wslot(warp, e); };
+    uint32_t N2 = 1;
+    while (N2 < n) N2 <<= 1;
+    for (uint32_t size = 2; size <= N2; size <<= 1) {
+        const uint32_t half = size >> 1;
+        for (uint32_t t = lane; t < N2 / 2; t += 32) {
+            uint32_t blk = t / half, o = t % half;
+            uint32_t i = blk * size + o, j = blk * size + size - 1 - o;
+            if (j < n) {
+                uint32_t x = col[idx(i)], y = col[idx(j)];
+                if (x > y) { col[idx(i)] = y; col[idx(j)] = x; }
+            }
+        }
+        __syncwarp();
+        for (uint32_t stride = size >> 2; stride > 0; stride >>= 1) {
+            for (uint32_t t = lane; t < N2 / 2; t += 32) {
+                uint32_t i = (t / stride) * 2 * stride + (t % stride), j = i + stride;
+                if (j < n) {
+                    uint32_t x = col[idx(i)], y = col[idx(j)];
+                    if (x > y) { col[idx(i)] = y; col[idx(j)] = x; }
+                }
+            }
+            __syncwarp();
+        }
+    }
+    if (A.dbg_keys_sorted) {
+        const uint32_t o = A.dbg_off[site - A.w0];
+        for (uint32_t e = lane; e < n; e += 32) A.dbg_keys_sorted[o + e] = col[idx(e)];
+        __syncwarp();
+    }
+    walk_chunks(A, col, idx, n, slotcnt);
+    double acc[10];
+#pragma unroll
+    for (int j = 0; j < 10; ++j) acc[j] = 0.0;
+    uint32_t cu[4] = {0, 0, 0, 0}, qs[4] = {0, 0, 0, 0};
+    for (uint32_t e = lane; e < n; e += 32) {
+        const uint32_t kk = col[idx(e)];
+        const uint32_t b = key_base(kk);
+        add_row(A.T, A.L, kk >> 17, key_cyc(kk), b, acc);
+#pragma unroll
+        for (int x = 0; x < 4; ++x) { cu[x] += b == (uint32_t)x; qs[x] += b == (uint32_t)x ? key_q(kk) : 0u; }
+    }
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) {
+#pragma unroll
+        for (int j = 0; j < 10; ++j) acc[j] += __shfl_xor_sync(FULL, acc[j], d);
+#pragma unroll
+        for (int x = 0; x < 4; ++x) {
+            cu[x] += __shfl_xor_sync(FULL, cu[x], d);
+            qs[x] += __shfl_xor_sync(FULL, qs[x], d);
+        }
+    }
+    int refb;
+    const int64_t kidx = site_ref(A, site, refb);
+    double wsum = 0.0, tie = 0.0;
+    {
+        const double* prow = kidx >= 0 ? A.known_lp + kidx * 10 : A.LP + refb * 10;
+        double lp[10];
+        for (int j = 0; j < 10; ++j) lp[j] = acc[j] + prow[j];
+        int t1, t2;
+        top2(lp, t1, t2);
+        const int a1 = geno_a1(t1), a2 = geno_a2(t1);
+        if (a1 != a2 && (A.flags & GSNP_RANK_SUM) && lane == 0) hist_ranks(col, idx, n, a1, a2, wsum, tie);
+        wsum = __shfl_sync(FULL, wsum, 0);
+        tie = __shfl_sync(FULL, tie, 0);
+    }
+    group_epilogue(A, site, refb, kidx, acc, cu, qs, ca0, ca1, ca2, ca3, rep, wsum, tie);
+    __syncwarp();
 }
 
 // In-place ascending bitonic sort of a[0..n) in shared memory by the whole CTA (n arbitrary:
@@ -707,46 +983,19 @@ __device__ void cta_sort(uint32_t* a, uint32_t n) {
     }
 }
 
-// CTA path for 256 < n <= deep_cap: keys gathered into the col region, CTA bitonic sort,
-// warp 0 walks the chunks for the dependency counters (q_adj stored in key bits 17..22), all
-// warps gather and reduce, warp 0 finishes.
-__device__ __noinline__ void cta_site(const CallArgs& A, const TileSmem& sm, uint32_t* a,
-                                      uint32_t n, uint64_t site, int site_local,
-                                      const double* sLP, double* red) {
+// CTA path for n > 1024 (k_big_sites): keys in one shared buffer, CTA bitonic sort,
+// warp 0 walks the chunks, all warps gather and reduce, warp 0 finishes.
+__device__ __noinline__ void cta_site(const CallArgs& A, uint8_t* slotcnt, uint32_t* a,
+                                      uint32_t n, uint64_t site, uint32_t ca0, uint32_t ca1,
+                                      uint32_t ca2, uint32_t ca3, uint32_t rep, double* red) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int L2 = 2 * A.L;
+    auto flat = [](uint32_t e) { return e; };
     cta_sort(a, n);
     if (A.dbg_keys_sorted) {
         const uint32_t o = A.dbg_off[site - A.w0];
         for (uint32_t e = threadIdx.x; e < n; e += NT) A.dbg_keys_sorted[o + e] = a[e];
     }
-    if (warp == 0) {
-        uint8_t* slotcnt = sm.slotcnt;
-        int d0 = 0, d1 = 0, d2 = 0, d3 = 0;
-        const uint32_t lt = lanemask_lt(), le = lt | (1u << lane);
-        for (uint32_t c0 = 0; c0 < n; c0 += 32) {
-            const uint32_t e = c0 + lane;
-            const bool valid = e < n;
-            const uint32_t kk = valid ? a[e] : KEY_INF;
-            const uint32_t b = key_base(kk), q = key_q(kk), slot = key_slot(kk);
-            const uint32_t peers = __match_any_sync(FULL, valid ? (b << 9 | slot) : (0x80000000u | lane));
-            uint32_t pcr = 1u + __popc(peers & lt) + (valid ? slotcnt[b * L2 + slot] : 0u);
-            const bool first = valid && pcr == 1u;
-            const uint32_t fb = __ballot_sync(FULL, first);
-            const uint32_t bmask = __match_any_sync(FULL, valid ? b : (0x80000000u | lane));
-            const int db = b == 0 ? d0 : b == 1 ? d1 : b == 2 ? d2 : d3;
-            const uint32_t g = (uint32_t)(db + __popc(fb & bmask & le) - 1);
-            if (valid && (peers >> lane) == 1u) slotcnt[b * L2 + slot] = (uint8_t)min(pcr, 255u);
-            d0 += __popc(fb & __ballot_sync(FULL, valid && b == 0));
-            d1 += __popc(fb & __ballot_sync(FULL, valid && b == 1));
-            d2 += __popc(fb & __ballot_sync(FULL, valid && b == 2));
-            d3 += __popc(fb & __ballot_sync(FULL, valid && b == 3));
-            __syncwarp();
-            if (valid) a[e] = (kk & 0x1FFFFu) | (uint32_t)adj_lookup(A, q, pcr, g) << 17;
-        }
-        __syncwarp();
-        for (uint32_t e = lane; e < n; e += 32) slotcnt[key_base(a[e]) * L2 + key_slot(a[e])] = 0;
-    }
+    if (warp == 0) walk_chunks(A, a, flat, n, slotcnt);
     __syncthreads();
     double acc[10];
 #pragma unroll
@@ -777,70 +1026,56 @@ __device__ __noinline__ void cta_site(const CallArgs& A, const TileSmem& sm, uin
         }
     }
     __syncthreads();
-    __shared__ double rk[2];
-    const int refb = A.ref[site - A.origin];
-    const int64_t kidx = known_index(A, site);
-    double L10[10];
-    uint32_t cut[4], qst[4];
+    if (warp == 0) {
+        int refb;
+        const int64_t kidx = site_ref(A, site, refb);
+        double L10[10];
+        uint32_t cut[4], qst[4];
 #pragma unroll
-    for (int j = 0; j < 10; ++j) {
-        double v = 0.0;
-        for (int w = 0; w < NW; ++w) v += red[w * 18 + j];
-        L10[j] = v;
-    }
+        for (int j = 0; j < 10; ++j) {
+            double v = 0.0;
+            for (int w = 0; w < NW; ++w) v += red[w * 18 + j];
+            L10[j] = v;
+        }
 #pragma unroll
-    for (int x = 0; x < 4; ++x) {
-        double c = 0.0, qq = 0.0;
-        for (int w = 0; w < NW; ++w) { c += red[w * 18 + 10 + x]; qq += red[w * 18 + 14 + x]; }
-        cut[x] = (uint32_t)c;
-        qst[x] = (uint32_t)qq;
-    }
-    if (threadIdx.x == 0) {
-        // rank-sum pieces by histogram over the 64 quality values (het calls only)
+        for (int x = 0; x < 4; ++x) {
+            double c = 0.0, qq = 0.0;
+            for (int w = 0; w < NW; ++w) { c += red[w * 18 + 10 + x]; qq += red[w * 18 + 14 + x]; }
+            cut[x] = (uint32_t)c;
+            qst[x] = (uint32_t)qq;
+        }
         double wsum = 0.0, tie = 0.0;
-        const double* prow = kidx >= 0 ? A.known_lp + kidx * 10 : sLP + refb * 10;
+        const double* prow = kidx >= 0 ? A.known_lp + kidx * 10 : A.LP + refb * 10;
         double lp[10];
         for (int j = 0; j < 10; ++j) lp[j] = L10[j] + prow[j];
         int t1, t2;
         top2(lp, t1, t2);
         const int a1 = geno_a1(t1), a2 = geno_a2(t1);
-        if (a1 != a2 && (A.flags & GSNP_RANK_SUM)) {
-            uint32_t hx[64], hy[64];
-            for (int v = 0; v < 64; ++v) { hx[v] = 0; hy[v] = 0; }
-            for (uint32_t e = 0; e < n; ++e) {
-                uint32_t b = key_base(a[e]), q = key_q(a[e]);
-                if (b == (uint32_t)a1) hx[q]++;
-                else if (b == (uint32_t)a2) hy[q]++;
-            }
-            double less = 0.0;
-            for (int v = 0; v < 64; ++v) {
-                double t = (double)hx[v] + (double)hy[v];
-                wsum += (double)hx[v] * (less + (t + 1.0) / 2.0);
-                tie += t * t * t - t;
-                less += t;
-            }
-        }
-        rk[0] = wsum;
-        rk[1] = tie;
+        if (a1 != a2 && (A.flags & GSNP_RANK_SUM) && lane == 0) hist_ranks(a, flat, n, a1, a2, wsum, tie);
+        wsum = __shfl_sync(FULL, wsum, 0);
+        tie = __shfl_sync(FULL, tie, 0);
+        group_epilogue(A, site, refb, kidx, L10, cut, qst, ca0, ca1, ca2, ca3, rep, wsum, tie);
     }
-    __syncthreads();
-    if (warp == 0)
-        group_epilogue(A, site, refb, kidx, sLP, L10, cut, qst, sm.cnt_all[0 * TS + site_local],
-                       sm.cnt_all[1 * TS + site_local], sm.cnt_all[2 * TS + site_local],
-                       sm.cnt_all[3 * TS + site_local], sm.rep[site_local], rk[0], rk[1]);
     __syncthreads();
 }
 
 // ------------------------------------------------------------------------------------------
-// The fused per-tile kernel (a4..a8): counting + base_word gather (site-major, no atomics),
-// likelihood_sort + likelihood_comp + posterior + record, per site.
-__global__ void __launch_bounds__(NT, 2) k_call_tile(CallArgs A) {
+// Sites with more than 32*COLS unique keys are handed to k_big_sites through a global list.
+struct BigSite {
+    uint64_t site;
+    uint32_t n, ca0, ca1, ca2, ca3, rep;
+};
+
+// The fused per-tile kernel (a4..a8).  Every warp owns 32 consecutive sites and works
+// independently (no CTA barrier): counting + base_word gather (site-major, no atomics), then
+// thread-per-site sort + likelihood + posterior + record; its sites with more than 32 keys
+// follow on the warp paths; beyond 1024 keys they go to k_big_sites.
+#ifndef GSNP_CALL_MINB
+#define GSNP_CALL_MINB 2
+#endif
+__global__ void __launch_bounds__(NT, GSNP_CALL_MINB) k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n,
+                                                     uint32_t big_cap) {
     extern __shared__ __align__(16) unsigned char smem[];
-    __shared__ double sLP[50];
-    __shared__ double red[NW * 18];
-    __shared__ uint64_t wr[NW][2];
-    __shared__ uint32_t ovf_n, deep_n;
-    __shared__ uint16_t ovf[TS], deep[TS];
     TileSmem sm;
     call_smem_bytes(A.L, &sm, smem);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -848,26 +1083,26 @@ __global__ void __launch_bounds__(NT, 2) k_call_tile(CallArgs A) {
     const uint64_t site = t0 + tid;
     const bool active = site < A.w1;
     const uint64_t grp = (uint64_t)blockIdx.x * NW + warp;
-    const bool wactive = t0 + warp * 32 < A.w1;
-    const uint64_t wra = wactive ? A.tile_ra[grp] : 0, wrb = wactive ? A.tile_rb[grp] : 0;
-    if (tid < 50) sLP[tid] = A.LP[tid];
-    if (tid == 0) { ovf_n = 0; deep_n = 0; }
-    if (lane == 0) { wr[warp][0] = wra; wr[warp][1] = wrb; }
-    for (int i = tid; i < NW * 2 * A.L; i += NT) reinterpret_cast<uint32_t*>(sm.slotcnt)[i] = 0;
+    if (t0 + warp * 32 >= A.w1) return;                      // whole warp past the window
+    const uint64_t wra = A.tile_ra[grp], wrb = A.tile_rb[grp];
+    uint8_t* myslot = sm.slotcnt + warp * 8 * A.L;
+    for (int i = lane; i < 2 * A.L; i += 32) reinterpret_cast<uint32_t*>(myslot)[i] = 0;
+    uint32_t* colp = sm.col + tid;                           // this site's column
 
     // ---- counting + base_word gather, one site per lane.  The warp
-    // walks the reads covering its 32 sites; metadata for 32 reads is loaded coalesced and
-    // broadcast by shuffles; each lane reads the base at its own site (consecutive lanes ->
-    // consecutive bytes of the read).
+    // walks the reads covering its 32 sites: metadata of 32 reads is loaded coalesced and
+    // broadcast by shuffles; each lane reads the base and quality at its own site (consecutive
+    // lanes -> consecutive bytes of a read).  Loads are issued four reads at a time.
     uint32_t ca0 = 0, ca1 = 0, ca2 = 0, ca3 = 0, rep = 0, n = 0;
-    bool dup = false, have_minus = false;
-    uint64_t last_plus = ~0ull, last_end = 0;
+    bool slow_pcr = false, have_minus = false;
+    uint64_t run_pos = ~0ull, last_end = 0, last_end_pos = 0;
+    uint32_t run_start = 0;
     int err = 0;
+    uint32_t* dbg_built = A.dbg_keys_built ? A.dbg_keys_built + (active ? A.dbg_off[site - A.w0] : 0) : nullptr;
     for (uint64_t r0 = wra; r0 < wrb; r0 += 32) {
         const uint64_t r = r0 + lane;
-        uint64_t p = 0, o = 0;
-        uint32_t lh = 0;                          // len | hits << 16 ... packed with strand
-        uint32_t st = 0;
+        uint64_t p = ~0ull, o = 0;
+        uint32_t lh = 0, st = 0;
         if (r < wrb) {
             p = A.R.pos[r];
             o = A.R.off[r] - A.R.off0;
@@ -875,30 +1110,63 @@ __global__ void __launch_bounds__(NT, 2) k_call_tile(CallArgs A) {
             st = A.R.strand[r];
         }
         const int nr = (int)min((uint64_t)32, wrb - r0);
-#pragma unroll 4
-        for (int k = 0; k < nr; ++k) {
-            const uint64_t pk = __shfl_sync(FULL, p, k);
-            const uint64_t ok = __shfl_sync(FULL, o, k);
-            const uint32_t lhk = __shfl_sync(FULL, lh, k);
-            const uint32_t sk = __shfl_sync(FULL, st, k);
-            const uint32_t lk = lhk & 0xFFFFu, hk = lhk >> 16;
-            const uint64_t i = site - pk;         // wraps (huge) when site < pk
-            if (!active || i >= lk) continue;
-            const uint32_t b = A.R.bases[ok + i];
-            if (b >= 4) { if (b > 4) err |= ERR_RANGE; continue; }
-            ca0 += b == 0; ca1 += b == 1; ca2 += b == 2; ca3 += b == 3;
-            rep += hk;
-            if (hk != 1) continue;
-            const uint32_t q = A.R.quals[ok + i];
-            if (q > (uint32_t)A.q_max) { err |= ERR_QUAL; continue; }
-            const uint32_t cyc = sk ? lk - 1 - (uint32_t)i : (uint32_t)i;
-            const uint32_t key = b << 15 | (63u - q) << 9 | cyc << 1 | sk;
-            if (n < COLS) sm.col[n * TS + tid] = key;
-            if (A.dbg_keys_built) A.dbg_keys_built[A.dbg_off[site - A.w0] + n] = key;
-            ++n;
-            // same (strand, coord) twice at a site <=> same start on '+', same end on '-'
-            if (sk == 0) { dup |= pk == last_plus; last_plus = pk; }
-            else { const uint64_t e = pk + lk - 1; dup |= have_minus && e <= last_end; last_end = e; have_minus = true; }
+        for (int k0 = 0; k0 < nr; k0 += 4) {
+            uint64_t pk[4], ii[4];
+            uint32_t lk[4], hk[4], sk[4], bb[4], qq[4];
+            bool cov[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                const int k = (k0 + u) & 31;
+                pk[u] = __shfl_sync(FULL, p, k);
+                const uint64_t ok = __shfl_sync(FULL, o, k);
+                const uint32_t lhk = __shfl_sync(FULL, lh, k);
+                sk[u] = __shfl_sync(FULL, st, k);
+                lk[u] = lhk & 0xFFFFu;
+                hk[u] = lhk >> 16;
+                ii[u] = site - pk[u];             // wraps (huge) when site < pos
+                cov[u] = active && k0 + u < nr && ii[u] < lk[u];
+                bb[u] = cov[u] ? A.R.bases[ok + ii[u]] : 4u;
+                qq[u] = cov[u] ? A.R.quals[ok + ii[u]] : 0u;
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                const uint32_t b = bb[u], q = qq[u];
+                const bool nb = cov[u] && b < 4;                 // a non-N aligned base
+                err |= (cov[u] && b > 4) ? ERR_RANGE : 0;
+                ca0 += nb && b == 0; ca1 += nb && b == 1; ca2 += nb && b == 2; ca3 += nb && b == 3;
+                rep += nb ? hk[u] : 0u;
+                const bool uni = nb && hk[u] == 1;               // uniquely aligned
+                err |= (uni && q > (uint32_t)A.q_max) ? ERR_QUAL : 0;
+                const bool use = uni && q <= (uint32_t)A.q_max;
+                const uint32_t i = (uint32_t)ii[u];
+                const uint32_t cyc = sk[u] ? lk[u] - 1 - i : i;
+                const uint32_t key = b << 15 | (63u - q) << 9 | cyc << 1 | sk[u];
+                if (dbg_built && use) dbg_built[n] = key;
+                // pcr: keys sharing (base, strand, coord) come from reads with the same start
+                // ('+') or the same end ('-'); with equal starts they are one run of this
+                // column.  Canonical order among them is quality descending (R3).
+                if (pk[u] != run_pos) { run_pos = pk[u]; run_start = n; }
+                uint32_t pcr1 = 0;
+                if (use && run_start < n) {
+                    const uint32_t jend = min(n, (uint32_t)COLS);
+                    for (uint32_t j = run_start; j < jend; ++j) {
+                        const uint32_t kj = colp[j * TS];
+                        if ((((kj >> 8) ^ key) & KEY_BSLOT) == 0) {
+                            if (key_q(kj >> 8) >= q) ++pcr1;
+                            else if ((kj & 255u) < 255u) colp[j * TS] = kj + 1;
+                        }
+                    }
+                }
+                // '-' ends must rise between start runs, else recount pcr in thread_site
+                const uint64_t e = pk[u] + lk[u] - 1;
+                const bool minus = use && sk[u];
+                slow_pcr |= minus && have_minus && (e < last_end || (e == last_end && pk[u] != last_end_pos));
+                last_end = minus ? e : last_end;
+                last_end_pos = minus ? pk[u] : last_end_pos;
+                have_minus |= minus;
+                if (use && n < COLS) colp[n * TS] = key << 8 | min(pcr1, 255u);
+                n += use;
+            }
         }
     }
     if (err) atomicOr(A.err, err);
@@ -906,75 +1174,69 @@ __global__ void __launch_bounds__(NT, 2) k_call_tile(CallArgs A) {
         if (active) A.dbg_nuni[site - A.w0] = n;
         return;
     }
-    sm.cnt_all[0 * TS + tid] = ca0; sm.cnt_all[1 * TS + tid] = ca1;
-    sm.cnt_all[2 * TS + tid] = ca2; sm.cnt_all[3 * TS + tid] = ca3;
-    sm.rep[tid] = rep;
-    sm.nuni[tid] = n;
-    __syncthreads();
 
-    // ---- thread-per-site likelihood for n <= 32 (network size chosen per warp: 8/16/32)
+    // ---- thread-per-site sort (in-register network sized per warp: 16 / 32) + likelihood
     const bool small = active && n <= COLS;
-    if (active && !small) {
-        if (n <= WBUF) ovf[atomicAdd(&ovf_n, 1u)] = (uint16_t)tid;
-        else deep[atomicAdd(&deep_n, 1u)] = (uint16_t)tid;
-    }
     const uint32_t maxn = __reduce_max_sync(FULL, small ? n : 0u);
     if (small) {
-        if (maxn <= 8) thread_site<8>(A, sm, site, n, dup, ca0, ca1, ca2, ca3, rep, sLP);
-        else if (maxn <= 16) thread_site<16>(A, sm, site, n, dup, ca0, ca1, ca2, ca3, rep, sLP);
-        else thread_site<32>(A, sm, site, n, dup, ca0, ca1, ca2, ca3, rep, sLP);
+        if (maxn <= 16) sort_column<16>(colp, n);
+        else sort_column<32>(colp, n);
+        thread_site(A, colp, site, n, slow_pcr, ca0, ca1, ca2, ca3, rep);
     }
-    __syncthreads();
+    __syncwarp();
 
-    // ---- warp path: 32 < n <= 256 (keys re-gathered from the owning warp's reads)
-    uint32_t* buf = sm.wbuf + warp * WBUF;
-    uint8_t* myslot = sm.slotcnt + warp * 8 * A.L;
-    for (uint32_t j = warp; j < ovf_n; j += NW) {
-        const int sl = ovf[j];
-        const uint64_t s = t0 + sl;
-        const uint64_t ra = wr[sl >> 5][0], rb = wr[sl >> 5][1];
-        uint32_t m = 0;
-        for (uint64_t r0 = ra; r0 < rb; r0 += 32) {
-            const uint64_t r = r0 + lane;
-            uint32_t key = KEY_INF;
-            if (r < rb && A.R.hits[r] == 1) {
-                const uint64_t i = s - A.R.pos[r];
-                const uint32_t l = A.R.len[r];
-                if (i < l) {
-                    const uint64_t bi = A.R.off[r] - A.R.off0 + i;
-                    const uint32_t b = A.R.bases[bi];
-                    if (b < 4) {
-                        const uint32_t st = A.R.strand[r];
-                        const uint32_t cyc = st ? l - 1 - (uint32_t)i : (uint32_t)i;
-                        key = b << 15 | (63u - A.R.quals[bi]) << 9 | cyc << 1 | st;
-                    }
-                }
+    // ---- this warp's deeper sites: warp paths (n <= 1024) or the k_big_sites list
+    uint32_t ovf = __ballot_sync(FULL, active && n > COLS);
+    while (ovf) {
+        const int l = __ffs(ovf) - 1;
+        ovf &= ovf - 1;
+        const uint32_t nn = __shfl_sync(FULL, n, l);
+        const uint32_t c0 = __shfl_sync(FULL, ca0, l), c1 = __shfl_sync(FULL, ca1, l);
+        const uint32_t c2 = __shfl_sync(FULL, ca2, l), c3 = __shfl_sync(FULL, ca3, l);
+        const uint32_t rp = __shfl_sync(FULL, rep, l);
+        const uint64_t s = t0 + warp * 32 + l;
+        if (nn > 32 * COLS) {
+            if (lane == l) {
+                const uint32_t j = atomicAdd(big_n, 1u);
+                if (j < big_cap) big[j] = BigSite{s, nn, c0, c1, c2, c3, rp};
+                else atomicOr(A.err, ERR_DEEP);
             }
-            const uint32_t v = __ballot_sync(FULL, key != KEY_INF);
-            if (key != KEY_INF) buf[m + __popc(v & lanemask_lt())] = key;
-            m += __popc(v);
+            continue;
         }
-        __syncwarp();
-        const uint32_t c0 = sm.cnt_all[sl], c1 = sm.cnt_all[TS + sl], c2 = sm.cnt_all[2 * TS + sl],
-                       c3 = sm.cnt_all[3 * TS + sl], rp = sm.rep[sl];
-        if (m <= 64) warp_site<2>(A, buf, m, s, c0, c1, c2, c3, rp, sLP, myslot);
-        else if (m <= 128) warp_site<4>(A, buf, m, s, c0, c1, c2, c3, rp, sLP, myslot);
-        else warp_site<8>(A, buf, m, s, c0, c1, c2, c3, rp, sLP, myslot);
+        const uint32_t m = warp_gather(A, sm.col, warp, s, wra, wrb);
+        if (m <= 64) warp_site<2>(A, sm.col, warp, m, s, c0, c1, c2, c3, rp, myslot);
+        else if (m <= 128) warp_site<4>(A, sm.col, warp, m, s, c0, c1, c2, c3, rp, myslot);
+        else if (m <= 256) warp_site<8>(A, sm.col, warp, m, s, c0, c1, c2, c3, rp, myslot);
+        else warp_deep_site(A, sm.col, warp, m, s, c0, c1, c2, c3, rp, myslot);
         __syncwarp();
     }
-    // ---- CTA path: n > 256, one site at a time in the col region
-    for (uint32_t j = 0; j < deep_n; ++j) {
-        __syncthreads();
-        const int sl = deep[j];
-        const uint64_t s = t0 + sl;
-        if (sm.nuni[sl] > (uint32_t)sm.deep_cap) {
+}
+
+// Sites with more than 1024 unique keys: one CTA per site (persistent loop over the list),
+// keys gathered into a shared buffer of `cap` keys (GSNP_E_CAPACITY beyond it).
+__global__ void __launch_bounds__(NT) k_big_sites(CallArgs A, const BigSite* big,
+                                                  const uint32_t* big_n, uint32_t cap) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    __shared__ double red[NW * 18];
+    __shared__ uint32_t cnt;
+    uint32_t* buf = reinterpret_cast<uint32_t*>(smem);
+    uint8_t* slotcnt = smem + 4 * (size_t)cap;
+    const int tid = threadIdx.x;
+    for (int i = tid; i < 2 * A.L; i += NT) reinterpret_cast<uint32_t*>(slotcnt)[i] = 0;
+    const uint32_t count = *big_n;
+    for (uint32_t j = blockIdx.x; j < count; j += gridDim.x) {
+        const BigSite bs = big[j];
+        if (bs.n > cap) {
             if (tid == 0) atomicOr(A.err, ERR_DEEP);
             continue;
         }
-        __shared__ uint32_t cnt;
+        __syncthreads();
         if (tid == 0) cnt = 0;
         __syncthreads();
-        const uint64_t ra = wr[sl >> 5][0], rb = wr[sl >> 5][1];
+        const uint64_t s = bs.site;
+        const uint64_t lo = s >= (uint64_t)(A.L - 1) ? s - (A.L - 1) : 0;
+        const uint64_t ra = lower_bound_u64(A.R.pos, 0, A.R.n, lo);
+        const uint64_t rb = lower_bound_u64(A.R.pos, ra, A.R.n, s + 1);
         for (uint64_t r = ra + tid; r < rb; r += NT) {
             if (A.R.hits[r] != 1) continue;
             const uint64_t i = s - A.R.pos[r];
@@ -985,10 +1247,13 @@ __global__ void __launch_bounds__(NT, 2) k_call_tile(CallArgs A) {
             if (b >= 4) continue;
             const uint32_t st = A.R.strand[r];
             const uint32_t cyc = st ? l - 1 - (uint32_t)i : (uint32_t)i;
-            sm.col[atomicAdd(&cnt, 1u)] = b << 15 | (63u - A.R.quals[bi]) << 9 | cyc << 1 | st;
+            const uint32_t key = b << 15 | (63u - A.R.quals[bi]) << 9 | cyc << 1 | st;
+            const uint32_t slot = atomicAdd(&cnt, 1u);
+            buf[slot] = key;
+            if (A.dbg_keys_built) A.dbg_keys_built[A.dbg_off[s - A.w0] + slot] = key;
         }
         __syncthreads();
-        cta_site(A, sm, sm.col, cnt, s, sl, sLP, red);
+        cta_site(A, slotcnt, buf, cnt, s, bs.ca0, bs.ca1, bs.ca2, bs.ca3, bs.rep, red);
     }
 }
 

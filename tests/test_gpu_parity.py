@@ -217,3 +217,38 @@ def test_errors_are_statuses():
         assert e.value.status == -2
         rec = ctx.call(w, 0, 2_000)                        # still usable after errors
         assert len(rec) == 2_000
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_variable_length_reads_parity(seed):
+    """Reads of unequal length: '-' strand reads ending at the same coordinate share a cycle
+    from different starts; same-start reads of unequal length do not."""
+    rng = np.random.default_rng(100 + seed)
+    S = 600
+    ref = rng.integers(0, 4, S).astype(np.uint8)
+    reads = []
+    for _ in range(260):
+        ln = int(rng.integers(30, 101))
+        p = int(rng.integers(0, S - ln))
+        st = int(rng.integers(2))
+        b = ref[p:p + ln].copy()
+        err = rng.random(ln) < 0.05
+        b[err] = (b[err] + rng.integers(1, 4, err.sum())) % 4
+        q = list(rng.integers(2, 41, ln))
+        reads.append(dict(pos=p, strand=st, hits=1 if rng.random() > 0.05 else 2, bases=b, quals=q))
+        if rng.random() < 0.3:                 # partner ending at the same coordinate on '-'
+            ln2 = int(rng.integers(30, 101))
+            p2 = p + ln - ln2
+            if 0 <= p2 <= S - ln2:
+                reads.append(dict(pos=p2, strand=1, bases=ref[p2:p2 + ln2],
+                                  quals=list(rng.integers(2, 41, ln2))))
+        if rng.random() < 0.2:                 # same start, other length / strand
+            ln3 = int(rng.integers(30, 101))
+            if p + ln3 <= S:
+                reads.append(dict(pos=p, strand=int(rng.integers(2)), bases=ref[p:p + ln3],
+                                  quals=list(rng.integers(2, 41, ln3))))
+    w = workload(ref, reads)
+    C, p, _, _ = _oracle_all(w, w0=0, w1=1)
+    with _ctx(w) as ctx:
+        ctx.calibrate(w)
+        _check_window(ctx, w, 0, S, C, p)
