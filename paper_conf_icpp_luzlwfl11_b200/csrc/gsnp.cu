@@ -382,14 +382,23 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
     A.tile_rb = ctx->tile_rb.p;
     A.out = d_out;
     A.err = ctx->d_err.p;
-    const size_t smem = call_smem_bytes(A.L, nullptr, nullptr);
+    // persistent CTAs; warps pull 32-site groups from a counter.  The adjust table rides in
+    // shared memory when small (it is 64 x 7 x 37 bytes at the default coefficients).
+    const size_t adj_bytes = (size_t)64 * A.adjP * A.adjG;
+    const uint32_t adj_smem = adj_bytes <= 48 * 1024 ? 1u : 0u;
+    const size_t smem = call_smem_bytes(A.L, adj_smem ? adj_bytes : 0, nullptr, nullptr);
     const uint32_t big_cap = (uint32_t)std::min<uint64_t>(w1 - w0, 1u << 22);
     CK(ctx->big.ensure(big_cap));
-    CK(ctx->big_n.ensure(1));
-    CK(cudaMemsetAsync(ctx->big_n.p, 0, 4, s));
+    CK(ctx->big_n.ensure(2));
+    CK(cudaMemsetAsync(ctx->big_n.p, 0, 8, s));     // [0] big-site count, [1] work counter
     CK(cudaFuncSetAttribute(k_call_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int per_sm = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_call_tile, NT, smem));
+    const uint64_t want = (uint64_t)g_num_sms * std::max(per_sm, 1);
+    const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, n_tiles));
     ctx->begin();
-    k_call_tile<<<(unsigned)n_tiles, NT, smem, s>>>(A, ctx->big.p, ctx->big_n.p, big_cap);
+    k_call_tile<<<grid, NT, smem, s>>>(A, ctx->big.p, ctx->big_n.p, big_cap, ctx->big_n.p + 1,
+                                       adj_smem);
     ctx->end(GSNP_STAGE_CALL);
     ctx->launches++;
     CK(cudaGetLastError());

@@ -328,15 +328,19 @@ struct TileSmem {
     uint32_t* col;       // [COLS][TS] keys: column of site t at col[j*TS + t]; a warp's 32
                          // columns double as its 1024-key buffer on the warp paths
     uint8_t* slotcnt;    // [NW][4 * 2L] per-warp (base, strand, coord) counters
+    uint8_t* adj;        // copy of the adjust table (adj_bytes, 0 = use global)
 };
 
-__host__ __device__ inline size_t call_smem_bytes(int L, TileSmem* s, unsigned char* base) {
+__host__ __device__ inline size_t call_smem_bytes(int L, size_t adj_bytes, TileSmem* s,
+                                                   unsigned char* base) {
     size_t o_col = 0;
     size_t o_slot = align16(4 * (size_t)COLS * TS);
-    size_t total = align16(o_slot + (size_t)NW * 8 * L);
+    size_t o_adj = align16(o_slot + (size_t)NW * 8 * L);
+    size_t total = align16(o_adj + adj_bytes);
     if (s) {
         s->col = reinterpret_cast<uint32_t*>(base + o_col);
         s->slotcnt = base + o_slot;
+        s->adj = base + o_adj;
     }
     return total;
 }
@@ -362,6 +366,12 @@ __device__ __forceinline__ void add_row(const double* __restrict__ T, int L, uin
 __device__ __forceinline__ int adj_lookup(const CallArgs& A, uint32_t q, uint32_t pcr, uint32_t g) {
     uint32_t pi = min(pcr, (uint32_t)A.adjP) - 1u, gi = min(g, (uint32_t)A.adjG - 1u);
     return __ldg(A.adj + ((size_t)q * A.adjP + pi) * A.adjG + gi);
+}
+// same, from a copy of the table (shared memory in k_call_tile)
+__device__ __forceinline__ int adj_lookup_t(const uint8_t* adj, int P, int G, uint32_t q,
+                                            uint32_t pcr, uint32_t g) {
+    uint32_t pi = min(pcr, (uint32_t)P) - 1u, gi = min(g, (uint32_t)G - 1u);
+    return adj[(q * (uint32_t)P + pi) * (uint32_t)G + gi];
 }
 
 // ---- per-site epilogue helpers ---------------------------------------------------------------
@@ -525,36 +535,45 @@ __device__ __forceinline__ void sort_column(uint32_t* colp, uint32_t n) {
     for (int j = 0; j < N; ++j) if (j < (int)n) colp[j * TS] = k[j];
 }
 
-__device__ __noinline__ void thread_site(const CallArgs& A, uint32_t* colp, uint64_t site,
-                                         uint32_t n, bool slow_pcr, uint32_t ca0, uint32_t ca1,
-                                         uint32_t ca2, uint32_t ca3, uint32_t rep) {
+__device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* adj, uint32_t* colp,
+                                            uint64_t site, uint32_t n, bool slow_pcr, uint32_t ca0,
+                                            uint32_t ca1, uint32_t ca2, uint32_t ca3, uint32_t rep) {
     if (A.dbg_keys_sorted) {
         const uint32_t o = A.dbg_off[site - A.w0];
         for (uint32_t j = 0; j < n; ++j) A.dbg_keys_sorted[o + j] = colp[j * TS] >> 8;
     }
-    // Alg. 4 lines 6-17 in canonical order: dep_count reset per base (l.8-11); pcr from the
-    // gather, or recounted when '-' strand reads of unequal length can share a coordinate;
-    // g = distinct (strand, coord) so far in this base - 1 (R3).
-    double acc[10];
-#pragma unroll
-    for (int j = 0; j < 10; ++j) acc[j] = 0.0;
+    // Alg. 4 lines 6-17 in canonical order, pass 1 (integers): dep_count reset per base
+    // (l.8-11); pcr from the gather, or recounted when '-' strand reads of unequal length can
+    // share a coordinate; g = distinct (strand, coord) so far in this base - 1 (R3);
+    // q_adj = adjust(q, pcr, g).  Each key becomes key | q_adj << 17.
     uint64_t cu = 0, qs = 0;
     uint32_t prev_b = 4, distinct = 0;
-#pragma unroll 4
     for (uint32_t j = 0; j < n; ++j) {
         const uint32_t kw = colp[j * TS];
         const uint32_t kk = kw >> 8, b = key_base(kk), q = key_q(kk);
         uint32_t pcr = (kw & 255u) + 1u;
         if (slow_pcr) {
             pcr = 1;
-            for (uint32_t i = 0; i < j; ++i) pcr += (((colp[i * TS] >> 8) ^ kk) & KEY_BSLOT) == 0;
+            // entries before j already hold key | q_adj << 17
+            for (uint32_t i = 0; i < j; ++i) pcr += ((colp[i * TS] ^ kk) & KEY_BSLOT) == 0;
         }
         if (b != prev_b) { distinct = 0; prev_b = b; }
         distinct += pcr == 1;
-        const int qa = adj_lookup(A, q, pcr, distinct - 1);
-        add_row(A.T, A.L, (uint32_t)qa, key_cyc(kk), b, acc);
+        colp[j * TS] = kk | (uint32_t)adj_lookup_t(adj, A.adjP, A.adjG, q, pcr, distinct - 1) << 17;
         cu += 1ull << (16 * b);
         qs += (uint64_t)q << (16 * b);
+    }
+    // pass 2: type_likely[n] += new_p_matrix[row][n] (Alg. 3) in canonical order; no load
+    // depends on another, so four rows are in flight per thread
+    double acc[10];
+#pragma unroll
+    for (int j = 0; j < 10; ++j) acc[j] = 0.0;
+    const double* __restrict__ T = A.T;
+    const uint32_t L = (uint32_t)A.L;
+#pragma unroll 4
+    for (uint32_t j = 0; j < n; ++j) {
+        const uint32_t kk = colp[j * TS];
+        add_row(T, (int)L, kk >> 17, key_cyc(kk), key_base(kk), acc);
     }
     // C6/C7: priors, posterior, top-2
     int refb;
@@ -592,12 +611,12 @@ __device__ __noinline__ void thread_site(const CallArgs& A, uint32_t* colp, uint
     double wsum = 0.0, tie = 0.0;
     if (a1 != a2 && (A.flags & GSNP_RANK_SUM) && f16(cu, a1) && f16(cu, a2)) {
         for (uint32_t x = 0; x < n; ++x) {
-            const uint32_t xk = colp[x * TS] >> 8;
+            const uint32_t xk = colp[x * TS] & 0x1FFFFu;
             const uint32_t xb = key_base(xk), xq = key_q(xk);
             if (xb != (uint32_t)a1 && xb != (uint32_t)a2) continue;
             uint32_t less = 0, eq = 0;
             for (uint32_t y = 0; y < n; ++y) {
-                const uint32_t yk = colp[y * TS] >> 8, yb = key_base(yk), yq = key_q(yk);
+                const uint32_t yk = colp[y * TS] & 0x1FFFFu, yb = key_base(yk), yq = key_q(yk);
                 const bool yin = yb == (uint32_t)a1 || yb == (uint32_t)a2;
                 less += yin && yq < xq;
                 eq += yin && yq == xq;
@@ -1073,21 +1092,31 @@ struct BigSite {
 #ifndef GSNP_CALL_MINB
 #define GSNP_CALL_MINB 2
 #endif
-__global__ void __launch_bounds__(NT, GSNP_CALL_MINB) k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n,
-                                                     uint32_t big_cap) {
+__global__ void __launch_bounds__(NT, GSNP_CALL_MINB)
+k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_t* work,
+            uint32_t adj_smem) {
     extern __shared__ __align__(16) unsigned char smem[];
     TileSmem sm;
-    call_smem_bytes(A.L, &sm, smem);
+    const size_t adj_bytes = adj_smem ? (size_t)64 * A.adjP * A.adjG : 0;
+    call_smem_bytes(A.L, adj_bytes, &sm, smem);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const uint64_t t0 = A.w0 + (uint64_t)blockIdx.x * TS;
-    const uint64_t site = t0 + tid;
-    const bool active = site < A.w1;
-    const uint64_t grp = (uint64_t)blockIdx.x * NW + warp;
-    if (t0 + warp * 32 >= A.w1) return;                      // whole warp past the window
-    const uint64_t wra = A.tile_ra[grp], wrb = A.tile_rb[grp];
+    for (size_t i = tid; i < adj_bytes; i += NT) sm.adj[i] = A.adj[i];
+    const uint8_t* adj = adj_smem ? sm.adj : A.adj;
     uint8_t* myslot = sm.slotcnt + warp * 8 * A.L;
     for (int i = lane; i < 2 * A.L; i += 32) reinterpret_cast<uint32_t*>(myslot)[i] = 0;
-    uint32_t* colp = sm.col + tid;                           // this site's column
+    uint32_t* colp = sm.col + tid;                           // this lane's column
+    __syncthreads();
+    const uint64_t n_groups = (A.w1 - A.w0 + 31) / 32;
+    // persistent warps: each takes the next group of 32 consecutive sites from a counter
+    for (;;) {
+    uint64_t grp = 0;
+    if (lane == 0) grp = atomicAdd(work, 1u);
+    grp = __shfl_sync(FULL, grp, 0);
+    if (grp >= n_groups) break;
+    const uint64_t g0 = A.w0 + grp * 32;                     // first site of the group
+    const uint64_t site = g0 + lane;
+    const bool active = site < A.w1;
+    const uint64_t wra = A.tile_ra[grp], wrb = A.tile_rb[grp];
 
     // ---- counting + base_word gather, one site per lane.  The warp
     // walks the reads covering its 32 sites: metadata of 32 reads is loaded coalesced and
@@ -1172,7 +1201,7 @@ __global__ void __launch_bounds__(NT, GSNP_CALL_MINB) k_call_tile(CallArgs A, Bi
     if (err) atomicOr(A.err, err);
     if (A.count_only) {
         if (active) A.dbg_nuni[site - A.w0] = n;
-        return;
+        continue;
     }
 
     // ---- thread-per-site sort (in-register network sized per warp: 16 / 32) + likelihood
@@ -1181,7 +1210,7 @@ __global__ void __launch_bounds__(NT, GSNP_CALL_MINB) k_call_tile(CallArgs A, Bi
     if (small) {
         if (maxn <= 16) sort_column<16>(colp, n);
         else sort_column<32>(colp, n);
-        thread_site(A, colp, site, n, slow_pcr, ca0, ca1, ca2, ca3, rep);
+        thread_site(A, adj, colp, site, n, slow_pcr, ca0, ca1, ca2, ca3, rep);
     }
     __syncwarp();
 
@@ -1194,7 +1223,7 @@ __global__ void __launch_bounds__(NT, GSNP_CALL_MINB) k_call_tile(CallArgs A, Bi
         const uint32_t c0 = __shfl_sync(FULL, ca0, l), c1 = __shfl_sync(FULL, ca1, l);
         const uint32_t c2 = __shfl_sync(FULL, ca2, l), c3 = __shfl_sync(FULL, ca3, l);
         const uint32_t rp = __shfl_sync(FULL, rep, l);
-        const uint64_t s = t0 + warp * 32 + l;
+        const uint64_t s = g0 + l;
         if (nn > 32 * COLS) {
             if (lane == l) {
                 const uint32_t j = atomicAdd(big_n, 1u);
@@ -1210,6 +1239,7 @@ __global__ void __launch_bounds__(NT, GSNP_CALL_MINB) k_call_tile(CallArgs A, Bi
         else warp_deep_site(A, sm.col, warp, m, s, c0, c1, c2, c3, rp, myslot);
         __syncwarp();
     }
+    }  // persistent loop
 }
 
 // Sites with more than 1024 unique keys: one CTA per site (persistent loop over the list),
