@@ -108,10 +108,16 @@ def _dist():
 
 
 def make_shard(cfg_name: str, rank: int, ws: int):
+    """Weak scaling: rank r holds sites [r*n, (r+1)*n) of one genome of ws*n sites (the config's
+    recipe with its N blocks spread over the genome), generated region by region — the reads
+    covering the shard and the reference under them (shard.py)."""
     import synth
     base = synth.CONFIGS[cfg_name]
-    # weak scaling: rank r holds sites [r*n, (r+1)*n) of a genome of ws*n sites
-    cfg = base.scaled(seed=base.seed + 1000 * rank, origin=rank * base.n_sites)
+    if ws == 1:
+        return synth.generate(base)
+    n = base.n_sites
+    cfg = base.scaled(n_sites=n * ws, n_lead_frac=base.n_lead_frac / ws,
+                      n_blocks=base.n_blocks * ws, region_lo=rank * n, region_hi=(rank + 1) * n)
     return synth.generate(cfg)
 
 
@@ -183,14 +189,32 @@ def run_gpu(args):
     ws, rank, local = _dist()
     if ws != args.gpus:
         args.gpus = ws
+    # debug knobs to exercise the multi-rank flow on a one-GPU box (not for timing):
+    # GSNP_BENCH_BACKEND=gloo (collectives staged through host memory), GSNP_BENCH_SAME_GPU=1
+    backend = os.environ.get("GSNP_BENCH_BACKEND", "nccl")
+    if os.environ.get("GSNP_BENCH_SAME_GPU"):
+        local = 0
     torch.cuda.set_device(local)
     dist = None
     if ws > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+
+    def all_reduce_(t, op=None):
+        kw = {} if op is None else {"op": op}
+        if backend == "nccl":
+            dist.all_reduce(t, **kw)
+        else:
+            c = t.cpu()
+            dist.all_reduce(c, **kw)
+            t.copy_(c)
+    from paper_conf_icpp_luzlwfl11_b200 import shard
     w = make_shard(args.config, rank, ws)
-    S = len(w["ref"])
-    w0, w1 = int(w["origin"]), int(w["origin"]) + S
+    w0, w1 = w["region"]                      # this rank's sites; w["ref"] also covers the halo
+    S = w1 - w0
     stream = torch.cuda.current_stream()
     keys = ("pos", "len", "off", "bases", "quals", "strand", "hits")
     host = {k: torch.from_numpy(np.ascontiguousarray(w[k])) for k in keys}
@@ -201,16 +225,20 @@ def run_gpu(args):
     counts = torch.zeros(64 * 256 * 16, dtype=torch.uint64, device="cuda")
     out = torch.empty(40 * S, dtype=torch.uint8, device="cuda")
     rd = gsnp.make_reads(dev)
+    # calibration counts a read only on the rank that owns its start (no double counting)
+    ora, orb = shard.owned_reads(w["pos"], w0, w1)
+
+    def owned(d):
+        return dict(d, pos=d["pos"][ora:orb], len=d["len"][ora:orb], off=d["off"][ora:orb + 1],
+                    strand=d["strand"][ora:orb], hits=d["hits"][ora:orb])
 
     def step():
-        ctx.calibrate_count(rd_dict, counts)
+        ctx.calibrate_count(owned(dev), counts)
         if dist is not None:
-            c64 = counts.view(torch.int64)
-            dist.all_reduce(c64)
+            all_reduce_(counts.view(torch.int64))
         ctx.calibrate_finalize(counts)
         ctx.call_reads(rd, w0, w1, out)
 
-    rd_dict = dev
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
@@ -233,29 +261,67 @@ def run_gpu(args):
     st = ctx.stage_times(reset=True)
     t = torch.tensor([ms_total], dtype=torch.float64, device="cuda")
     if dist is not None:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        all_reduce_(t, dist.ReduceOp.MAX)
     ms_max = float(t.item())
     ms_step = ms_max / args.steps
     total_sites = S * ws
     value = total_sites / (ms_step / 1e3)
 
-    # ---- e2e: same metric through the public API with host (pinned) inputs and outputs
+    # ---- e2e: the same step through the public API with pinned host inputs and outputs, the
+    # host->device copy of the reads and the device->host copy of the records inside the timed
+    # region.  Transfers overlap compute: reads go up in chunks on a copy stream while the
+    # calibration counts each chunk that has arrived; records come down per window chunk while
+    # the next chunk is being called.
+    K = 8
     pinned = {k: v.pin_memory() for k, v in host.items()}
     out_h = torch.empty(40 * S, dtype=torch.uint8).pin_memory()
     dev2 = {k: torch.empty_like(v, device="cuda") for k, v in host.items()}
-    rd2 = gsnp.make_reads(dev2)
     h2d = sum(v.numel() * v.element_size() for v in pinned.values())
     d2h = out_h.numel()
+    nr_all = int(len(w["pos"]))
+    rcut = [nr_all * i // K for i in range(K + 1)]
+    ocut = [int(w["off"][r]) for r in rcut]
+    wcut = [w0 + S * i // K for i in range(K + 1)]
+    copy_stream = torch.cuda.Stream()
+    part = torch.zeros_like(counts)
 
     def e2e_step():
-        for k in keys:
-            dev2[k].copy_(pinned[k], non_blocking=True)
-        ctx.calibrate_count(dev2, counts)
+        evs = []
+        with torch.cuda.stream(copy_stream):
+            for i in range(K):
+                a, b, oa, ob = rcut[i], rcut[i + 1], ocut[i], ocut[i + 1]
+                for k in ("pos", "len", "strand", "hits"):
+                    dev2[k][a:b].copy_(pinned[k][a:b], non_blocking=True)
+                dev2["off"][a:b + 1].copy_(pinned["off"][a:b + 1], non_blocking=True)
+                dev2["bases"][oa:ob].copy_(pinned["bases"][oa:ob], non_blocking=True)
+                dev2["quals"][oa:ob].copy_(pinned["quals"][oa:ob], non_blocking=True)
+                e = torch.cuda.Event()
+                e.record(copy_stream)
+                evs.append(e)
+        counts.zero_()
+        for i in range(K):                    # count chunk i (owned reads only) once it landed
+            stream.wait_event(evs[i])
+            a, b = max(rcut[i], ora), min(rcut[i + 1], orb)
+            if a < b:
+                sub = dict(dev2, pos=dev2["pos"][a:b], len=dev2["len"][a:b],
+                           off=dev2["off"][a:b + 1], strand=dev2["strand"][a:b],
+                           hits=dev2["hits"][a:b])
+                ctx.calibrate_count(sub, part)
+                counts.view(torch.int64).add_(part.view(torch.int64))
         if dist is not None:
-            dist.all_reduce(counts.view(torch.int64))
+            all_reduce_(counts.view(torch.int64))
         ctx.calibrate_finalize(counts)
-        ctx.call_reads(rd2, w0, w1, out)
-        out_h.copy_(out, non_blocking=True)
+        rd2 = gsnp.make_reads(dev2)
+        for j in range(K):                    # call window chunk j, then ship its records
+            lo, hi = wcut[j], wcut[j + 1]
+            ctx.call_reads(rd2, lo, hi, out[40 * (lo - w0):40 * (hi - w0)])
+            e = torch.cuda.Event()
+            e.record(stream)
+            copy_stream.wait_event(e)
+            with torch.cuda.stream(copy_stream):
+                out_h[40 * (lo - w0):40 * (hi - w0)].copy_(out[40 * (lo - w0):40 * (hi - w0)],
+                                                           non_blocking=True)
+        stream.wait_stream(copy_stream)
 
     for _ in range(max(1, args.warmup // 2)):
         e2e_step()
@@ -269,9 +335,9 @@ def run_gpu(args):
     torch.cuda.synchronize()
     te = torch.tensor([e0.elapsed_time(e1) / n_e2e], dtype=torch.float64, device="cuda")
     if dist is not None:
-        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        all_reduce_(te, dist.ReduceOp.MAX)
     e2e_val = total_sites / (float(te.item()) / 1e3)
-    ok = bytes(out_h[:40 * 1000].numpy()) == bytes(out[:40 * 1000].cpu().numpy())
+    ok = bool(torch.equal(out_h, out.cpu()))
 
     if rank != 0:
         if dist is not None:
@@ -289,6 +355,10 @@ def run_gpu(args):
     nbases = int(w["off"][-1] - w["off"][0])
     hits_b = np.repeat(w["hits"], w["len"].astype(np.int64))
     keys = int(np.count_nonzero((hits_b == 1) & (w["bases"] < 4)))
+    if nreads and (int(w["pos"][0]) < w0 or int(w["pos"][-1]) + 256 > w1):   # halo reads
+        site_b = np.repeat(w["pos"].astype(np.int64), w["len"].astype(np.int64)) + (
+            np.arange(nbases) - np.repeat(w["off"][:-1].astype(np.int64), w["len"].astype(np.int64)))
+        keys = int(np.count_nonzero((hits_b == 1) & (w["bases"] < 4) & (site_b >= w0) & (site_b < w1)))
     # algorithmic HBM bytes of one k_call_tile launch: bases+quals (2 B/base), read metadata
     # (pos 8 + len 2 + off 8 + strand 1 + hits 2 = 21 B/read), reference (1 B/site), records (40 B/site)
     alg_bytes = 2 * nbases + 21 * nreads + 1 * S + 40 * S

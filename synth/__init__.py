@@ -34,7 +34,8 @@ class _Cfg(ctypes.Structure):
                 ("hom_rate", ctypes.c_double), ("multi_hit_rate", ctypes.c_double),
                 ("dup_rate", ctypes.c_double), ("base_n_rate", ctypes.c_double),
                 ("known_frac", ctypes.c_double), ("n_threads", ctypes.c_uint32),
-                ("_pad", ctypes.c_uint32)]
+                ("_pad", ctypes.c_uint32), ("region_lo", ctypes.c_uint64),
+                ("region_hi", ctypes.c_uint64)]
 
 
 @dataclass
@@ -56,6 +57,8 @@ class SynthConfig:
     base_n_rate: float = 1e-3
     known_frac: float = 0.5
     n_threads: int = field(default_factory=lambda: min(32, os.cpu_count() or 1))
+    region_lo: int = 0           # generate only genome sites [region_lo, region_hi) plus the
+    region_hi: int = 0           # reads covering them and the reference under those (0,0 = all)
 
     def scaled(self, **kw) -> "SynthConfig":
         d = asdict(self)
@@ -85,10 +88,12 @@ CONFIGS = {
 def _lib():
     lib = ctypes.CDLL(build())
     P = ctypes.c_void_p
+    lib.syn_window.restype = None
+    lib.syn_window.argtypes = [ctypes.POINTER(_Cfg), P]
     lib.syn_plan.restype = ctypes.c_uint64
-    lib.syn_plan.argtypes = [ctypes.POINTER(_Cfg), P, P, P, P, ctypes.POINTER(ctypes.c_double)]
+    lib.syn_plan.argtypes = [ctypes.POINTER(_Cfg), P, P, P, P]
     lib.syn_fill.restype = ctypes.c_uint64
-    lib.syn_fill.argtypes = [ctypes.POINTER(_Cfg), P, P, P, P, ctypes.c_double] + [P] * 7
+    lib.syn_fill.argtypes = [ctypes.POINTER(_Cfg), P, P, P, P] + [P] * 7
     lib.syn_known.restype = ctypes.c_uint64
     lib.syn_known.argtypes = [ctypes.POINTER(_Cfg), P, P, P, P, P]
     return lib
@@ -99,9 +104,10 @@ def _p(a: np.ndarray):
 
 
 def generate(cfg: SynthConfig | str, **overrides) -> dict:
-    """Generate one workload.  Returns a dict of numpy arrays:
+    """Generate one workload (or one region of it).  Returns a dict of numpy arrays:
 
-    ref (u8[n_sites], 0=A 1=C 2=T 3=G 4=N), origin, snp/alt (planted truth),
+    ref (u8, 0=A 1=C 2=T 3=G 4=N) over the generated window, origin (global coordinate of
+    ref[0]), region (global [lo, hi) the reads cover completely), snp/alt (planted truth),
     known_pos (u64[k]), known_prior10 (f64[k,10]),
     pos (u64[n]), len (u16[n]), off (u64[n+1]), bases (u8), quals (u8), strand (u8), hits (u16).
     """
@@ -111,15 +117,18 @@ def generate(cfg: SynthConfig | str, **overrides) -> dict:
         cfg = cfg.scaled(**overrides)
     c = _Cfg(cfg.seed, cfg.n_sites, cfg.origin, cfg.depth, cfg.read_len, cfg.q_hi, cfg.n_frac,
              cfg.n_lead_frac, cfg.n_blocks, cfg.het_rate, cfg.hom_rate, cfg.multi_hit_rate,
-             cfg.dup_rate, cfg.base_n_rate, cfg.known_frac, cfg.n_threads, 0)
+             cfg.dup_rate, cfg.base_n_rate, cfg.known_frac, cfg.n_threads, 0, cfg.region_lo,
+             cfg.region_hi)
     lib = _lib()
-    n = cfg.n_sites
+    win = np.zeros(2, np.uint64)
+    lib.syn_window(ctypes.byref(c), _p(win))
+    g0, g1 = int(win[0]), int(win[1])
+    n = g1 - g0
     ref = np.empty(n, np.uint8)
     snp = np.empty(n, np.uint8)
     alt = np.empty(n, np.uint8)
     elig = np.empty(n, np.uint8)
-    lam = ctypes.c_double(0)
-    nr = lib.syn_plan(ctypes.byref(c), _p(ref), _p(snp), _p(alt), _p(elig), ctypes.byref(lam))
+    nr = lib.syn_plan(ctypes.byref(c), _p(ref), _p(snp), _p(alt), _p(elig))
     if nr == (1 << 64) - 1:
         raise ValueError("bad synth config")
     L = cfg.read_len
@@ -130,16 +139,19 @@ def generate(cfg: SynthConfig | str, **overrides) -> dict:
     quals = np.empty(nr * L, np.uint8)
     strand = np.empty(nr, np.uint8)
     hits = np.empty(nr, np.uint16)
-    lib.syn_fill(ctypes.byref(c), _p(ref), _p(snp), _p(alt), _p(elig), lam.value, _p(pos), _p(ln),
+    lib.syn_fill(ctypes.byref(c), _p(ref), _p(snp), _p(alt), _p(elig), _p(pos), _p(ln),
                  _p(off), _p(bases), _p(quals), _p(strand), _p(hits))
     nk = lib.syn_known(ctypes.byref(c), _p(ref), _p(snp), _p(alt), None, None)
     kpos = np.empty(nk, np.uint64)
     kpr = np.empty((nk, 10), np.float64)
     lib.syn_known(ctypes.byref(c), _p(ref), _p(snp), _p(alt), _p(kpos), _p(kpr))
     del elig
-    return dict(config=cfg, ref=ref, origin=cfg.origin, snp=snp, alt=alt, known_pos=kpos,
+    lo = cfg.region_lo if cfg.region_hi > cfg.region_lo else 0
+    hi = min(cfg.region_hi, cfg.n_sites) if cfg.region_hi > cfg.region_lo else cfg.n_sites
+    return dict(config=cfg, ref=ref, origin=cfg.origin + g0, snp=snp, alt=alt, known_pos=kpos,
                 known_prior10=kpr, pos=pos, len=ln, off=off, bases=bases, quals=quals,
-                strand=strand, hits=hits, read_len=L)
+                strand=strand, hits=hits, read_len=L,
+                region=(cfg.origin + lo, cfg.origin + hi))
 
 
 def read_range(w: dict, lo: int, hi: int, max_read_len: int | None = None):

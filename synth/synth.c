@@ -34,6 +34,7 @@ typedef struct {
     double known_frac;      /* fraction of planted SNPs put in the known-SNP list (+ as many decoys) */
     uint32_t n_threads;
     uint32_t _pad;
+    uint64_t region_lo, region_hi; /* generate only genome sites [lo, hi) + read halo (0,0 = all) */
 } syn_config;
 
 /* ---- counter-based hashing ---------------------------------------------------------------- */
@@ -55,15 +56,16 @@ enum { T_REF = 1, T_SNP, T_SNPALT, T_SNPHAP, T_NBLK, T_FRAG, T_READ, T_QRUN, T_Q
  * ref: 0=A 1=C 2=T 3=G 4=N with human-like composition A/T 29.5%, C/G 20.5%.
  * snp: 0 none, 1 het (alt on hap 0), 2 het (alt on hap 1), 3 hom-alt.  alt: the alt base.
  * Transition:transversion 2:1.  Transition partner of b is 3-b (A<->G, C<->T). */
-static void make_reference(const syn_config* c, uint8_t* ref, uint8_t* snp, uint8_t* alt) {
+static void make_reference(const syn_config* c, uint64_t g0, uint64_t g1, uint8_t* ref,
+                           uint8_t* snp, uint8_t* alt) {
     uint64_t n = c->n_sites;
-    for (uint64_t s = 0; s < n; ++s) {
+    for (uint64_t s = g0; s < g1; ++s) {
         double u = u01(h4(c->seed, T_REF, s, 0));
-        ref[s] = u < 0.295 ? 0 : u < 0.5 ? 1 : u < 0.795 ? 2 : 3;
+        ref[s - g0] = u < 0.295 ? 0 : u < 0.5 ? 1 : u < 0.795 ? 2 : 3;
     }
-    /* N blocks */
+    /* N blocks (placed by global coordinates) */
     uint64_t lead = (uint64_t)(c->n_lead_frac * (double)n);
-    for (uint64_t s = 0; s < lead && s < n; ++s) ref[s] = 4;
+    for (uint64_t s = g0; s < lead && s < g1; ++s) ref[s - g0] = 4;
     double rest = c->n_frac - c->n_lead_frac;
     if (rest > 0 && c->n_blocks > 0 && n > lead) {
         uint64_t blk = (uint64_t)(rest * (double)n / c->n_blocks);
@@ -71,41 +73,47 @@ static void make_reference(const syn_config* c, uint8_t* ref, uint8_t* snp, uint
         for (uint32_t j = 0; j < c->n_blocks; ++j) {
             uint64_t jit = span > blk ? h4(c->seed, T_NBLK, j, 0) % (span - blk) : 0;
             uint64_t st = lead + (uint64_t)j * span + jit;
-            for (uint64_t s = st; s < st + blk && s < n; ++s) ref[s] = 4;
+            uint64_t a = st > g0 ? st : g0, b = st + blk < g1 ? st + blk : g1;
+            for (uint64_t s = a; s < b && s < n; ++s) ref[s - g0] = 4;
         }
     }
-    for (uint64_t s = 0; s < n; ++s) {
-        snp[s] = 0;
-        alt[s] = 4;
-        if (ref[s] == 4) continue;
+    for (uint64_t s = g0; s < g1; ++s) {
+        uint64_t k = s - g0;
+        snp[k] = 0;
+        alt[k] = 4;
+        if (ref[k] == 4) continue;
         double u = u01(h4(c->seed, T_SNP, s, 0));
         if (u >= c->het_rate + c->hom_rate) continue;
-        int b = ref[s];
+        int b = ref[k];
         double v = u01(h4(c->seed, T_SNPALT, s, 0));
         int a;
         if (v < 2.0 / 3.0) a = 3 - b;                  /* transition */
         else {                                         /* one of the two transversions */
-            int tv[2], k = 0;
-            for (int x = 0; x < 4; ++x) if (x != b && x != 3 - b) tv[k++] = x;
+            int tv[2], m = 0;
+            for (int x = 0; x < 4; ++x) if (x != b && x != 3 - b) tv[m++] = x;
             a = tv[v < 5.0 / 6.0 ? 0 : 1];
         }
-        alt[s] = (uint8_t)a;
-        if (u < c->het_rate) snp[s] = (h4(c->seed, T_SNPHAP, s, 0) & 1) ? 2 : 1;
-        else snp[s] = 3;
+        alt[k] = (uint8_t)a;
+        if (u < c->het_rate) snp[k] = (h4(c->seed, T_SNPHAP, s, 0) & 1) ? 2 : 1;
+        else snp[k] = 3;
     }
 }
 
 /* ---- read placement -------------------------------------------------------------------------
  * A site is read-eligible when [s, s+L) holds no N.  Fragment starts per eligible site are
- * Poisson(lambda/(1+dup)); each fragment is sequenced twice with probability dup_rate. */
+ * Poisson(depth / (L (1+dup))); each fragment is sequenced twice with probability dup_rate.
+ * Everything is keyed by the global site s, so any region of the genome can be generated on its
+ * own and agrees with the whole-genome generation (multi-GPU shards).  Arrays cover the window
+ * [g0, g1) of the genome: ref/snp/alt/elig[s - g0]. */
 typedef struct {
     const syn_config* c;
     const uint8_t* ref;
     const uint8_t* snp;
     const uint8_t* alt;
     const uint8_t* elig;
+    uint64_t g0;             /* window origin (genome index of array element 0) */
     double lam_frag;
-    uint64_t s0, s1;
+    uint64_t s0, s1;         /* read starts handled by this job (genome indices) */
     uint64_t n_reads;        /* count pass result */
     uint64_t r0;             /* fill pass: first read index */
     uint64_t* pos; uint16_t* len; uint64_t* off; uint8_t* bases; uint8_t* quals;
@@ -120,7 +128,7 @@ static inline uint32_t poisson(double lam, double u) {
 }
 
 static inline uint32_t site_frags(const job_t* j, uint64_t s) {
-    if (!j->elig[s]) return 0;
+    if (!j->elig[s - j->g0]) return 0;
     return poisson(j->lam_frag, u01(h4(j->c->seed, T_FRAG, s, 0)));
 }
 static inline uint32_t frag_copies(const job_t* j, uint64_t s, uint32_t f) {
@@ -183,7 +191,7 @@ static void* fill_job(void* arg) {
                 uint8_t* bb = j->bases + r * (uint64_t)L;
                 uint8_t* qq = j->quals + r * (uint64_t)L;
                 for (uint32_t i = 0; i < L; ++i) {
-                    uint64_t site = s + i;
+                    uint64_t site = s + i - j->g0;
                     uint32_t cy = st ? L - 1 - i : i;
                     uint8_t q = qcyc[cy];
                     int tb = j->ref[site];
@@ -207,29 +215,48 @@ static void* fill_job(void* arg) {
 }
 
 /* ---- public API -------------------------------------------------------------------------- */
-typedef struct {
-    uint8_t* ref; uint8_t* snp; uint8_t* alt;   /* n_sites each (caller-allocated) */
-    uint8_t* elig;                              /* scratch n_sites */
-    uint64_t n_reads;
-    double lam_frag;
-} syn_state;
+/* The generated window: reads starting in [start_lo, start_hi) (all reads that can touch the
+ * region [lo, hi)) and the reference [g0, g1) under them. */
+typedef struct { uint64_t lo, hi, start_lo, start_hi, g0, g1; } syn_win;
 
-static uint64_t run_jobs(const syn_config* c, syn_state* st, int fill, uint64_t* pos, uint16_t* len,
-                         uint64_t* off, uint8_t* bases, uint8_t* quals, uint8_t* strand,
-                         uint16_t* hits) {
+static syn_win window(const syn_config* c) {
+    syn_win w;
+    uint64_t n = c->n_sites, L = c->read_len;
+    w.lo = c->region_hi > c->region_lo ? c->region_lo : 0;
+    w.hi = c->region_hi > c->region_lo ? (c->region_hi < n ? c->region_hi : n) : n;
+    w.start_lo = w.lo + 1 >= L ? w.lo + 1 - L : 0;
+    w.start_hi = w.hi;
+    w.g0 = w.start_lo;
+    w.g1 = w.hi + L - 1 < n ? w.hi + L - 1 : n;
+    if (w.g1 < w.hi) w.g1 = w.hi;
+    return w;
+}
+
+/* Window bounds: out[0] = g0, out[1] = g1 (reference array length g1 - g0). */
+void syn_window(const syn_config* c, uint64_t* out) {
+    syn_win w = window(c);
+    out[0] = w.g0;
+    out[1] = w.g1;
+}
+
+static uint64_t run_jobs(const syn_config* c, const uint8_t* ref, const uint8_t* snp,
+                         const uint8_t* alt, const uint8_t* elig, int fill, uint64_t* pos,
+                         uint16_t* len, uint64_t* off, uint8_t* bases, uint8_t* quals,
+                         uint8_t* strand, uint16_t* hits) {
+    syn_win w = window(c);
     uint32_t nt = c->n_threads ? c->n_threads : 1;
     if (nt > 256) nt = 256;
-    uint64_t n = c->n_sites;
+    uint64_t n = w.start_hi - w.start_lo;
     uint64_t chunk = (n + nt - 1) / nt;
     job_t jobs[256];
     pthread_t th[256];
     for (uint32_t t = 0; t < nt; ++t) {
         job_t* j = &jobs[t];
         memset(j, 0, sizeof *j);
-        j->c = c; j->ref = st->ref; j->snp = st->snp; j->alt = st->alt; j->elig = st->elig;
-        j->lam_frag = st->lam_frag;
-        j->s0 = t * chunk < n ? t * chunk : n;
-        j->s1 = (t + 1) * chunk < n ? (t + 1) * chunk : n;
+        j->c = c; j->ref = ref; j->snp = snp; j->alt = alt; j->elig = elig; j->g0 = w.g0;
+        j->lam_frag = c->depth / ((double)c->read_len * (1.0 + c->dup_rate));
+        j->s0 = w.start_lo + (t * chunk < n ? t * chunk : n);
+        j->s1 = w.start_lo + ((t + 1) * chunk < n ? (t + 1) * chunk : n);
     }
     for (uint32_t t = 0; t < nt; ++t) pthread_create(&th[t], NULL, count_job, &jobs[t]);
     for (uint32_t t = 0; t < nt; ++t) pthread_join(th[t], NULL);
@@ -247,54 +274,50 @@ static uint64_t run_jobs(const syn_config* c, syn_state* st, int fill, uint64_t*
     return total;
 }
 
-/* Phase 1: reference, SNPs, eligibility; returns the number of reads phase 2 will produce. */
-uint64_t syn_plan(const syn_config* c, uint8_t* ref, uint8_t* snp, uint8_t* alt, uint8_t* elig,
-                  double* lam_out) {
+/* Phase 1: reference window, SNPs, eligibility (arrays of g1 - g0); returns the read count. */
+uint64_t syn_plan(const syn_config* c, uint8_t* ref, uint8_t* snp, uint8_t* alt, uint8_t* elig) {
     if (c->read_len == 0 || c->read_len > 256 || c->n_sites == 0) return (uint64_t)-1;
-    make_reference(c, ref, snp, alt);
-    uint64_t n = c->n_sites, L = c->read_len, nonN = 0, nel = 0, run = 0;
-    for (uint64_t s = 0; s < n; ++s) nonN += ref[s] != 4;
-    /* elig[s] = 1 iff ref[s..s+L) has no N: scan right-to-left counting the non-N run */
-    for (uint64_t k = n; k-- > 0;) {
+    syn_win w = window(c);
+    make_reference(c, w.g0, w.g1, ref, snp, alt);
+    uint64_t L = c->read_len, run = 0, m = w.g1 - w.g0;
+    /* elig[s] = 1 iff ref[s..s+L) has no N (and lies in the genome): right-to-left non-N run */
+    for (uint64_t k = m; k-- > 0;) {
         run = ref[k] == 4 ? 0 : run + 1;
         elig[k] = run >= L;
-        nel += elig[k];
     }
-    double lam = nel ? c->depth * (double)nonN / ((double)L * (double)nel) : 0.0;
-    syn_state st = {ref, snp, alt, elig, 0, lam / (1.0 + c->dup_rate)};
-    *lam_out = st.lam_frag;
-    return run_jobs(c, &st, 0, 0, 0, 0, 0, 0, 0, 0);
+    return run_jobs(c, ref, snp, alt, elig, 0, 0, 0, 0, 0, 0, 0, 0);
 }
 
 /* Phase 2: fill reads (arrays sized by syn_plan's count; off has n_reads+1 entries). */
 uint64_t syn_fill(const syn_config* c, uint8_t* ref, uint8_t* snp, uint8_t* alt, uint8_t* elig,
-                  double lam_frag, uint64_t* pos, uint16_t* len, uint64_t* off, uint8_t* bases,
-                  uint8_t* quals, uint8_t* strand, uint16_t* hits) {
-    syn_state st = {ref, snp, alt, elig, 0, lam_frag};
-    return run_jobs(c, &st, 1, pos, len, off, bases, quals, strand, hits);
+                  uint64_t* pos, uint16_t* len, uint64_t* off, uint8_t* bases, uint8_t* quals,
+                  uint8_t* strand, uint16_t* hits) {
+    return run_jobs(c, ref, snp, alt, elig, 1, pos, len, off, bases, quals, strand, hits);
 }
 
-/* Known-SNP list: known_frac of the planted SNPs plus decoys at the same rate over non-SNP
- * non-N sites.  Priors (linear, > 0) per genotype n (order AA AC AT AG CC CT CG TT TG GG):
- * ref-hom 0.85, ref/alt het 0.1, alt-hom 0.05, any other genotype 1e-4.
+/* Known-SNP list over the reference window: known_frac of the planted SNPs plus decoys at the
+ * same rate over non-SNP non-N sites.  Priors (linear, > 0) per genotype n (order AA AC AT AG
+ * CC CT CG TT TG GG): ref-hom 0.85, ref/alt het 0.1, alt-hom 0.05, any other genotype 1e-4.
  * Pass known_pos == NULL to count. */
 uint64_t syn_known(const syn_config* c, const uint8_t* ref, const uint8_t* snp, const uint8_t* alt,
                    uint64_t* known_pos, double* prior10) {
     static const int A1[10] = {0, 0, 0, 0, 1, 1, 1, 2, 2, 3};
     static const int A2[10] = {0, 1, 2, 3, 1, 2, 3, 2, 3, 3};
+    syn_win w = window(c);
     double decoy_rate = c->known_frac * (c->het_rate + c->hom_rate);
     uint64_t k = 0;
-    for (uint64_t s = 0; s < c->n_sites; ++s) {
-        if (ref[s] == 4) continue;
+    for (uint64_t s = w.g0; s < w.g1; ++s) {
+        uint64_t i = s - w.g0;
+        if (ref[i] == 4) continue;
         int a = -1;
-        if (snp[s]) {
-            if (u01(h4(c->seed, T_KNOWN, s, 0)) < c->known_frac) a = alt[s];
+        if (snp[i]) {
+            if (u01(h4(c->seed, T_KNOWN, s, 0)) < c->known_frac) a = alt[i];
         } else if (u01(h4(c->seed, T_DECOY, s, 0)) < decoy_rate) {
-            a = (ref[s] + 1 + (int)(h4(c->seed, T_DECOYALT, s, 0) % 3)) & 3;
+            a = (ref[i] + 1 + (int)(h4(c->seed, T_DECOYALT, s, 0) % 3)) & 3;
         }
         if (a < 0) continue;
         if (known_pos) {
-            int r = ref[s];
+            int r = ref[i];
             known_pos[k] = c->origin + s;
             for (int n = 0; n < 10; ++n) {
                 int x = A1[n], y = A2[n];
