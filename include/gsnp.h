@@ -153,7 +153,8 @@ gsnp_status gsnp_debug_window(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w
 
 /* Copy the context's tables to host buffers (any may be NULL):
  *   counts u64[64*256*16]; p_matrix f64[64*256*16] (index q<<12|coord<<4|allele<<2|base);
- *   T f64[64*L*4*10] (index ((q*L+coord)*4+base)*10+n, Alg. 3); adj u8[64*adj_pcr*adj_g].
+ *   T f64[64*L*4*10] (index ((q*L+coord)*4+base)*10+n, Alg. 3; rows q = 1..q_max are built —
+ *   adjust() never leaves that range — the others are zero); adj u8[64*adj_pcr*adj_g].
  * dims (may be NULL) receives {L, adj_pcr, adj_g}. */
 gsnp_status gsnp_get_tables(gsnp_ctx* ctx, uint64_t* counts, double* p_matrix, double* T,
                             uint8_t* adj, uint32_t* dims);

@@ -65,7 +65,9 @@ struct gsnp_ctx {
     DevBuf<double> LP;
     std::vector<uint64_t> h_counts;
     std::vector<double> h_p;   // [64][256][4][4]
-    std::vector<double> h_T;   // [64][L][4][10]
+    double* h_T = nullptr;     // [64][L][4][10], pinned host copy of the score table
+    size_t h_T_n = 0;
+    uint64_t* h_cnt_pinned = nullptr;   // staging for device-resident counts
     DevBuf<double> T;
     bool calibrated = false;
     // scratch
@@ -200,72 +202,57 @@ gsnp_status build_adj(gsnp_ctx* ctx) {
     return GSNP_OK;
 }
 
-// R1 estimator (host): p[q][c][t][o], index q<<12 | c<<4 | t<<2 | o.
-void estimate_p(const gsnp_params& prm, const uint64_t* C, std::vector<double>& p) {
+// R1 estimator (host) for one quality q: p[q][c][t][o], index q<<12 | c<<4 | t<<2 | o.
+void estimate_p_q(const gsnp_params& prm, const uint64_t* C, double* p, int q) {
     const int L = (int)prm.max_read_len;
     const double tau = (double)prm.calib_min_count;
-    p.assign((size_t)64 * 256 * 16, 0.0);
-    for (int q = 0; q < 64; ++q) {
-        double tot = 0, mm = 0;
+    double tot = 0, mm = 0;
+    for (int c = 0; c < L; ++c)
+        for (int t = 0; t < 4; ++t)
+            for (int o = 0; o < 4; ++o) {
+                double v = (double)C[q << 12 | c << 4 | t << 2 | o];
+                tot += v;
+                if (t != o) mm += v;
+            }
+    for (int t = 0; t < 4; ++t) {
+        double npool[4] = {0, 0, 0, 0}, Npool = 0;
         for (int c = 0; c < L; ++c)
-            for (int t = 0; t < 4; ++t)
-                for (int o = 0; o < 4; ++o) {
-                    double v = (double)C[q << 12 | c << 4 | t << 2 | o];
-                    tot += v;
-                    if (t != o) mm += v;
+            for (int o = 0; o < 4; ++o) {
+                double v = (double)C[q << 12 | c << 4 | t << 2 | o];
+                npool[o] += v;
+                Npool += v;
+            }
+        for (int c = 0; c < L; ++c) {
+            double Nct = 0;
+            for (int o = 0; o < 4; ++o) Nct += (double)C[q << 12 | c << 4 | t << 2 | o];
+            for (int o = 0; o < 4; ++o) {
+                double n = (double)C[q << 12 | c << 4 | t << 2 | o], v;
+                if (n > tau) v = n / Nct;
+                else if (npool[o] > tau) v = npool[o] / Npool;
+                else if (mm > 0 && mm < tot) v = (o == t) ? (tot - mm) / tot : mm / (3.0 * tot);
+                else {
+                    double e = pow(10.0, -(double)q / 10.0);
+                    if (e > 0.75) e = 0.75;
+                    v = (o == t) ? 1.0 - e : e / 3.0;
                 }
-        for (int t = 0; t < 4; ++t) {
-            double npool[4] = {0, 0, 0, 0}, Npool = 0;
-            for (int c = 0; c < L; ++c)
-                for (int o = 0; o < 4; ++o) {
-                    double v = (double)C[q << 12 | c << 4 | t << 2 | o];
-                    npool[o] += v;
-                    Npool += v;
-                }
-            for (int c = 0; c < L; ++c) {
-                double Nct = 0;
-                for (int o = 0; o < 4; ++o) Nct += (double)C[q << 12 | c << 4 | t << 2 | o];
-                for (int o = 0; o < 4; ++o) {
-                    double n = (double)C[q << 12 | c << 4 | t << 2 | o], v;
-                    if (n > tau) v = n / Nct;
-                    else if (npool[o] > tau) v = npool[o] / Npool;
-                    else if (mm > 0 && mm < tot) v = (o == t) ? (tot - mm) / tot : mm / (3.0 * tot);
-                    else {
-                        double e = pow(10.0, -(double)q / 10.0);
-                        if (e > 0.75) e = 0.75;
-                        v = (o == t) ? 1.0 - e : e / 3.0;
-                    }
-                    p[q << 12 | c << 4 | t << 2 | o] = v;
-                }
+                p[q << 12 | c << 4 | t << 2 | o] = v;
             }
         }
     }
 }
 
-// Alg. 3 score table: T[qa][c][b][n] = log10(0.5 p[qa][c][a1][b] + 0.5 p[qa][c][a2][b]),
-// the value Alg. 2 returns; built once on the CPU (§IV-G).  Rows qa = 1..63 (adjust >= 1).
-void build_T(int L, const std::vector<double>& p, std::vector<double>& T) {
+// Alg. 3 score-table rows of quality qa: T[qa][c][b][n] = log10(0.5 p[qa][c][a1][b] +
+// 0.5 p[qa][c][a2][b]), the value Alg. 2 returns, built on the CPU (§IV-G).
+void build_T_q(int L, const double* p, double* T, int qa) {
     static const int A1[10] = {0, 0, 0, 0, 1, 1, 1, 2, 2, 3};
     static const int A2[10] = {0, 1, 2, 3, 1, 2, 3, 2, 3, 3};
-    T.assign((size_t)64 * L * 4 * 10, 0.0);
-    auto work = [&](int q0, int q1) {
-        for (int qa = q0; qa < q1; ++qa)
-            for (int c = 0; c < L; ++c)
-                for (int b = 0; b < 4; ++b)
-                    for (int n = 0; n < 10; ++n) {
-                        int p1 = qa << 12 | c << 4 | A1[n] << 2 | b;
-                        int p2 = qa << 12 | c << 4 | A2[n] << 2 | b;
-                        T[(((size_t)qa * L + c) * 4 + b) * 10 + n] = log10(0.5 * p[p1] + 0.5 * p[p2]);
-                    }
-    };
-    unsigned nt = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
-    std::vector<std::thread> th;
-    int per = (64 + (int)nt - 1) / (int)nt;
-    for (unsigned i = 0; i < nt; ++i) {
-        int q0 = (int)i * per, q1 = std::min(64, q0 + per);
-        if (q0 < q1) th.emplace_back(work, q0, q1);
-    }
-    for (auto& t : th) t.join();
+    for (int c = 0; c < L; ++c)
+        for (int b = 0; b < 4; ++b)
+            for (int n = 0; n < 10; ++n) {
+                int p1 = qa << 12 | c << 4 | A1[n] << 2 | b;
+                int p2 = qa << 12 | c << 4 | A2[n] << 2 | b;
+                T[(((size_t)qa * L + c) * 4 + b) * 10 + n] = log10(0.5 * p[p1] + 0.5 * p[p2]);
+            }
 }
 
 gsnp_status check_params(gsnp_ctx* ctx, const gsnp_params* p) {
@@ -441,18 +428,22 @@ gsnp_status count_impl(gsnp_ctx* ctx, const gsnp_reads* reads) {
         A.n_sites = ctx->n_sites;
         A.L = (int)ctx->prm.max_read_len;
         A.q_max = (int)ctx->prm.q_max;
-        A.CT = (A.L + 31) / 32 * 32;
+        A.CT = (A.L + 1 + 31) / 32 * 32;              // one spare thread issues the copies
         A.SB = 12 * 1024;                              // bases (and quals) per stage
+        A.RB = 4 * 1024 + 32;                          // reference window per stage
         A.CB = std::max(1, std::min<int>(CAL_MAXB, (int)(A.SB - 32) / A.L));
         A.C = ctx->d_counts.p;
         A.err = ctx->d_err.p;
-        const size_t smem = align16((size_t)(A.q_max + 1) * 4 * A.CT * 2) + 4 * (size_t)A.SB;
-        const int per_sm = (int)std::max<size_t>(1, std::min<size_t>(4, (227 * 1024) / (smem + 10 * 1024)));
+        const size_t hist = (size_t)(A.q_max + 1) * 4 * A.L * 2, stages = 2 * (2 * (size_t)A.SB + A.RB);
+        A.G = CAL_GMAX;                                // as many histogram copies as fit
+        while (A.G > 1 && (align16(A.G * hist) + stages > 200 * 1024 || A.G * A.CT > 1024)) A.G >>= 1;
+        const size_t smem = align16(A.G * hist) + stages;
+        const int per_sm = 1;
         unsigned grid = (unsigned)std::min<uint64_t>((uint64_t)g_num_sms * per_sm, (d.n + A.CB - 1) / A.CB);
         grid = std::max(grid, 1u);
         CK(cudaFuncSetAttribute(k_calib_count, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         ctx->begin();
-        k_calib_count<<<grid, A.CT, smem, s>>>(A);
+        k_calib_count<<<grid, A.CT * A.G, smem, s>>>(A);
         ctx->end(GSNP_STAGE_CALIB);
         ctx->launches++;
         CK(cudaGetLastError());
@@ -462,12 +453,36 @@ gsnp_status count_impl(gsnp_ctx* ctx, const gsnp_reads* reads) {
 
 gsnp_status finalize_impl(gsnp_ctx* ctx, const uint64_t* counts_host) {
     auto t0 = std::chrono::steady_clock::now();
+    const int L = (int)ctx->prm.max_read_len;
+    const int qmax = (int)ctx->prm.q_max;
     ctx->h_counts.assign(counts_host, counts_host + 64 * 256 * 16);
-    estimate_p(ctx->prm, ctx->h_counts.data(), ctx->h_p);
-    build_T((int)ctx->prm.max_read_len, ctx->h_p, ctx->h_T);
-    CK(ctx->T.ensure(ctx->h_T.size()));
-    CK(cudaMemcpyAsync(ctx->T.p, ctx->h_T.data(), ctx->h_T.size() * 8, cudaMemcpyHostToDevice,
-                       ctx->stream));
+    ctx->h_p.assign((size_t)64 * 256 * 16, 0.0);
+    const size_t tn = (size_t)64 * L * 4 * 10;
+    if (!ctx->h_T || ctx->h_T_n != tn) {
+        if (ctx->h_T) cudaFreeHost(ctx->h_T);
+        ctx->h_T = nullptr;
+        CK(cudaMallocHost(&ctx->h_T, tn * sizeof(double)));
+        ctx->h_T_n = tn;
+        memset(ctx->h_T, 0, tn * sizeof(double));     // rows 0 and > q_max are never indexed
+    }
+    // p for every quality; T rows only for q_adj in [1, q_max] (adjust never leaves that range)
+    const uint64_t* C = ctx->h_counts.data();
+    double* p = ctx->h_p.data();
+    double* T = ctx->h_T;
+    const gsnp_params prm = ctx->prm;
+    auto work = [&](int tid, int nt) {
+        for (int q = tid; q < 64; q += nt) {
+            estimate_p_q(prm, C, p, q);
+            if (q >= 1 && q <= qmax) build_T_q(L, p, T, q);
+        }
+    };
+    const int nt = (int)std::max(1u, std::min(8u, std::thread::hardware_concurrency()));
+    std::vector<std::thread> th;
+    for (int i = 1; i < nt; ++i) th.emplace_back(work, i, nt);
+    work(0, nt);
+    for (auto& t : th) t.join();
+    CK(ctx->T.ensure(tn));
+    CK(cudaMemcpyAsync(ctx->T.p, ctx->h_T, tn * 8, cudaMemcpyHostToDevice, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
     ctx->calibrated = true;
     if (ctx->timing()) {
@@ -557,7 +572,8 @@ gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
     if ((st = build_adj(ctx))) return bail(st);
     gsnp_ctx* c = ctx;
 #define CKC(x) do { if ((x) != cudaSuccess) { cudaGetLastError(); return bail(fail(c, GSNP_E_CUDA, "%s", #x)); } } while (0)
-    CKC(ctx->ref.ensure(ref->n_sites));
+    CKC(ctx->ref.ensure(ref->n_sites + 64));       // padded: 16-byte TMA windows may overrun
+    CKC(cudaMemset(ctx->ref.p + ref->n_sites, 4, 64));
     CKC(cudaMemcpy(ctx->ref.p, code.data(), ref->n_sites, cudaMemcpyHostToDevice));
     CKC(ctx->known_pos.ensure(std::max<uint64_t>(nk, 1)));
     if (nk) CKC(cudaMemcpy(ctx->known_pos.p, ctx->h_known_pos.data(), nk * 8, cudaMemcpyHostToDevice));
@@ -588,14 +604,14 @@ gsnp_status gsnp_calibrate_count(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_
 gsnp_status gsnp_calibrate_finalize(gsnp_ctx* ctx, const uint64_t* counts) {
     if (!ctx || !counts) return GSNP_E_INVAL;
     if (cudaSetDevice(ctx->prm.device) != cudaSuccess) return fail(ctx, GSNP_E_CUDA, "set device");
-    std::vector<uint64_t> h(64 * 256 * 16);
     if (is_device_ptr(counts)) {
-        CK(cudaMemcpyAsync(h.data(), counts, h.size() * 8, cudaMemcpyDeviceToHost, ctx->stream));
+        if (!ctx->h_cnt_pinned) CK(cudaMallocHost(&ctx->h_cnt_pinned, 64 * 256 * 16 * 8));
+        CK(cudaMemcpyAsync(ctx->h_cnt_pinned, counts, 64 * 256 * 16 * 8, cudaMemcpyDeviceToHost,
+                           ctx->stream));
         CK(cudaStreamSynchronize(ctx->stream));
-    } else {
-        memcpy(h.data(), counts, h.size() * 8);
+        return finalize_impl(ctx, ctx->h_cnt_pinned);
     }
-    return finalize_impl(ctx, h.data());
+    return finalize_impl(ctx, counts);
 }
 
 gsnp_status gsnp_calibrate(gsnp_ctx* ctx, const gsnp_reads* reads) {
@@ -717,7 +733,7 @@ gsnp_status gsnp_get_tables(gsnp_ctx* ctx, uint64_t* counts, double* p_matrix, d
     if ((counts || p_matrix || T) && !ctx->calibrated) return fail(ctx, GSNP_E_STATE, "not calibrated");
     if (counts) memcpy(counts, ctx->h_counts.data(), ctx->h_counts.size() * 8);
     if (p_matrix) memcpy(p_matrix, ctx->h_p.data(), ctx->h_p.size() * 8);
-    if (T) memcpy(T, ctx->h_T.data(), ctx->h_T.size() * 8);
+    if (T) memcpy(T, ctx->h_T, ctx->h_T_n * 8);
     return GSNP_OK;
 }
 
@@ -763,6 +779,8 @@ void gsnp_destroy(gsnp_ctx* ctx) {
     ctx->r_bases.release(); ctx->r_quals.release(); ctx->r_strand.release();
     ctx->dbg_u32a.release(); ctx->dbg_u32b.release(); ctx->dbg_u32c.release();
     ctx->dbg_u32d.release(); ctx->dbg_u32e.release(); ctx->dbg_f64a.release(); ctx->dbg_f64b.release();
+    if (ctx->h_T) cudaFreeHost(ctx->h_T);
+    if (ctx->h_cnt_pinned) cudaFreeHost(ctx->h_cnt_pinned);
     for (auto& p : ctx->pending) { cudaEventDestroy(p.a); cudaEventDestroy(p.b); }
     for (auto e : ctx->ev_pool) cudaEventDestroy(e);
     delete ctx;

@@ -183,126 +183,171 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
 // counts before any cell can overflow); mismatches go straight to global u64 REDs.
 struct CalibArgs {
     DevReads R;
-    const uint8_t* ref;               // code | known << 3, indexed by site - origin
+    const uint8_t* ref;               // code | known << 3, indexed by site - origin (16 B padded)
     uint64_t origin, n_sites;
     int L, q_max;
-    int CT;                           // threads per CTA = L rounded up to a multiple of 32
+    int CT;                           // threads per group (>= L; thread CT-1 issues the copies)
+    int G;                            // groups per CTA (1, 2 or 4), one histogram copy each
     int CB;                           // reads per batch
     uint32_t SB;                      // bytes per stage buffer (bases; quals the same)
+    uint32_t RB;                      // bytes per reference-window buffer
     unsigned long long* C;            // [64][256][4][4]
     int* err;
 };
 
 constexpr int CAL_MAXB = 512;         // max reads per batch (metadata arrays)
 
-__device__ __forceinline__ void calib_flush(const CalibArgs& A, uint16_t* h, int nbins) {
-    const int c = threadIdx.x;
-    if (c >= A.L) return;
+constexpr int CAL_GMAX = 4;           // thread groups per CTA (A.G), one histogram copy each
+
+// Add the G histogram copies of cycle c into the global counts and clear them (threads of
+// group 0; the caller synchronises before and after).
+__device__ __forceinline__ void calib_flush(const CalibArgs& A, uint16_t* h, int nbins, int c) {
+    if (c >= A.L || threadIdx.x >= (unsigned)A.CT) return;
+    const size_t copy = (size_t)nbins * A.L;
     for (int k = 0; k < nbins; ++k) {                 // k = q*4 + t
-        uint16_t* cell = h + (size_t)k * A.CT + c;
-        const uint32_t v = *cell;
+        uint32_t v = 0;
+        for (int g = 0; g < A.G; ++g) {
+            uint16_t* cell = h + g * copy + (size_t)k * A.L + c;
+            v += *cell;
+            *cell = 0;
+        }
         if (v) {
             const uint32_t q = k >> 2, t = k & 3;
             atomicAdd(&A.C[q << 12 | (uint32_t)c << 4 | t << 2 | t], (unsigned long long)v);
-            *cell = 0;
         }
     }
 }
 
-__global__ void __launch_bounds__(256) k_calib_count(CalibArgs A) {
+__global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
     extern __shared__ __align__(16) unsigned char smem[];
-    __shared__ uint32_t m_rs[CAL_MAXB];               // read start - origin
-    __shared__ uint32_t m_off[CAL_MAXB];              // byte offset within the stage buffer
-    __shared__ uint32_t m_lhs[CAL_MAXB];              // len | strand << 16 | counted << 17
+    __shared__ uint64_t m_desc[2][CAL_MAXB];          // counted reads: rs | stage offset << 32
+    __shared__ uint16_t m_ls[2][CAL_MAXB];            // len | strand << 9
+    __shared__ uint32_t m_n[2];                       // counted reads per stage
     __shared__ __align__(8) uint64_t bar[2];
     __shared__ uint64_t st_base[2];                   // global byte index of each stage's start
-    __shared__ int st_direct[2];                      // batch too wide for the stage: read global
+    __shared__ uint32_t st_rs[2];                     // reference index of each ref window's start
+    __shared__ int st_direct[2];                      // too wide for the buffers: read global
     const int nbins = (A.q_max + 1) * 4;
-    uint16_t* h = reinterpret_cast<uint16_t*>(smem);
-    unsigned char* stage = smem + align16((size_t)nbins * A.CT * 2);
-    const int c = threadIdx.x;
-    for (int i = c; i < nbins * A.CT; i += blockDim.x) h[i] = 0;
+    const int tid = threadIdx.x;
+    const int grp = tid / A.CT, c = tid % A.CT;       // group grp counts reads grp, grp+G, ...
+    const int L = A.L;
+    uint16_t* h0 = reinterpret_cast<uint16_t*>(smem);
+    uint16_t* h = h0 + (size_t)grp * nbins * L;       // this group's histogram copy
+    unsigned char* stage = smem + align16((size_t)A.G * nbins * L * 2);
+    const size_t stage_bytes = 2 * (size_t)A.SB + A.RB;
+    for (int i = tid; i < A.G * nbins * L; i += blockDim.x) h0[i] = 0;
     const uint64_t per = (A.R.n + gridDim.x - 1) / gridDim.x;
     const uint64_t ra = min(A.R.n, (uint64_t)blockIdx.x * per), rb = min(A.R.n, ra + per);
     const uint64_t nbatch = (rb - ra + A.CB - 1) / A.CB;
-    if (c == 0) { mbar_init(&bar[0], 1); mbar_init(&bar[1], 1); }
+    const int issuer = A.CT - 1;                      // beyond the last cycle when CT > L
+    if (tid == 0) { mbar_init(&bar[0], 1); mbar_init(&bar[1], 1); }
     __syncthreads();
-    // issue the bulk copies of batch k into stage k & 1 (thread 0)
+    // thread `issuer`: bulk copies of batch k's bases, quals and reference window into stage k&1
     auto issue = [&](uint64_t k) {
         const uint64_t b0 = ra + k * A.CB, b1 = min(rb, b0 + A.CB);
         const uint64_t o0 = A.R.off[b0] - A.R.off0, o1 = A.R.off[b1] - A.R.off0;
         const uint64_t a0 = o0 & ~15ull, a1 = (o1 + 15) & ~15ull;
+        const uint64_t p0 = A.R.pos[b0], p1 = A.R.pos[b1 - 1];
         const int sidx = (int)(k & 1);
         st_base[sidx] = a0;
-        if (a1 - a0 > A.SB) { st_direct[sidx] = 1; return; }
-        st_direct[sidx] = 0;
-        unsigned char* sb = stage + (size_t)sidx * 2 * A.SB;
-        const uint32_t bytes = (uint32_t)(a1 - a0);
+        const uint64_t r0 = p0 >= A.origin ? ((p0 - A.origin) & ~15ull) : 0;
+        const uint64_t r1 = ((p1 + L - A.origin) + 15) & ~15ull;
+        st_rs[sidx] = (uint32_t)r0;
+        const bool fits = a1 - a0 <= A.SB && p0 >= A.origin && p1 + L <= A.origin + A.n_sites &&
+                          r1 - r0 <= A.RB;
+        st_direct[sidx] = fits ? 0 : 1;
+        if (!fits) return;
+        unsigned char* sb = stage + (size_t)sidx * stage_bytes;
+        const uint32_t bytes = (uint32_t)(a1 - a0), rbytes = (uint32_t)(r1 - r0);
         fence_proxy_async_smem();
-        mbar_arrive_expect_tx(&bar[sidx], 2 * bytes);
+        mbar_arrive_expect_tx(&bar[sidx], 2 * bytes + rbytes);
         tma_g2s(sb, A.R.bases + a0, bytes, &bar[sidx]);
         tma_g2s(sb + A.SB, A.R.quals + a0, bytes, &bar[sidx]);
+        tma_g2s(sb + 2 * A.SB, A.ref + r0, rbytes, &bar[sidx]);
     };
-    if (c == 0 && nbatch > 0) issue(0);
-    int err = 0;
-    uint32_t since_flush = 0;
-    // count cycle c of reads [0, nr) of the current batch from byte arrays sb/sq
-    auto count = [&](const unsigned char* __restrict__ sb, const unsigned char* __restrict__ sq,
-                     uint32_t nr) {
-#pragma unroll 4
-        for (uint32_t j = 0; j < nr; ++j) {
-            const uint32_t lhs = m_lhs[j], l = lhs & 0xFFFFu, st = (lhs >> 16) & 1u;
-            const bool take = (lhs >> 17) && (uint32_t)c < l;       // counted read, cycle exists
-            const uint32_t i = st ? l - 1 - c : c;                 // read position of cycle c
-            const uint32_t bi = m_off[j] + (take ? i : 0u);
-            const uint32_t o = sb[bi], q = sq[bi];
-            const uint32_t rt = A.ref[take ? m_rs[j] + i : 0u];     // code | known << 3
-            const uint32_t t = rt & 7u;
-            err |= (take && o > 4) ? ERR_RANGE : 0;
-            err |= (take && q > (uint32_t)A.q_max) ? ERR_QUAL : 0;
-            const bool cnt = take && t < 4 && o < 4 && q <= (uint32_t)A.q_max && !(rt & 8u);
-            if (cnt && t == o) h[(q * 4 + t) * A.CT + c] += 1;
-            else if (cnt) atomicAdd(&A.C[q << 12 | (uint32_t)c << 4 | t << 2 | o], 1ull);
-        }
-    };
-    for (uint64_t k = 0; k < nbatch; ++k) {
+    // all threads: compact the counted reads of batch k (unique, inside the reference)
+    auto stage_meta = [&](uint64_t k) {
         const int sidx = (int)(k & 1);
         const uint64_t b0 = ra + k * A.CB, b1 = min(rb, b0 + A.CB);
-        const uint32_t nr = (uint32_t)(b1 - b0);
-        __syncthreads();                               // stage (k+1)&1 and metadata free
-        if (c == 0 && k + 1 < nbatch) issue(k + 1);
-        for (uint32_t j = c; j < nr; j += blockDim.x) {
-            const uint64_t r = b0 + j;
-            const uint64_t p = A.R.pos[r];
-            const uint32_t l = A.R.len[r];
-            // unique reads inside the reference are counted (others are flagged by validate)
-            const bool in = p >= A.origin && p + l <= A.origin + A.n_sites;
-            m_rs[j] = in ? (uint32_t)(p - A.origin) : 0u;
-            m_off[j] = (uint32_t)(A.R.off[r] - A.R.off0 - st_base[sidx]);
-            m_lhs[j] = l | (uint32_t)A.R.strand[r] << 16 | ((A.R.hits[r] == 1 && in) ? 1u << 17 : 0u);
-        }
-        if (since_flush + nr > 65535u) {               // u16 cells could overflow: flush
-            __syncthreads();
-            calib_flush(A, h, nbins);
-            since_flush = 0;
-        }
-        since_flush += nr;
-        __syncthreads();
-        if (c < A.L) {
-            if (st_direct[sidx]) {
-                count(A.R.bases + st_base[sidx], A.R.quals + st_base[sidx], nr);
-            } else {
-                mbar_wait(&bar[sidx], (uint32_t)((k >> 1) & 1));
-                const unsigned char* sb = stage + (size_t)sidx * 2 * A.SB;
-                count(sb, sb + A.SB, nr);
+        for (uint64_t r0 = b0; r0 < b1; r0 += blockDim.x) {
+            const uint64_t r = r0 + tid;
+            bool keep = false;
+            uint64_t d = 0;
+            uint16_t ls = 0;
+            if (r < b1 && A.R.hits[r] == 1) {
+                const uint64_t p = A.R.pos[r];
+                const uint32_t l = A.R.len[r];
+                keep = p >= A.origin && p + l <= A.origin + A.n_sites && l >= 1 && l <= (uint32_t)L;
+                d = (uint64_t)(uint32_t)(p - A.origin) |
+                    (uint64_t)(uint32_t)(A.R.off[r] - A.R.off0 - st_base[sidx]) << 32;
+                ls = (uint16_t)(l | (uint32_t)A.R.strand[r] << 9);
             }
-        } else if (!st_direct[sidx]) {
-            mbar_wait(&bar[sidx], (uint32_t)((k >> 1) & 1));
+            const uint32_t bal = __ballot_sync(FULL, keep);
+            uint32_t base = 0;
+            if ((tid & 31) == 0 && bal) base = atomicAdd(&m_n[sidx], (uint32_t)__popc(bal));
+            base = __shfl_sync(FULL, base, 0);
+            if (keep) {
+                const uint32_t j = base + __popc(bal & lanemask_lt());
+                m_desc[sidx][j] = d;
+                m_ls[sidx][j] = ls;
+            }
         }
+    };
+    if (tid == 0) { m_n[0] = 0; m_n[1] = 0; }
+    __syncthreads();
+    if (tid == issuer && nbatch > 0) issue(0);
+    __syncthreads();
+    if (nbatch > 0) stage_meta(0);
+    int err = 0;
+    uint32_t since_flush = 0;
+    uint32_t phase0 = 0, phase1 = 0;                   // mbarrier parity per stage (TMA'd uses)
+    for (uint64_t k = 0; k < nbatch; ++k) {
+        const int sidx = (int)(k & 1);
+        __syncthreads();                               // metadata of stage k complete
+        if (tid == issuer && k + 1 < nbatch) issue(k + 1);
+        const uint32_t nr = m_n[sidx];
+        const uint32_t per_grp = (nr + A.G - 1) / A.G;
+        if (since_flush + per_grp > 65535u) {          // u16 cells could overflow: flush
+            calib_flush(A, h0, nbins, c + grp * A.CT);
+            since_flush = 0;
+            __syncthreads();
+        }
+        since_flush += per_grp;
+        const bool direct = st_direct[sidx] != 0;
+        if (!direct) {
+            mbar_wait(&bar[sidx], sidx ? phase1 : phase0);
+            if (sidx) phase1 ^= 1u; else phase0 ^= 1u;
+        }
+        if (c < L) {
+            const unsigned char* sb = stage + (size_t)sidx * stage_bytes;
+            const unsigned char* bq = direct ? A.R.bases + st_base[sidx] : sb;
+            const unsigned char* qq = direct ? A.R.quals + st_base[sidx] : sb + A.SB;
+            const unsigned char* rr = direct ? A.ref : sb + 2 * A.SB - st_rs[sidx];
+            const uint64_t* md = m_desc[sidx];
+            const uint16_t* ml = m_ls[sidx];
+#pragma unroll 4
+            for (uint32_t j = grp; j < nr; j += A.G) {
+                const uint64_t d = md[j];
+                const uint32_t ls = ml[j], l = ls & 511u;
+                if ((uint32_t)c >= l) continue;
+                const uint32_t i = (ls >> 9) ? l - 1 - c : (uint32_t)c;    // read position of cycle c
+                const uint32_t bi = (uint32_t)(d >> 32) + i;
+                const uint32_t o = bq[bi], q = qq[bi];
+                const uint32_t rt = rr[(uint32_t)d + i];                    // code | known << 3
+                err |= (o > 4 ? ERR_RANGE : 0) | (q > (uint32_t)A.q_max ? ERR_QUAL : 0);
+                if (rt >= 4 || o >= 4 || q > (uint32_t)A.q_max) continue;   // N, known SNP, bad
+                if (rt == o) h[(q * 4 + rt) * L + c] += 1;
+                else atomicAdd(&A.C[q << 12 | (uint32_t)c << 4 | rt << 2 | o], 1ull);
+            }
+        }
+        __syncthreads();                               // stage k fully consumed
+        if (tid == 0) m_n[sidx] = 0;
+        __syncthreads();
+        if (k + 1 < nbatch) stage_meta(k + 1);         // metadata for the next stage
     }
     if (err) atomicOr(A.err, err);
     __syncthreads();
-    calib_flush(A, h, nbins);
+    calib_flush(A, h0, nbins, c + grp * A.CT);
 }
 // ------------------------------------------------------------------------------------------
 // a3: read ranges.  For each group of 32 consecutive sites [s0, s0+32) (one warp of
@@ -1122,54 +1167,65 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
     // walks the reads covering its 32 sites: metadata of 32 reads is loaded coalesced and
     // broadcast by shuffles; each lane reads the base and quality at its own site (consecutive
     // lanes -> consecutive bytes of a read).  Loads are issued four reads at a time.
+    // Positions are handled relative to the group's first site g0 (32-bit).  If every read in
+    // the range has the same length, '-' strand reads share a coordinate only within one start
+    // run and the end tracking below is skipped.
+    uint32_t one_len = 1;
+    {
+        const uint32_t L0 = wra < wrb ? A.R.len[wra] : 0u;
+        for (uint64_t r0 = wra; r0 < wrb; r0 += 32) {          // warp-uniform trip count
+            const uint64_t r = r0 + lane;
+            one_len &= (uint32_t)__all_sync(FULL, r >= wrb || A.R.len[r] == L0);
+        }
+    }
     uint32_t ca0 = 0, ca1 = 0, ca2 = 0, ca3 = 0, rep = 0, n = 0;
     bool slow_pcr = false, have_minus = false;
-    uint64_t run_pos = ~0ull, last_end = 0, last_end_pos = 0;
+    int run_pos = INT32_MIN;
     uint32_t run_start = 0;
+    int64_t last_end = 0, last_end_pos = 0;
     int err = 0;
     uint32_t* dbg_built = A.dbg_keys_built ? A.dbg_keys_built + (active ? A.dbg_off[site - A.w0] : 0) : nullptr;
     for (uint64_t r0 = wra; r0 < wrb; r0 += 32) {
         const uint64_t r = r0 + lane;
-        uint64_t p = ~0ull, o = 0;
-        uint32_t lh = 0, st = 0;
+        int pr = INT32_MAX;                                   // read start - g0
+        uint64_t o = 0;
+        uint32_t meta = 0;                                    // len | strand << 9 | hits << 10
         if (r < wrb) {
-            p = A.R.pos[r];
+            pr = (int)((int64_t)A.R.pos[r] - (int64_t)g0);
             o = A.R.off[r] - A.R.off0;
-            lh = (uint32_t)A.R.len[r] | (uint32_t)A.R.hits[r] << 16;
-            st = A.R.strand[r];
+            meta = (uint32_t)A.R.len[r] | (uint32_t)A.R.strand[r] << 9 | (uint32_t)A.R.hits[r] << 10;
         }
         const int nr = (int)min((uint64_t)32, wrb - r0);
+        uint32_t cpack = 0;                                   // 4 x 8-bit base counts this batch
         for (int k0 = 0; k0 < nr; k0 += 4) {
-            uint64_t pk[4], ii[4];
-            uint32_t lk[4], hk[4], sk[4], bb[4], qq[4];
+            int pk[4];
+            uint32_t ii[4], mk[4], bb[4], qq[4];
             bool cov[4];
 #pragma unroll
             for (int u = 0; u < 4; ++u) {
                 const int k = (k0 + u) & 31;
-                pk[u] = __shfl_sync(FULL, p, k);
+                pk[u] = __shfl_sync(FULL, pr, k);
                 const uint64_t ok = __shfl_sync(FULL, o, k);
-                const uint32_t lhk = __shfl_sync(FULL, lh, k);
-                sk[u] = __shfl_sync(FULL, st, k);
-                lk[u] = lhk & 0xFFFFu;
-                hk[u] = lhk >> 16;
-                ii[u] = site - pk[u];             // wraps (huge) when site < pos
-                cov[u] = active && k0 + u < nr && ii[u] < lk[u];
+                mk[u] = __shfl_sync(FULL, meta, k);
+                ii[u] = (uint32_t)(lane - pk[u]);            // wraps (huge) when lane < start
+                cov[u] = active && k0 + u < nr && ii[u] < (mk[u] & 511u);
                 bb[u] = cov[u] ? A.R.bases[ok + ii[u]] : 4u;
                 qq[u] = cov[u] ? A.R.quals[ok + ii[u]] : 0u;
             }
 #pragma unroll
             for (int u = 0; u < 4; ++u) {
                 const uint32_t b = bb[u], q = qq[u];
+                const uint32_t lk = mk[u] & 511u, sk = (mk[u] >> 9) & 1u, hk = mk[u] >> 10;
                 const bool nb = cov[u] && b < 4;                 // a non-N aligned base
                 err |= (cov[u] && b > 4) ? ERR_RANGE : 0;
-                ca0 += nb && b == 0; ca1 += nb && b == 1; ca2 += nb && b == 2; ca3 += nb && b == 3;
-                rep += nb ? hk[u] : 0u;
-                const bool uni = nb && hk[u] == 1;               // uniquely aligned
+                cpack += nb ? 1u << (8 * b) : 0u;
+                rep += nb ? hk : 0u;
+                const bool uni = nb && hk == 1;                  // uniquely aligned
                 err |= (uni && q > (uint32_t)A.q_max) ? ERR_QUAL : 0;
                 const bool use = uni && q <= (uint32_t)A.q_max;
-                const uint32_t i = (uint32_t)ii[u];
-                const uint32_t cyc = sk[u] ? lk[u] - 1 - i : i;
-                const uint32_t key = b << 15 | (63u - q) << 9 | cyc << 1 | sk[u];
+                const uint32_t i = ii[u];
+                const uint32_t cyc = sk ? lk - 1 - i : i;
+                const uint32_t key = b << 15 | (63u - q) << 9 | cyc << 1 | sk;
                 if (dbg_built && use) dbg_built[n] = key;
                 // pcr: keys sharing (base, strand, coord) come from reads with the same start
                 // ('+') or the same end ('-'); with equal starts they are one run of this
@@ -1186,17 +1242,20 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
                         }
                     }
                 }
-                // '-' ends must rise between start runs, else recount pcr in thread_site
-                const uint64_t e = pk[u] + lk[u] - 1;
-                const bool minus = use && sk[u];
-                slow_pcr |= minus && have_minus && (e < last_end || (e == last_end && pk[u] != last_end_pos));
-                last_end = minus ? e : last_end;
-                last_end_pos = minus ? pk[u] : last_end_pos;
-                have_minus |= minus;
+                if (!one_len) {       // '-' ends must rise between start runs, else recount pcr
+                    const int64_t e = (int64_t)pk[u] + lk - 1;
+                    const bool minus = use && sk;
+                    slow_pcr |= minus && have_minus &&
+                                (e < last_end || (e == last_end && pk[u] != last_end_pos));
+                    last_end = minus ? e : last_end;
+                    last_end_pos = minus ? pk[u] : last_end_pos;
+                    have_minus |= minus;
+                }
                 if (use && n < COLS) colp[n * TS] = key << 8 | min(pcr1, 255u);
                 n += use;
             }
         }
+        ca0 += cpack & 255u; ca1 += (cpack >> 8) & 255u; ca2 += (cpack >> 16) & 255u; ca3 += cpack >> 24;
     }
     if (err) atomicOr(A.err, err);
     if (A.count_only) {

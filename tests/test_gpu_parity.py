@@ -64,13 +64,15 @@ def test_c1_calibration_tables_bit_exact(c1):
         assert np.array_equal(t["counts"], C)
         L = OP.max_read_len
         assert np.array_equal(t["p"][:, :L], p[:, :L])
-        # T rows are Alg. 2's value for every (q, coord, base, genotype)
-        q = np.arange(1, 64)[:, None, None]
+        # T rows are Alg. 2's value for every (q_adj, coord, base, genotype), q_adj in [1, q_max]
+        # (adjust never leaves that range); the other rows are never indexed
         import math
         log10 = np.vectorize(math.log10)            # glibc log10, as Alg. 2 on the host
+        Q = OP.q_max + 1
         for n in range(10):
-            want = log10(0.5 * p[1:, :L, oracle.GA1[n], :] + 0.5 * p[1:, :L, oracle.GA2[n], :])
-            assert np.array_equal(t["T"][1:, :, :, n], want)
+            want = log10(0.5 * p[1:Q, :L, oracle.GA1[n], :] + 0.5 * p[1:Q, :L, oracle.GA2[n], :])
+            assert np.array_equal(t["T"][1:Q, :, :, n], want)
+        assert not t["T"][Q:].any() and not t["T"][0].any()
         # adjust table == the oracle's adjust in every cell
         adj = t["adj"]
         for qq in range(64):
@@ -78,7 +80,6 @@ def test_c1_calibration_tables_bit_exact(c1):
                 for g in range(0, adj.shape[2] + 3):
                     got = adj[qq, min(pcr, adj.shape[1]) - 1, min(g, adj.shape[2] - 1)]
                     assert got == oracle.adjust(OP, qq, pcr, g), (qq, pcr, g)
-        del q
 
 
 def test_c1_window_parity(c1):
@@ -252,3 +253,16 @@ def test_variable_length_reads_parity(seed):
     with _ctx(w) as ctx:
         ctx.calibrate(w)
         _check_window(ctx, w, 0, S, C, p)
+
+
+def test_long_reads_full_quality_range_parity():
+    """max_read_len 256 and q_max 63: 150-bp reads with qualities up to 63 (one histogram copy
+    per CTA in calibration, 256-cycle tables)."""
+    w = synth.generate("C1", n_sites=4_000, depth=25.0, read_len=150, q_hi=63, seed=77)
+    P = oracle.Params(max_read_len=256, q_max=63)
+    C, p, _, _ = _oracle_all(w, P, w0=0, w1=1)
+    with _ctx(w, max_read_len=256, q_max=63) as ctx:
+        counts = ctx.calibrate_count(w)
+        assert np.array_equal(counts.reshape(64, 256, 4, 4), C)
+        ctx.calibrate_finalize(counts)
+        _check_window(ctx, w, 0, 4_000, C, p, P)
