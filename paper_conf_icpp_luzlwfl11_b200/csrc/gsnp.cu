@@ -372,7 +372,10 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
     // persistent CTAs; warps pull 32-site groups from a counter.  The adjust table rides in
     // shared memory when small (it is 64 x 7 x 37 bytes at the default coefficients).
     const size_t adj_bytes = (size_t)64 * A.adjP * A.adjG;
-    const uint32_t adj_smem = adj_bytes <= 48 * 1024 ? 1u : 0u;
+#ifndef GSNP_ADJ_SMEM_MAX
+#define GSNP_ADJ_SMEM_MAX (48 * 1024)
+#endif
+    const uint32_t adj_smem = adj_bytes <= GSNP_ADJ_SMEM_MAX ? 1u : 0u;
     const size_t smem = call_smem_bytes(A.L, adj_smem ? adj_bytes : 0, nullptr, nullptr);
     const uint32_t big_cap = (uint32_t)std::min<uint64_t>(w1 - w0, 1u << 22);
     CK(ctx->big.ensure(big_cap));

@@ -367,7 +367,10 @@ __global__ void k_tile_ranges(const uint64_t* pos, uint64_t n, uint64_t w0, uint
 // k_call_tile: one CTA = TS = 256 consecutive sites, one thread per site (GSNP's baseline
 // parallelisation).  Shared-memory layout (host: call_smem_bytes()).
 constexpr int TS = NT;
-constexpr int COLS = 32;              // key slots per site on the thread-per-site path
+#ifndef GSNP_COLS
+#define GSNP_COLS 32
+#endif
+constexpr int COLS = GSNP_COLS;       // key slots per site on the thread-per-site path
 
 struct TileSmem {
     uint32_t* col;       // [COLS][TS] keys: column of site t at col[j*TS + t]; a warp's 32
@@ -396,13 +399,31 @@ __device__ __forceinline__ uint32_t key_cyc(uint32_t k) { return (k >> 1) & 255u
 __device__ __forceinline__ uint32_t key_slot(uint32_t k) { return k & 511u; }   // cyc<<1|strand
 constexpr uint32_t KEY_BSLOT = (3u << 15) | 511u;                               // base + slot
 
+#ifndef GSNP_T_NOALLOC
+#define GSNP_T_NOALLOC 0
+#endif
+#ifndef GSNP_P2_UNROLL
+#define GSNP_P2_UNROLL 2
+#endif
+constexpr int kP2Unroll = GSNP_P2_UNROLL;      // rows in flight per thread in likelihood pass 2
+// read-only 16-byte load that does not allocate in L1 (the table has little L1 reuse)
+__device__ __forceinline__ double2 ld_na(const double2* p) {
+    double2 v;
+    asm volatile("ld.global.nc.L1::no_allocate.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
+    return v;
+}
 // Score-table row of Alg. 3: 10 consecutive doubles at ((qa*L + coord)*4 + base)*10.
 __device__ __forceinline__ void add_row(const double* __restrict__ T, int L, uint32_t qa,
                                         uint32_t cyc, uint32_t b, double* acc) {
     const double2* row =
         reinterpret_cast<const double2*>(T + ((size_t)(qa * (uint32_t)L + cyc) * 4u + b) * 10u);
+#if GSNP_T_NOALLOC
+    double2 v0 = ld_na(row + 0), v1 = ld_na(row + 1), v2 = ld_na(row + 2), v3 = ld_na(row + 3),
+            v4 = ld_na(row + 4);
+#else
     double2 v0 = __ldg(row + 0), v1 = __ldg(row + 1), v2 = __ldg(row + 2), v3 = __ldg(row + 3),
             v4 = __ldg(row + 4);
+#endif
     acc[0] += v0.x; acc[1] += v0.y; acc[2] += v1.x; acc[3] += v1.y; acc[4] += v2.x;
     acc[5] += v2.y; acc[6] += v3.x; acc[7] += v3.y; acc[8] += v4.x; acc[9] += v4.y;
 }
@@ -615,7 +636,7 @@ __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* ad
     for (int j = 0; j < 10; ++j) acc[j] = 0.0;
     const double* __restrict__ T = A.T;
     const uint32_t L = (uint32_t)A.L;
-#pragma unroll 4
+#pragma unroll kP2Unroll
     for (uint32_t j = 0; j < n; ++j) {
         const uint32_t kk = colp[j * TS];
         add_row(T, (int)L, kk >> 17, key_cyc(kk), key_base(kk), acc);
