@@ -381,14 +381,15 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
     CK(ctx->big.ensure(big_cap));
     CK(ctx->big_n.ensure(2));
     CK(cudaMemsetAsync(ctx->big_n.p, 0, 8, s));     // [0] big-site count, [1] work counter
-    CK(cudaFuncSetAttribute(k_call_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    const bool dbg = A.count_only || A.dbg_off || A.dbg_counters || A.dbg_L10 || A.dbg_post10;
+    auto kern = dbg ? k_call_tile<true> : k_call_tile<false>;
+    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int per_sm = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_call_tile, NT, smem));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NT, smem));
     const uint64_t want = (uint64_t)g_num_sms * std::max(per_sm, 1);
     const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, n_tiles));
     ctx->begin();
-    k_call_tile<<<grid, NT, smem, s>>>(A, ctx->big.p, ctx->big_n.p, big_cap, ctx->big_n.p + 1,
-                                       adj_smem);
+    kern<<<grid, NT, smem, s>>>(A, ctx->big.p, ctx->big_n.p, big_cap, ctx->big_n.p + 1, adj_smem);
     ctx->end(GSNP_STAGE_CALL);
     ctx->launches++;
     CK(cudaGetLastError());

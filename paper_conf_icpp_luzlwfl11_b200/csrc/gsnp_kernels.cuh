@@ -601,10 +601,11 @@ __device__ __forceinline__ void sort_column(uint32_t* colp, uint32_t n) {
     for (int j = 0; j < N; ++j) if (j < (int)n) colp[j * TS] = k[j];
 }
 
+template <bool DBG>
 __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* adj, uint32_t* colp,
                                             uint64_t site, uint32_t n, bool slow_pcr, uint32_t ca0,
                                             uint32_t ca1, uint32_t ca2, uint32_t ca3, uint32_t rep) {
-    if (A.dbg_keys_sorted) {
+    if (DBG && A.dbg_keys_sorted) {
         const uint32_t o = A.dbg_off[site - A.w0];
         for (uint32_t j = 0; j < n; ++j) A.dbg_keys_sorted[o + j] = colp[j * TS] >> 8;
     }
@@ -656,7 +657,7 @@ __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* ad
     // posterior denominator in genotype order; a term below 1e-18 of the maximum cannot change
     // the double sum (every term is <= 1 and the maximum's term is exactly 1), so it is skipped
     // unless the debug dump wants every posterior
-    const bool all_terms = A.dbg_post10 != nullptr;
+    const bool all_terms = DBG && A.dbg_post10 != nullptr;
     uint32_t need = 0;
 #pragma unroll
     for (int j = 0; j < 10; ++j) need |= (all_terms || lp[j] - m > -18.0) ? 1u << j : 0u;
@@ -691,7 +692,7 @@ __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* ad
             tie += (double)eq * (double)eq - 1.0;
         }
     }
-    if (A.dbg_L10 || A.dbg_post10) {
+    if (DBG && (A.dbg_L10 || A.dbg_post10)) {
         const uint64_t s = site - A.w0;
         for (int j = 0; j < 10; ++j) {
             if (A.dbg_L10) A.dbg_L10[s * 10 + j] = acc[j];
@@ -1158,6 +1159,7 @@ struct BigSite {
 #ifndef GSNP_CALL_MINB
 #define GSNP_CALL_MINB 2
 #endif
+template <bool DBG>
 __global__ void __launch_bounds__(NT, GSNP_CALL_MINB)
 k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_t* work,
             uint32_t adj_smem) {
@@ -1182,7 +1184,8 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
     const uint64_t g0 = A.w0 + grp * 32;                     // first site of the group
     const uint64_t site = g0 + lane;
     const bool active = site < A.w1;
-    const uint64_t wra = A.tile_ra[grp], wrb = A.tile_rb[grp];
+    const uint64_t wra = A.tile_ra[grp];
+    uint64_t wrb = A.tile_rb[grp];
 
     // ---- counting + base_word gather, one site per lane.  The warp
     // walks the reads covering its 32 sites: metadata of 32 reads is loaded coalesced and
@@ -1205,49 +1208,57 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
     uint32_t run_start = 0;
     int64_t last_end = 0, last_end_pos = 0;
     int err = 0;
-    uint32_t* dbg_built = A.dbg_keys_built ? A.dbg_keys_built + (active ? A.dbg_off[site - A.w0] : 0) : nullptr;
+    uint32_t* dbg_built = nullptr;
+    if (DBG && A.dbg_keys_built) dbg_built = A.dbg_keys_built + (active ? A.dbg_off[site - A.w0] : 0);
+    // byte arrays addressed from the warp's first read with 32-bit offsets: the bases of the
+    // reads covering 32 consecutive sites must span < 2 GB (else GSNP_E_RANGE)
+    const uint64_t ob = wra < wrb ? A.R.off[wra] - A.R.off0 : 0;
+    if (wra < wrb && A.R.off[wrb] - A.R.off[wra] >= (1ull << 31)) { err |= ERR_RANGE; wrb = wra; }
+    const uint8_t* __restrict__ wbases = A.R.bases + ob;
+    const uint8_t* __restrict__ wquals = A.R.quals + ob;
+    const int lane_rel = active ? lane : INT32_MIN / 2;     // inactive lanes are never covered
     for (uint64_t r0 = wra; r0 < wrb; r0 += 32) {
         const uint64_t r = r0 + lane;
-        int pr = INT32_MAX;                                   // read start - g0
-        uint64_t o = 0;
-        uint32_t meta = 0;                                    // len | strand << 9 | hits << 10
+        int pr = INT32_MAX / 2;                                // read start - g0
+        uint32_t o = 0;                                        // bases offset - ob
+        uint32_t meta = 0;                                     // len | strand << 9 | hits << 10
         if (r < wrb) {
             pr = (int)((int64_t)A.R.pos[r] - (int64_t)g0);
-            o = A.R.off[r] - A.R.off0;
+            o = (uint32_t)(A.R.off[r] - A.R.off0 - ob);
             meta = (uint32_t)A.R.len[r] | (uint32_t)A.R.strand[r] << 9 | (uint32_t)A.R.hits[r] << 10;
         }
         const int nr = (int)min((uint64_t)32, wrb - r0);
-        uint32_t cpack = 0;                                   // 4 x 8-bit base counts this batch
+        uint32_t cpack = 0;                                    // 4 x 8-bit base counts this batch
         for (int k0 = 0; k0 < nr; k0 += 4) {
             int pk[4];
             uint32_t ii[4], mk[4], bb[4], qq[4];
-            bool cov[4];
 #pragma unroll
             for (int u = 0; u < 4; ++u) {
                 const int k = (k0 + u) & 31;
                 pk[u] = __shfl_sync(FULL, pr, k);
-                const uint64_t ok = __shfl_sync(FULL, o, k);
+                const uint32_t ok = __shfl_sync(FULL, o, k);
                 mk[u] = __shfl_sync(FULL, meta, k);
-                ii[u] = (uint32_t)(lane - pk[u]);            // wraps (huge) when lane < start
-                cov[u] = active && k0 + u < nr && ii[u] < (mk[u] & 511u);
-                bb[u] = cov[u] ? A.R.bases[ok + ii[u]] : 4u;
-                qq[u] = cov[u] ? A.R.quals[ok + ii[u]] : 0u;
+                if (k0 + u >= nr) pk[u] = INT32_MAX / 2;       // past the batch: covers nothing
+                ii[u] = (uint32_t)(lane_rel - pk[u]);           // huge unless 0 <= i < len
+                const bool cov = ii[u] < (mk[u] & 511u);
+                bb[u] = cov ? wbases[ok + ii[u]] : 4u;
+                qq[u] = cov ? wquals[ok + ii[u]] : 0u;
+                if (!cov) mk[u] = 0;                           // len 0: not covered below
             }
 #pragma unroll
             for (int u = 0; u < 4; ++u) {
                 const uint32_t b = bb[u], q = qq[u];
                 const uint32_t lk = mk[u] & 511u, sk = (mk[u] >> 9) & 1u, hk = mk[u] >> 10;
-                const bool nb = cov[u] && b < 4;                 // a non-N aligned base
-                err |= (cov[u] && b > 4) ? ERR_RANGE : 0;
+                const bool cov = lk != 0;
+                err |= (cov && (b > 4 || q > (uint32_t)A.q_max)) ? ERR_RANGE : 0;
+                const bool nb = b < 4;                           // a non-N aligned base
                 cpack += nb ? 1u << (8 * b) : 0u;
                 rep += nb ? hk : 0u;
-                const bool uni = nb && hk == 1;                  // uniquely aligned
-                err |= (uni && q > (uint32_t)A.q_max) ? ERR_QUAL : 0;
-                const bool use = uni && q <= (uint32_t)A.q_max;
+                const bool use = nb && hk == 1;                  // uniquely aligned
                 const uint32_t i = ii[u];
                 const uint32_t cyc = sk ? lk - 1 - i : i;
-                const uint32_t key = b << 15 | (63u - q) << 9 | cyc << 1 | sk;
-                if (dbg_built && use) dbg_built[n] = key;
+                const uint32_t key = b << 15 | ((63u - q) & 63u) << 9 | cyc << 1 | sk;
+                if (DBG && dbg_built && use) dbg_built[n] = key;
                 // pcr: keys sharing (base, strand, coord) come from reads with the same start
                 // ('+') or the same end ('-'); with equal starts they are one run of this
                 // column.  Canonical order among them is quality descending (R3).
@@ -1279,7 +1290,7 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
         ca0 += cpack & 255u; ca1 += (cpack >> 8) & 255u; ca2 += (cpack >> 16) & 255u; ca3 += cpack >> 24;
     }
     if (err) atomicOr(A.err, err);
-    if (A.count_only) {
+    if (DBG && A.count_only) {
         if (active) A.dbg_nuni[site - A.w0] = n;
         continue;
     }
@@ -1290,7 +1301,7 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
     if (small) {
         if (maxn <= 16) sort_column<16>(colp, n);
         else sort_column<32>(colp, n);
-        thread_site(A, adj, colp, site, n, slow_pcr, ca0, ca1, ca2, ca3, rep);
+        thread_site<DBG>(A, adj, colp, site, n, slow_pcr, ca0, ca1, ca2, ca3, rep);
     }
     __syncwarp();
 
