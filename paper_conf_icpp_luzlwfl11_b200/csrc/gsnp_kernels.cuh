@@ -406,6 +406,9 @@ constexpr uint32_t KEY_BSLOT = (3u << 15) | 511u;                               
 #define GSNP_P2_UNROLL 2
 #endif
 constexpr int kP2Unroll = GSNP_P2_UNROLL;      // rows in flight per thread in likelihood pass 2
+#ifndef GSNP_FUSED_PASS
+#define GSNP_FUSED_PASS 0
+#endif
 // read-only 16-byte load that does not allocate in L1 (the table has little L1 reuse)
 __device__ __forceinline__ double2 ld_na(const double2* p) {
     double2 v;
@@ -615,6 +618,31 @@ __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* ad
     // q_adj = adjust(q, pcr, g).  Each key becomes key | q_adj << 17.
     uint64_t cu = 0, qs = 0;
     uint32_t prev_b = 4, distinct = 0;
+    double acc[10];
+#pragma unroll
+    for (int j = 0; j < 10; ++j) acc[j] = 0.0;
+    const double* __restrict__ T = A.T;
+    const uint32_t L = (uint32_t)A.L;
+#if GSNP_FUSED_PASS
+    // one pass: q_adj and the Alg. 3 row per key (keys keep their key << 8 | pcr-1 form)
+#pragma unroll kP2Unroll
+    for (uint32_t j = 0; j < n; ++j) {
+        const uint32_t kw = colp[j * TS];
+        const uint32_t kk = kw >> 8, b = key_base(kk), q = key_q(kk);
+        uint32_t pcr = (kw & 255u) + 1u;
+        if (slow_pcr) {
+            pcr = 1;
+            for (uint32_t i = 0; i < j; ++i) pcr += (((colp[i * TS] >> 8) ^ kk) & KEY_BSLOT) == 0;
+        }
+        if (b != prev_b) { distinct = 0; prev_b = b; }
+        distinct += pcr == 1;
+        const uint32_t qa = (uint32_t)adj_lookup_t(adj, A.adjP, A.adjG, q, pcr, distinct - 1);
+        add_row(T, (int)L, qa, key_cyc(kk), b, acc);
+        cu += 1ull << (16 * b);
+        qs += (uint64_t)q << (16 * b);
+    }
+#define COLKEY(w) ((w) >> 8)
+#else
     for (uint32_t j = 0; j < n; ++j) {
         const uint32_t kw = colp[j * TS];
         const uint32_t kk = kw >> 8, b = key_base(kk), q = key_q(kk);
@@ -631,17 +659,14 @@ __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* ad
         qs += (uint64_t)q << (16 * b);
     }
     // pass 2: type_likely[n] += new_p_matrix[row][n] (Alg. 3) in canonical order; no load
-    // depends on another, so four rows are in flight per thread
-    double acc[10];
-#pragma unroll
-    for (int j = 0; j < 10; ++j) acc[j] = 0.0;
-    const double* __restrict__ T = A.T;
-    const uint32_t L = (uint32_t)A.L;
+    // depends on another, so several rows are in flight per thread
 #pragma unroll kP2Unroll
     for (uint32_t j = 0; j < n; ++j) {
         const uint32_t kk = colp[j * TS];
         add_row(T, (int)L, kk >> 17, key_cyc(kk), key_base(kk), acc);
     }
+#define COLKEY(w) ((w) & 0x1FFFFu)
+#endif
     // C6/C7: priors, posterior, top-2
     int refb;
     const int64_t kidx = site_ref(A, site, refb);
@@ -677,19 +702,24 @@ __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* ad
     const int a1 = geno_a1(t1), a2 = geno_a2(t1);
     double wsum = 0.0, tie = 0.0;
     if (a1 != a2 && (A.flags & GSNP_RANK_SUM) && f16(cu, a1) && f16(cu, a2)) {
-        for (uint32_t x = 0; x < n; ++x) {
-            const uint32_t xk = colp[x * TS] & 0x1FFFFu;
-            const uint32_t xb = key_base(xk), xq = key_q(xk);
-            if (xb != (uint32_t)a1 && xb != (uint32_t)a2) continue;
-            uint32_t less = 0, eq = 0;
-            for (uint32_t y = 0; y < n; ++y) {
-                const uint32_t yk = colp[y * TS] & 0x1FFFFu, yb = key_base(yk), yq = key_q(yk);
-                const bool yin = yb == (uint32_t)a1 || yb == (uint32_t)a2;
-                less += yin && yq < xq;
-                eq += yin && yq == xq;
-            }
-            if (xb == (uint32_t)a1) wsum += (double)less + ((double)eq + 1.0) / 2.0;
-            tie += (double)eq * (double)eq - 1.0;
+        // The column is in canonical order: each allele's keys are one run with qualities
+        // descending, so the pooled mid-ranks come from one merge from the low-quality ends.
+        uint32_t sx = 0, sy = 0;
+        for (int b = 0; b < a1; ++b) sx += f16(cu, b);
+        for (int b = 0; b < a2; ++b) sy += f16(cu, b);
+        uint32_t ix = sx + f16(cu, a1), iy = sy + f16(cu, a2);
+        double less = 0.0;
+        while (ix > sx || iy > sy) {
+            const uint32_t qx = ix > sx ? key_q(COLKEY(colp[(ix - 1) * TS])) : 99u;
+            const uint32_t qy = iy > sy ? key_q(COLKEY(colp[(iy - 1) * TS])) : 99u;
+            const uint32_t v = min(qx, qy);
+            uint32_t cx = 0, cy = 0;
+            while (ix > sx && key_q(COLKEY(colp[(ix - 1) * TS])) == v) { ++cx; --ix; }
+            while (iy > sy && key_q(COLKEY(colp[(iy - 1) * TS])) == v) { ++cy; --iy; }
+            const double t = (double)(cx + cy);
+            wsum += (double)cx * (less + (t + 1.0) / 2.0);
+            tie += t * t * t - t;
+            less += t;
         }
     }
     if (DBG && (A.dbg_L10 || A.dbg_post10)) {
