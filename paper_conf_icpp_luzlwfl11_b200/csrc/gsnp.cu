@@ -376,13 +376,24 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
 #define GSNP_ADJ_SMEM_MAX (48 * 1024)
 #endif
     const uint32_t adj_smem = adj_bytes <= GSNP_ADJ_SMEM_MAX ? 1u : 0u;
-    const size_t smem = call_smem_bytes(A.L, adj_smem ? adj_bytes : 0, nullptr, nullptr);
+    // deep windows (mean depth >= 48 by read count) keep up to 128 keys per thread
+    uint64_t rr[2] = {0, 0};
+    if (d.n) {
+        CK(cudaMemcpyAsync(&rr[0], ctx->tile_ra.p, 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(&rr[1], ctx->tile_rb.p + n_groups - 1, 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+    }
+    const double depth_est = (double)(rr[1] - rr[0]) * A.L / (double)(w1 - w0);
+    const bool deep = depth_est >= 48.0;
+    const int cols = deep ? COLS_DEEP : COLS;
+    const size_t smem = call_smem_bytes(A.L, adj_smem ? adj_bytes : 0, cols, nullptr, nullptr);
     const uint32_t big_cap = (uint32_t)std::min<uint64_t>(w1 - w0, 1u << 22);
     CK(ctx->big.ensure(big_cap));
     CK(ctx->big_n.ensure(2));
     CK(cudaMemsetAsync(ctx->big_n.p, 0, 8, s));     // [0] big-site count, [1] work counter
     const bool dbg = A.count_only || A.dbg_off || A.dbg_counters || A.dbg_L10 || A.dbg_post10;
-    auto kern = dbg ? k_call_tile<true> : k_call_tile<false>;
+    auto kern = dbg ? (deep ? k_call_tile<true, COLS_DEEP> : k_call_tile<true, COLS>)
+                    : (deep ? k_call_tile<false, COLS_DEEP> : k_call_tile<false, COLS>);
     CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int per_sm = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NT, smem));

@@ -367,10 +367,8 @@ __global__ void k_tile_ranges(const uint64_t* pos, uint64_t n, uint64_t w0, uint
 // k_call_tile: one CTA = TS = 256 consecutive sites, one thread per site (GSNP's baseline
 // parallelisation).  Shared-memory layout (host: call_smem_bytes()).
 constexpr int TS = NT;
-#ifndef GSNP_COLS
-#define GSNP_COLS 32
-#endif
-constexpr int COLS = GSNP_COLS;       // key slots per site on the thread-per-site path
+constexpr int COLS = 32;              // key slots per site, shallow kernel (thread path n <= 32)
+constexpr int COLS_DEEP = 128;        // key slots per site, deep kernel (thread path n <= 128)
 
 struct TileSmem {
     uint32_t* col;       // [COLS][TS] keys: column of site t at col[j*TS + t]; a warp's 32
@@ -379,10 +377,10 @@ struct TileSmem {
     uint8_t* adj;        // copy of the adjust table (adj_bytes, 0 = use global)
 };
 
-__host__ __device__ inline size_t call_smem_bytes(int L, size_t adj_bytes, TileSmem* s,
+__host__ __device__ inline size_t call_smem_bytes(int L, size_t adj_bytes, int cols, TileSmem* s,
                                                    unsigned char* base) {
     size_t o_col = 0;
-    size_t o_slot = align16(4 * (size_t)COLS * TS);
+    size_t o_slot = align16(4 * (size_t)cols * TS);
     size_t o_adj = align16(o_slot + (size_t)NW * 8 * L);
     size_t total = align16(o_adj + adj_bytes);
     if (s) {
@@ -604,6 +602,105 @@ __device__ __forceinline__ void sort_column(uint32_t* colp, uint32_t n) {
     for (int j = 0; j < N; ++j) if (j < (int)n) colp[j * TS] = k[j];
 }
 
+// key of a thread-path column entry after the likelihood pass(es)
+#if GSNP_FUSED_PASS
+#define COLKEY(w) ((w) >> 8)
+#else
+#define COLKEY(w) ((w) & 0x1FFFFu)
+#endif
+
+// C6-C9 for one site held by one thread: priors, posterior, top-2, rank-sum pieces, record.
+// SORTED: the column holds the site's keys in canonical order (rank-sum by one merge).
+template <bool DBG, bool SORTED>
+__device__ __forceinline__ void thread_finish(const CallArgs& A, const uint32_t* colp,
+                                              uint64_t site, uint32_t n, const double* acc,
+                                              uint64_t cu, uint64_t qs, uint32_t ca0,
+                                              uint32_t ca1, uint32_t ca2, uint32_t ca3,
+                                              uint32_t rep) {
+    // C6/C7: priors, posterior, top-2
+    int refb;
+    const int64_t kidx = site_ref(A, site, refb);
+    const double* prow = kidx >= 0 ? A.known_lp + kidx * 10 : A.LP + refb * 10;
+    double lp[10], m = -INFINITY;
+#pragma unroll
+    for (int j = 0; j < 10; ++j) {
+        lp[j] = acc[j] + __ldg(prow + j);
+        m = lp[j] > m ? lp[j] : m;
+    }
+    int t1, t2;
+    top2(lp, t1, t2);
+    // posterior denominator in genotype order; a term below 1e-18 of the maximum cannot change
+    // the double sum (every term is <= 1 and the maximum's term is exactly 1), so it is skipped
+    // unless the debug dump wants every posterior
+    const bool all_terms = DBG && A.dbg_post10 != nullptr;
+    uint32_t need = 0;
+#pragma unroll
+    for (int j = 0; j < 10; ++j) need |= (all_terms || lp[j] - m > -18.0) ? 1u << j : 0u;
+    double esum = 0.0;
+    const uint32_t am = __activemask();
+    while (__any_sync(am, need != 0)) {                // terms in genotype order, one per pass
+        if (need) {
+            const int jj = __ffs(need) - 1;
+            need &= need - 1;
+            double x = lp[0];
+#pragma unroll
+            for (int j = 1; j < 10; ++j) x = jj == j ? lp[j] : x;
+            esum += exp10(x - m);
+        }
+    }
+    // C8 pieces: W = sum of pooled mid-ranks of allele-1 qualities; tie = sum(t^3 - t)
+    const int a1 = geno_a1(t1), a2 = geno_a2(t1);
+    double wsum = 0.0, tie = 0.0;
+    if (SORTED && a1 != a2 && (A.flags & GSNP_RANK_SUM) && f16(cu, a1) && f16(cu, a2)) {
+        // The column is in canonical order: each allele's keys are one run with qualities
+        // descending, so the pooled mid-ranks come from one merge from the low-quality ends.
+        uint32_t sx = 0, sy = 0;
+        for (int b = 0; b < a1; ++b) sx += f16(cu, b);
+        for (int b = 0; b < a2; ++b) sy += f16(cu, b);
+        uint32_t ix = sx + f16(cu, a1), iy = sy + f16(cu, a2);
+        double less = 0.0;
+        while (ix > sx || iy > sy) {
+            const uint32_t qx = ix > sx ? key_q(COLKEY(colp[(ix - 1) * TS])) : 99u;
+            const uint32_t qy = iy > sy ? key_q(COLKEY(colp[(iy - 1) * TS])) : 99u;
+            const uint32_t v = min(qx, qy);
+            uint32_t cx = 0, cy = 0;
+            while (ix > sx && key_q(COLKEY(colp[(ix - 1) * TS])) == v) { ++cx; --ix; }
+            while (iy > sy && key_q(COLKEY(colp[(iy - 1) * TS])) == v) { ++cy; --iy; }
+            const double t = (double)(cx + cy);
+            wsum += (double)cx * (less + (t + 1.0) / 2.0);
+            tie += t * t * t - t;
+            less += t;
+        }
+    }
+    if (!SORTED && a1 != a2 && (A.flags & GSNP_RANK_SUM) && f16(cu, a1) && f16(cu, a2)) {
+        // column in chunk order: pooled mid-ranks by pairwise counts (het calls only)
+        for (uint32_t x = 0; x < n; ++x) {
+            const uint32_t xk = colp[x * TS] >> 8;
+            const uint32_t xb = key_base(xk), xq = key_q(xk);
+            if (xb != (uint32_t)a1 && xb != (uint32_t)a2) continue;
+            uint32_t less = 0, eq = 0;
+            for (uint32_t y = 0; y < n; ++y) {
+                const uint32_t yk = colp[y * TS] >> 8, yb = key_base(yk), yq = key_q(yk);
+                const bool yin = yb == (uint32_t)a1 || yb == (uint32_t)a2;
+                less += yin && yq < xq;
+                eq += yin && yq == xq;
+            }
+            if (xb == (uint32_t)a1) wsum += (double)less + ((double)eq + 1.0) / 2.0;
+            tie += (double)eq * (double)eq - 1.0;
+        }
+    }
+    if (DBG && (A.dbg_L10 || A.dbg_post10)) {
+        const uint64_t s = site - A.w0;
+        for (int j = 0; j < 10; ++j) {
+            if (A.dbg_L10) A.dbg_L10[s * 10 + j] = acc[j];
+            if (A.dbg_post10) A.dbg_post10[s * 10 + j] = exp10(lp[j] - m) / esum;
+        }
+    }
+    site_record(A, site, refb, kidx >= 0, t1, lp[t1] - lp[t2], 1.0 / esum, f16(cu, 0), f16(cu, 1),
+                f16(cu, 2), f16(cu, 3), f16(qs, 0), f16(qs, 1), f16(qs, 2), f16(qs, 3), ca0, ca1,
+                ca2, ca3, rep, wsum, tie);
+}
+
 template <bool DBG>
 __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* adj, uint32_t* colp,
                                             uint64_t site, uint32_t n, bool slow_pcr, uint32_t ca0,
@@ -641,7 +738,6 @@ __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* ad
         cu += 1ull << (16 * b);
         qs += (uint64_t)q << (16 * b);
     }
-#define COLKEY(w) ((w) >> 8)
 #else
     for (uint32_t j = 0; j < n; ++j) {
         const uint32_t kw = colp[j * TS];
@@ -665,73 +761,57 @@ __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* ad
         const uint32_t kk = colp[j * TS];
         add_row(T, (int)L, kk >> 17, key_cyc(kk), key_base(kk), acc);
     }
-#define COLKEY(w) ((w) & 0x1FFFFu)
 #endif
-    // C6/C7: priors, posterior, top-2
-    int refb;
-    const int64_t kidx = site_ref(A, site, refb);
-    const double* prow = kidx >= 0 ? A.known_lp + kidx * 10 : A.LP + refb * 10;
-    double lp[10], m = -INFINITY;
+    thread_finish<DBG, true>(A, colp, site, n, acc, cu, qs, ca0, ca1, ca2, ca3, rep);
+}
+
+// Deep thread path (32 < n <= 32*NCH, kernels built with 128 slots per site): each 32-key chunk
+// of the column is sorted in registers, then an NCH-way streaming merge visits the keys in
+// canonical order straight into Alg. 4 (q_adj and the Alg. 3 row per key).
+template <bool DBG, int NCH>
+__device__ __forceinline__ void thread_site_deep(const CallArgs& A, const uint8_t* adj,
+                                                 uint32_t* colp, uint64_t site, uint32_t n,
+                                                 uint32_t ca0, uint32_t ca1, uint32_t ca2,
+                                                 uint32_t ca3, uint32_t rep) {
+#pragma unroll 1
+    for (int c = 0; c < NCH; ++c) {
+        const uint32_t cn = n > 32u * c ? min(32u, n - 32u * c) : 0u;
+        if (cn) sort_column<32>(colp + (size_t)32 * c * TS, cn);
+    }
+    uint32_t hi[NCH], he[NCH], hk[NCH];
 #pragma unroll
-    for (int j = 0; j < 10; ++j) {
-        lp[j] = acc[j] + __ldg(prow + j);
-        m = lp[j] > m ? lp[j] : m;
+    for (int c = 0; c < NCH; ++c) {
+        hi[c] = 32u * c;
+        he[c] = min(n, 32u * c + 32u);
+        hk[c] = hi[c] < he[c] ? colp[hi[c] * TS] : KEY_INF;
     }
-    int t1, t2;
-    top2(lp, t1, t2);
-    // posterior denominator in genotype order; a term below 1e-18 of the maximum cannot change
-    // the double sum (every term is <= 1 and the maximum's term is exactly 1), so it is skipped
-    // unless the debug dump wants every posterior
-    const bool all_terms = DBG && A.dbg_post10 != nullptr;
-    uint32_t need = 0;
+    uint32_t* dbg = nullptr;
+    if (DBG && A.dbg_keys_sorted) dbg = A.dbg_keys_sorted + A.dbg_off[site - A.w0];
+    double acc[10];
 #pragma unroll
-    for (int j = 0; j < 10; ++j) need |= (all_terms || lp[j] - m > -18.0) ? 1u << j : 0u;
-    double esum = 0.0;
-    const uint32_t am = __activemask();
-    while (__any_sync(am, need != 0)) {                // terms in genotype order, one per pass
-        if (need) {
-            const int jj = __ffs(need) - 1;
-            need &= need - 1;
-            double x = lp[0];
+    for (int j = 0; j < 10; ++j) acc[j] = 0.0;
+    uint64_t cu = 0, qs = 0;
+    uint32_t prev_b = 4, distinct = 0;
+    const double* __restrict__ T = A.T;
+    for (uint32_t out = 0; out < n; ++out) {
+        uint32_t best = hk[0];
+        int bc = 0;
 #pragma unroll
-            for (int j = 1; j < 10; ++j) x = jj == j ? lp[j] : x;
-            esum += exp10(x - m);
-        }
+        for (int c = 1; c < NCH; ++c) if (hk[c] < best) { best = hk[c]; bc = c; }
+#pragma unroll
+        for (int c = 0; c < NCH; ++c)
+            if (c == bc) { ++hi[c]; hk[c] = hi[c] < he[c] ? colp[hi[c] * TS] : KEY_INF; }
+        const uint32_t kk = best >> 8, b = key_base(kk), q = key_q(kk);
+        if (DBG && dbg) dbg[out] = kk;
+        const uint32_t pcr = (best & 255u) + 1u;
+        if (b != prev_b) { distinct = 0; prev_b = b; }
+        distinct += pcr == 1;
+        const uint32_t qa = (uint32_t)adj_lookup_t(adj, A.adjP, A.adjG, q, pcr, distinct - 1);
+        add_row(T, A.L, qa, key_cyc(kk), b, acc);
+        cu += 1ull << (16 * b);
+        qs += (uint64_t)q << (16 * b);
     }
-    // C8 pieces: W = sum of pooled mid-ranks of allele-1 qualities; tie = sum(t^3 - t)
-    const int a1 = geno_a1(t1), a2 = geno_a2(t1);
-    double wsum = 0.0, tie = 0.0;
-    if (a1 != a2 && (A.flags & GSNP_RANK_SUM) && f16(cu, a1) && f16(cu, a2)) {
-        // The column is in canonical order: each allele's keys are one run with qualities
-        // descending, so the pooled mid-ranks come from one merge from the low-quality ends.
-        uint32_t sx = 0, sy = 0;
-        for (int b = 0; b < a1; ++b) sx += f16(cu, b);
-        for (int b = 0; b < a2; ++b) sy += f16(cu, b);
-        uint32_t ix = sx + f16(cu, a1), iy = sy + f16(cu, a2);
-        double less = 0.0;
-        while (ix > sx || iy > sy) {
-            const uint32_t qx = ix > sx ? key_q(COLKEY(colp[(ix - 1) * TS])) : 99u;
-            const uint32_t qy = iy > sy ? key_q(COLKEY(colp[(iy - 1) * TS])) : 99u;
-            const uint32_t v = min(qx, qy);
-            uint32_t cx = 0, cy = 0;
-            while (ix > sx && key_q(COLKEY(colp[(ix - 1) * TS])) == v) { ++cx; --ix; }
-            while (iy > sy && key_q(COLKEY(colp[(iy - 1) * TS])) == v) { ++cy; --iy; }
-            const double t = (double)(cx + cy);
-            wsum += (double)cx * (less + (t + 1.0) / 2.0);
-            tie += t * t * t - t;
-            less += t;
-        }
-    }
-    if (DBG && (A.dbg_L10 || A.dbg_post10)) {
-        const uint64_t s = site - A.w0;
-        for (int j = 0; j < 10; ++j) {
-            if (A.dbg_L10) A.dbg_L10[s * 10 + j] = acc[j];
-            if (A.dbg_post10) A.dbg_post10[s * 10 + j] = exp10(lp[j] - m) / esum;
-        }
-    }
-    site_record(A, site, refb, kidx >= 0, t1, lp[t1] - lp[t2], 1.0 / esum, f16(cu, 0), f16(cu, 1),
-                f16(cu, 2), f16(cu, 3), f16(qs, 0), f16(qs, 1), f16(qs, 2), f16(qs, 3), ca0, ca1,
-                ca2, ca3, rep, wsum, tie);
+    thread_finish<DBG, false>(A, colp, site, n, acc, cu, qs, ca0, ca1, ca2, ca3, rep);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1176,7 +1256,7 @@ __device__ __noinline__ void cta_site(const CallArgs& A, uint8_t* slotcnt, uint3
 }
 
 // ------------------------------------------------------------------------------------------
-// Sites with more than 32*COLS unique keys are handed to k_big_sites through a global list.
+// Sites with more than 32*CC unique keys are handed to k_big_sites through a global list.
 struct BigSite {
     uint64_t site;
     uint32_t n, ca0, ca1, ca2, ca3, rep;
@@ -1189,14 +1269,14 @@ struct BigSite {
 #ifndef GSNP_CALL_MINB
 #define GSNP_CALL_MINB 2
 #endif
-template <bool DBG>
+template <bool DBG, int CC>
 __global__ void __launch_bounds__(NT, GSNP_CALL_MINB)
 k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_t* work,
             uint32_t adj_smem) {
     extern __shared__ __align__(16) unsigned char smem[];
     TileSmem sm;
     const size_t adj_bytes = adj_smem ? (size_t)64 * A.adjP * A.adjG : 0;
-    call_smem_bytes(A.L, adj_bytes, &sm, smem);
+    call_smem_bytes(A.L, adj_bytes, CC, &sm, smem);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     for (size_t i = tid; i < adj_bytes; i += NT) sm.adj[i] = A.adj[i];
     const uint8_t* adj = adj_smem ? sm.adj : A.adj;
@@ -1295,7 +1375,7 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
                 if (pk[u] != run_pos) { run_pos = pk[u]; run_start = n; }
                 uint32_t pcr1 = 0;
                 if (use && run_start < n) {
-                    const uint32_t jend = min(n, (uint32_t)COLS);
+                    const uint32_t jend = min(n, (uint32_t)CC);
                     for (uint32_t j = run_start; j < jend; ++j) {
                         const uint32_t kj = colp[j * TS];
                         if ((((kj >> 8) ^ key) & KEY_BSLOT) == 0) {
@@ -1313,7 +1393,7 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
                     last_end_pos = minus ? pk[u] : last_end_pos;
                     have_minus |= minus;
                 }
-                if (use && n < COLS) colp[n * TS] = key << 8 | min(pcr1, 255u);
+                if (use && n < CC) colp[n * TS] = key << 8 | min(pcr1, 255u);
                 n += use;
             }
         }
@@ -1325,18 +1405,22 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
         continue;
     }
 
-    // ---- thread-per-site sort (in-register network sized per warp: 16 / 32) + likelihood
+    // ---- thread-per-site sort (in-register network sized per warp: 16 / 32) + likelihood;
+    // the deep kernel also keeps 33..128-key sites on the thread path (chunked sort + merge)
     const bool small = active && n <= COLS;
+    const bool mid = CC > COLS && active && n > COLS && n <= CC && !slow_pcr;
     const uint32_t maxn = __reduce_max_sync(FULL, small ? n : 0u);
     if (small) {
         if (maxn <= 16) sort_column<16>(colp, n);
         else sort_column<32>(colp, n);
         thread_site<DBG>(A, adj, colp, site, n, slow_pcr, ca0, ca1, ca2, ca3, rep);
+    } else if (mid) {
+        thread_site_deep<DBG, CC / 32>(A, adj, colp, site, n, ca0, ca1, ca2, ca3, rep);
     }
     __syncwarp();
 
     // ---- this warp's deeper sites: warp paths (n <= 1024) or the k_big_sites list
-    uint32_t ovf = __ballot_sync(FULL, active && n > COLS);
+    uint32_t ovf = __ballot_sync(FULL, active && n > COLS && !mid);
     while (ovf) {
         const int l = __ffs(ovf) - 1;
         ovf &= ovf - 1;
@@ -1345,7 +1429,7 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
         const uint32_t c2 = __shfl_sync(FULL, ca2, l), c3 = __shfl_sync(FULL, ca3, l);
         const uint32_t rp = __shfl_sync(FULL, rep, l);
         const uint64_t s = g0 + l;
-        if (nn > 32 * COLS) {
+        if (nn > 32 * CC) {
             if (lane == l) {
                 const uint32_t j = atomicAdd(big_n, 1u);
                 if (j < big_cap) big[j] = BigSite{s, nn, c0, c1, c2, c3, rp};
