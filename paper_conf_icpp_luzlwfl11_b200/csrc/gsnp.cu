@@ -243,6 +243,7 @@ void estimate_p_q(const gsnp_params& prm, const uint64_t* C, double* p, int q) {
 
 // Alg. 3 score-table rows of quality qa: T[qa][c][b][n] = log10(0.5 p[qa][c][a1][b] +
 // 0.5 p[qa][c][a2][b]), the value Alg. 2 returns, built on the CPU (§IV-G).
+// Rows are stored with TROW (>= 10) doubles each; the padding stays zero.
 void build_T_q(int L, const double* p, double* T, int qa) {
     static const int A1[10] = {0, 0, 0, 0, 1, 1, 1, 2, 2, 3};
     static const int A2[10] = {0, 1, 2, 3, 1, 2, 3, 2, 3, 3};
@@ -251,7 +252,7 @@ void build_T_q(int L, const double* p, double* T, int qa) {
             for (int n = 0; n < 10; ++n) {
                 int p1 = qa << 12 | c << 4 | A1[n] << 2 | b;
                 int p2 = qa << 12 | c << 4 | A2[n] << 2 | b;
-                T[(((size_t)qa * L + c) * 4 + b) * 10 + n] = log10(0.5 * p[p1] + 0.5 * p[p2]);
+                T[(((size_t)qa * L + c) * 4 + b) * TROW + n] = log10(0.5 * p[p1] + 0.5 * p[p2]);
             }
 }
 
@@ -472,7 +473,7 @@ gsnp_status finalize_impl(gsnp_ctx* ctx, const uint64_t* counts_host) {
     const int qmax = (int)ctx->prm.q_max;
     ctx->h_counts.assign(counts_host, counts_host + 64 * 256 * 16);
     ctx->h_p.assign((size_t)64 * 256 * 16, 0.0);
-    const size_t tn = (size_t)64 * L * 4 * 10;
+    const size_t tn = (size_t)64 * L * 4 * TROW;
     if (!ctx->h_T || ctx->h_T_n != tn) {
         if (ctx->h_T) cudaFreeHost(ctx->h_T);
         ctx->h_T = nullptr;
@@ -748,7 +749,10 @@ gsnp_status gsnp_get_tables(gsnp_ctx* ctx, uint64_t* counts, double* p_matrix, d
     if ((counts || p_matrix || T) && !ctx->calibrated) return fail(ctx, GSNP_E_STATE, "not calibrated");
     if (counts) memcpy(counts, ctx->h_counts.data(), ctx->h_counts.size() * 8);
     if (p_matrix) memcpy(p_matrix, ctx->h_p.data(), ctx->h_p.size() * 8);
-    if (T) memcpy(T, ctx->h_T, ctx->h_T_n * 8);
+    if (T) {                                        // unpadded [64][L][4][10] view
+        const size_t rows = ctx->h_T_n / TROW;
+        for (size_t r = 0; r < rows; ++r) memcpy(T + r * 10, ctx->h_T + r * TROW, 10 * 8);
+    }
     return GSNP_OK;
 }
 

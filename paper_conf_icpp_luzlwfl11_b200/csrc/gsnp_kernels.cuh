@@ -44,7 +44,7 @@ struct CallArgs {
     const double* known_lp;           // n_known x 10 log10 priors (host-built)
     uint64_t n_known;
     const double* LP;                 // [5][10] log10 novel priors per reference code (R6)
-    const double* T;                  // [64][L][4][10] score table (Alg. 3)
+    const double* T;                  // [64][L][4][TROW] score table (Alg. 3), rows padded
     const uint8_t* adj;               // [64][adjP][adjG] adjust table (R3)
     int adjP, adjG;
     int L, q_max;
@@ -368,6 +368,10 @@ __global__ void k_tile_ranges(const uint64_t* pos, uint64_t n, uint64_t w0, uint
 // parallelisation).  Shared-memory layout (host: call_smem_bytes()).
 constexpr int TS = NT;
 constexpr int COLS = 32;              // key slots per site, shallow kernel (thread path n <= 32)
+#ifndef GSNP_GB
+#define GSNP_GB 4
+#endif
+constexpr int GB = GSNP_GB;           // reads whose bytes are in flight together in the gather
 constexpr int COLS_DEEP = 128;        // key slots per site, deep kernel (thread path n <= 128)
 
 struct TileSmem {
@@ -413,20 +417,39 @@ __device__ __forceinline__ double2 ld_na(const double2* p) {
     asm volatile("ld.global.nc.L1::no_allocate.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
     return v;
 }
-// Score-table row of Alg. 3: 10 consecutive doubles at ((qa*L + coord)*4 + base)*10.
+// Score-table row of Alg. 3: the 10 values of (qa, coord, base), stored padded to
+// TROW = 12 doubles (96 bytes, 32-byte aligned: exactly three sectors) at
+// ((qa*L + coord)*4 + base)*TROW and gathered with three 256-bit loads.
+#ifndef GSNP_T256
+#define GSNP_T256 1
+#endif
+constexpr int TROW = GSNP_T256 ? 12 : 10;
+__device__ __forceinline__ void ld256(const double* p, double& a, double& b, double& c, double& d) {
+    asm volatile("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];"
+                 : "=d"(a), "=d"(b), "=d"(c), "=d"(d) : "l"(p));
+}
 __device__ __forceinline__ void add_row(const double* __restrict__ T, int L, uint32_t qa,
                                         uint32_t cyc, uint32_t b, double* acc) {
-    const double2* row =
-        reinterpret_cast<const double2*>(T + ((size_t)(qa * (uint32_t)L + cyc) * 4u + b) * 10u);
-#if GSNP_T_NOALLOC
-    double2 v0 = ld_na(row + 0), v1 = ld_na(row + 1), v2 = ld_na(row + 2), v3 = ld_na(row + 3),
-            v4 = ld_na(row + 4);
+    const double* row = T + ((size_t)(qa * (uint32_t)L + cyc) * 4u + b) * TROW;
+#if GSNP_T256
+    double v0, v1, v2, v3, v4, v5, v6, v7, v8, v9, p0, p1;
+    ld256(row, v0, v1, v2, v3);
+    ld256(row + 4, v4, v5, v6, v7);
+    ld256(row + 8, v8, v9, p0, p1);
+    acc[0] += v0; acc[1] += v1; acc[2] += v2; acc[3] += v3; acc[4] += v4;
+    acc[5] += v5; acc[6] += v6; acc[7] += v7; acc[8] += v8; acc[9] += v9;
 #else
-    double2 v0 = __ldg(row + 0), v1 = __ldg(row + 1), v2 = __ldg(row + 2), v3 = __ldg(row + 3),
-            v4 = __ldg(row + 4);
+    const double2* r2 = reinterpret_cast<const double2*>(row);
+#if GSNP_T_NOALLOC
+    double2 v0 = ld_na(r2 + 0), v1 = ld_na(r2 + 1), v2 = ld_na(r2 + 2), v3 = ld_na(r2 + 3),
+            v4 = ld_na(r2 + 4);
+#else
+    double2 v0 = __ldg(r2 + 0), v1 = __ldg(r2 + 1), v2 = __ldg(r2 + 2), v3 = __ldg(r2 + 3),
+            v4 = __ldg(r2 + 4);
 #endif
     acc[0] += v0.x; acc[1] += v0.y; acc[2] += v1.x; acc[3] += v1.y; acc[4] += v2.x;
     acc[5] += v2.y; acc[6] += v3.x; acc[7] += v3.y; acc[8] += v4.x; acc[9] += v4.y;
+#endif
 }
 
 // adjust(score, dep_count) through the host-built table (R3): adj[q][min(pcr,P)-1][min(g,G-1)]
@@ -1285,17 +1308,23 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
     uint32_t* colp = sm.col + tid;                           // this lane's column
     __syncthreads();
     const uint64_t n_groups = (A.w1 - A.w0 + 31) / 32;
-    // persistent warps: each takes the next group of 32 consecutive sites from a counter
+    // persistent warps: each takes the next group of 32 consecutive sites from a counter; the
+    // next group's index and read range are fetched while the current one is processed
+    uint64_t nxt = 0, nra = 0, nrb = 0;
+    if (lane == 0) nxt = atomicAdd(work, 1u);
+    nxt = __shfl_sync(FULL, nxt, 0);
+    if (nxt < n_groups) { nra = A.tile_ra[nxt]; nrb = A.tile_rb[nxt]; }
     for (;;) {
-    uint64_t grp = 0;
-    if (lane == 0) grp = atomicAdd(work, 1u);
-    grp = __shfl_sync(FULL, grp, 0);
+    const uint64_t grp = nxt;
     if (grp >= n_groups) break;
+    const uint64_t wra = nra;
+    uint64_t wrb = nrb;
+    if (lane == 0) nxt = atomicAdd(work, 1u);
+    nxt = __shfl_sync(FULL, nxt, 0);
+    if (nxt < n_groups) { nra = A.tile_ra[nxt]; nrb = A.tile_rb[nxt]; }
     const uint64_t g0 = A.w0 + grp * 32;                     // first site of the group
     const uint64_t site = g0 + lane;
     const bool active = site < A.w1;
-    const uint64_t wra = A.tile_ra[grp];
-    uint64_t wrb = A.tile_rb[grp];
 
     // ---- counting + base_word gather, one site per lane.  The warp
     // walks the reads covering its 32 sites: metadata of 32 reads is loaded coalesced and
@@ -1339,11 +1368,11 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
         }
         const int nr = (int)min((uint64_t)32, wrb - r0);
         uint32_t cpack = 0;                                    // 4 x 8-bit base counts this batch
-        for (int k0 = 0; k0 < nr; k0 += 4) {
-            int pk[4];
-            uint32_t ii[4], mk[4], bb[4], qq[4];
+        for (int k0 = 0; k0 < nr; k0 += GB) {
+            int pk[GB];
+            uint32_t ii[GB], mk[GB], bb[GB], qq[GB];
 #pragma unroll
-            for (int u = 0; u < 4; ++u) {
+            for (int u = 0; u < GB; ++u) {
                 const int k = (k0 + u) & 31;
                 pk[u] = __shfl_sync(FULL, pr, k);
                 const uint32_t ok = __shfl_sync(FULL, o, k);
@@ -1356,7 +1385,7 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
                 if (!cov) mk[u] = 0;                           // len 0: not covered below
             }
 #pragma unroll
-            for (int u = 0; u < 4; ++u) {
+            for (int u = 0; u < GB; ++u) {
                 const uint32_t b = bb[u], q = qq[u];
                 const uint32_t lk = mk[u] & 511u, sk = (mk[u] >> 9) & 1u, hk = mk[u] >> 10;
                 const bool cov = lk != 0;

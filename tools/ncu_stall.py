@@ -5,7 +5,8 @@ import sys
 
 rep, col = sys.argv[1], sys.argv[2]
 top = int(sys.argv[3]) if len(sys.argv) > 3 else 30
-out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
+KF = ["--kernel-name", "regex:" + sys.argv[4]] if len(sys.argv) > 4 else []
+out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"] + KF,
                      capture_output=True, text=True).stdout.splitlines()
 rows = list(csv.reader(out))
 hdr = None
