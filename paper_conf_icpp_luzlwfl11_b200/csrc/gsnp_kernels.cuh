@@ -320,25 +320,31 @@ __global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
         }
         if (c < L) {
             const unsigned char* sb = stage + (size_t)sidx * stage_bytes;
-            const unsigned char* bq = direct ? A.R.bases + st_base[sidx] : sb;
-            const unsigned char* qq = direct ? A.R.quals + st_base[sidx] : sb + A.SB;
-            const unsigned char* rr = direct ? A.ref : sb + 2 * A.SB - st_rs[sidx];
             const uint64_t* md = m_desc[sidx];
             const uint16_t* ml = m_ls[sidx];
+            // two instantiations: the staged loop's pointers are provably shared (LDS, not
+            // generic loads through a pointer that might be global)
+            auto count_batch = [&](const unsigned char* bq, const unsigned char* qq,
+                                   const unsigned char* rr) {
 #pragma unroll 4
-            for (uint32_t j = grp; j < nr; j += A.G) {
-                const uint64_t d = md[j];
-                const uint32_t ls = ml[j], l = ls & 511u;
-                if ((uint32_t)c >= l) continue;
-                const uint32_t i = (ls >> 9) ? l - 1 - c : (uint32_t)c;    // read position of cycle c
-                const uint32_t bi = (uint32_t)(d >> 32) + i;
-                const uint32_t o = bq[bi], q = qq[bi];
-                const uint32_t rt = rr[(uint32_t)d + i];                    // code | known << 3
-                err |= (o > 4 ? ERR_RANGE : 0) | (q > (uint32_t)A.q_max ? ERR_QUAL : 0);
-                if (rt >= 4 || o >= 4 || q > (uint32_t)A.q_max) continue;   // N, known SNP, bad
-                if (rt == o) h[(q * 4 + rt) * L + c] += 1;
-                else atomicAdd(&A.C[q << 12 | (uint32_t)c << 4 | rt << 2 | o], 1ull);
-            }
+                for (uint32_t j = grp; j < nr; j += A.G) {
+                    const uint64_t d = md[j];
+                    const uint32_t ls = ml[j], l = ls & 511u;
+                    if ((uint32_t)c >= l) continue;
+                    const uint32_t i = (ls >> 9) ? l - 1 - c : (uint32_t)c;    // read position of cycle c
+                    const uint32_t bi = (uint32_t)(d >> 32) + i;
+                    const uint32_t o = bq[bi], q = qq[bi];
+                    const uint32_t rt = rr[(uint32_t)d + i];                    // code | known << 3
+                    err |= (o > 4 ? ERR_RANGE : 0) | (q > (uint32_t)A.q_max ? ERR_QUAL : 0);
+                    if (rt >= 4 || o >= 4 || q > (uint32_t)A.q_max) continue;   // N, known SNP, bad
+                    if (rt == o) h[(q * 4 + rt) * L + c] += 1;
+                    else atomicAdd(&A.C[q << 12 | (uint32_t)c << 4 | rt << 2 | o], 1ull);
+                }
+            };
+            if (direct)
+                count_batch(A.R.bases + st_base[sidx], A.R.quals + st_base[sidx], A.ref);
+            else
+                count_batch(sb, sb + A.SB, sb + 2 * A.SB - st_rs[sidx]);
         }
         __syncthreads();                               // stage k fully consumed
         if (tid == 0) m_n[sidx] = 0;
