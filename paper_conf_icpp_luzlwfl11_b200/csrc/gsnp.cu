@@ -450,9 +450,10 @@ gsnp_status count_impl(gsnp_ctx* ctx, const gsnp_reads* reads) {
         A.CB = std::max(1, std::min<int>(CAL_MAXB, (int)(A.SB - 32) / A.L));
         A.C = ctx->d_counts.p;
         A.err = ctx->d_err.p;
-        const size_t hist = (size_t)(A.q_max + 1) * 4 * A.L * 2, stages = 2 * (2 * (size_t)A.SB + A.RB);
+        const size_t hist = (size_t)(A.q_max + 1) * 4 * A.L * sizeof(calcell_t), stages = 2 * (2 * (size_t)A.SB + A.RB);
         A.G = CAL_GMAX;                                // as many histogram copies as fit
         while (A.G > 1 && (align16(A.G * hist) + stages > 200 * 1024 || A.G * A.CT > 1024)) A.G >>= 1;
+        A.CB = std::min(A.CB, A.CT * A.G);             // one descriptor per thread
         const size_t smem = align16(A.G * hist) + stages;
         const int per_sm = 1;
         unsigned grid = (unsigned)std::min<uint64_t>((uint64_t)g_num_sms * per_sm, (d.n + A.CB - 1) / A.CB);

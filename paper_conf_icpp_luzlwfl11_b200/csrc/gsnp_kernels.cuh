@@ -197,17 +197,28 @@ struct CalibArgs {
 
 constexpr int CAL_MAXB = 512;         // max reads per batch (metadata arrays)
 
-constexpr int CAL_GMAX = 4;           // thread groups per CTA (A.G), one histogram copy each
+#ifndef GSNP_CAL_U8
+#define GSNP_CAL_U8 1
+#endif
+// Histogram cells: u8 (a full cell hands 255 to the global count) lets 8 groups of 128 threads
+// share one SM's shared memory; u16 cells are flushed before they could overflow.
+#if GSNP_CAL_U8
+typedef uint8_t calcell_t;
+constexpr int CAL_GMAX = 8;           // thread groups per CTA (A.G), one histogram copy each
+#else
+typedef uint16_t calcell_t;
+constexpr int CAL_GMAX = 4;
+#endif
 
 // Add the G histogram copies of cycle c into the global counts and clear them (threads of
 // group 0; the caller synchronises before and after).
-__device__ __forceinline__ void calib_flush(const CalibArgs& A, uint16_t* h, int nbins, int c) {
+__device__ __forceinline__ void calib_flush(const CalibArgs& A, calcell_t* h, int nbins, int c) {
     if (c >= A.L || threadIdx.x >= (unsigned)A.CT) return;
     const size_t copy = (size_t)nbins * A.L;
     for (int k = 0; k < nbins; ++k) {                 // k = q*4 + t
         uint32_t v = 0;
         for (int g = 0; g < A.G; ++g) {
-            uint16_t* cell = h + g * copy + (size_t)k * A.L + c;
+            calcell_t* cell = h + g * copy + (size_t)k * A.L + c;
             v += *cell;
             *cell = 0;
         }
@@ -222,7 +233,7 @@ __global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ uint64_t m_desc[2][CAL_MAXB];          // counted reads: rs | stage offset << 32
     __shared__ uint16_t m_ls[2][CAL_MAXB];            // len | strand << 9
-    __shared__ uint32_t m_n[2];                       // counted reads per stage
+    __shared__ uint32_t m_n[3];                       // counted reads of batch k: m_n[k % 3]
     __shared__ __align__(8) uint64_t bar[2];
     __shared__ uint64_t st_base[2];                   // global byte index of each stage's start
     __shared__ uint32_t st_rs[2];                     // reference index of each ref window's start
@@ -231,9 +242,9 @@ __global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
     const int tid = threadIdx.x;
     const int grp = tid / A.CT, c = tid % A.CT;       // group grp counts reads grp, grp+G, ...
     const int L = A.L;
-    uint16_t* h0 = reinterpret_cast<uint16_t*>(smem);
-    uint16_t* h = h0 + (size_t)grp * nbins * L;       // this group's histogram copy
-    unsigned char* stage = smem + align16((size_t)A.G * nbins * L * 2);
+    calcell_t* h0 = reinterpret_cast<calcell_t*>(smem);
+    calcell_t* h = h0 + (size_t)grp * nbins * L;      // this group's histogram copy
+    unsigned char* stage = smem + align16((size_t)A.G * nbins * L * sizeof(calcell_t));
     const size_t stage_bytes = 2 * (size_t)A.SB + A.RB;
     for (int i = tid; i < A.G * nbins * L; i += blockDim.x) h0[i] = 0;
     const uint64_t per = (A.R.n + gridDim.x - 1) / gridDim.x;
@@ -266,48 +277,53 @@ __global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
         tma_g2s(sb + 2 * A.SB, A.ref + r0, rbytes, &bar[sidx]);
     };
     // all threads: compact the counted reads of batch k (unique, inside the reference)
-    auto stage_meta = [&](uint64_t k) {
-        const int sidx = (int)(k & 1);
-        const uint64_t b0 = ra + k * A.CB, b1 = min(rb, b0 + A.CB);
-        for (uint64_t r0 = b0; r0 < b1; r0 += blockDim.x) {
-            const uint64_t r = r0 + tid;
-            bool keep = false;
-            uint64_t d = 0;
-            uint16_t ls = 0;
-            if (r < b1 && A.R.hits[r] == 1) {
-                const uint64_t p = A.R.pos[r];
-                const uint32_t l = A.R.len[r];
-                keep = p >= A.origin && p + l <= A.origin + A.n_sites && l >= 1 && l <= (uint32_t)L;
-                d = (uint64_t)(uint32_t)(p - A.origin) |
-                    (uint64_t)(uint32_t)(A.R.off[r] - A.R.off0 - st_base[sidx]) << 32;
-                ls = (uint16_t)(l | (uint32_t)A.R.strand[r] << 9);
-            }
-            const uint32_t bal = __ballot_sync(FULL, keep);
-            uint32_t base = 0;
-            if ((tid & 31) == 0 && bal) base = atomicAdd(&m_n[sidx], (uint32_t)__popc(bal));
-            base = __shfl_sync(FULL, base, 0);
-            if (keep) {
-                const uint32_t j = base + __popc(bal & lanemask_lt());
-                m_desc[sidx][j] = d;
-                m_ls[sidx][j] = ls;
-            }
+    // Descriptor of read b0 + tid of batch k (CB <= blockDim), loaded into registers one batch
+    // ahead so its global latency overlaps the count of the batch before.
+    struct Meta { uint64_t p, o, base; uint32_t l, st, hit; bool in; };
+    auto meta_load = [&](uint64_t k) {
+        Meta m;
+        const uint64_t b0 = ra + k * A.CB, b1 = min(rb, b0 + A.CB), r = b0 + tid;
+        m.in = tid < A.CB && r < b1;
+        m.base = (A.R.off[b0] - A.R.off0) & ~15ull;   // = st_base of batch k (see issue)
+        m.p = 0; m.o = 0; m.l = 0; m.st = 0; m.hit = 0;
+        if (m.in) {
+            m.p = A.R.pos[r]; m.o = A.R.off[r]; m.l = A.R.len[r];
+            m.st = A.R.strand[r]; m.hit = A.R.hits[r];
+        }
+        return m;
+    };
+    // Compact the counted reads of a batch into m_desc/m_ls[sidx], count in m_n[cidx].
+    auto meta_commit = [&](const Meta& m, int sidx, int cidx) {
+        const bool keep = m.in && m.hit == 1 && m.p >= A.origin && m.p + m.l <= A.origin + A.n_sites &&
+                          m.l >= 1 && m.l <= (uint32_t)L;
+        const uint32_t bal = __ballot_sync(FULL, keep);
+        uint32_t base = 0;
+        if ((tid & 31) == 0 && bal) base = atomicAdd(&m_n[cidx], (uint32_t)__popc(bal));
+        base = __shfl_sync(FULL, base, 0);
+        if (keep) {
+            const uint32_t j = base + __popc(bal & lanemask_lt());
+            m_desc[sidx][j] = (uint64_t)(uint32_t)(m.p - A.origin) |
+                              (uint64_t)(uint32_t)(m.o - A.R.off0 - m.base) << 32;
+            m_ls[sidx][j] = (uint16_t)(m.l | m.st << 9);
         }
     };
-    if (tid == 0) { m_n[0] = 0; m_n[1] = 0; }
+    if (tid == 0) { m_n[0] = 0; m_n[1] = 0; m_n[2] = 0; }
     __syncthreads();
     if (tid == issuer && nbatch > 0) issue(0);
-    __syncthreads();
-    if (nbatch > 0) stage_meta(0);
+    Meta nxt{};
+    if (nbatch > 0) meta_commit(meta_load(0), 0, 0);
+    if (nbatch > 1) nxt = meta_load(1);
     int err = 0;
     uint32_t since_flush = 0;
     uint32_t phase0 = 0, phase1 = 0;                   // mbarrier parity per stage (TMA'd uses)
     for (uint64_t k = 0; k < nbatch; ++k) {
         const int sidx = (int)(k & 1);
-        __syncthreads();                               // metadata of stage k complete
+        __syncthreads();                               // metadata of batch k complete
         if (tid == issuer && k + 1 < nbatch) issue(k + 1);
-        const uint32_t nr = m_n[sidx];
+        const uint32_t nr = m_n[k % 3];
+        if (tid == 0) m_n[(k + 2) % 3] = 0;           // last read for batch k-1, before the barrier
         const uint32_t per_grp = (nr + A.G - 1) / A.G;
-        if (since_flush + per_grp > 65535u) {          // u16 cells could overflow: flush
+        if (!GSNP_CAL_U8 && since_flush + per_grp > 65535u) {   // u16 cells could overflow: flush
             calib_flush(A, h0, nbins, c + grp * A.CT);
             since_flush = 0;
             __syncthreads();
@@ -337,8 +353,18 @@ __global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
                     const uint32_t rt = rr[(uint32_t)d + i];                    // code | known << 3
                     err |= (o > 4 ? ERR_RANGE : 0) | (q > (uint32_t)A.q_max ? ERR_QUAL : 0);
                     if (rt >= 4 || o >= 4 || q > (uint32_t)A.q_max) continue;   // N, known SNP, bad
-                    if (rt == o) h[(q * 4 + rt) * L + c] += 1;
-                    else atomicAdd(&A.C[q << 12 | (uint32_t)c << 4 | rt << 2 | o], 1ull);
+                    if (rt == o) {
+                        calcell_t* cell = h + (q * 4 + rt) * L + c;
+                        const uint32_t v = *cell + 1u;
+                        if (GSNP_CAL_U8 && v == 255u) {        // full u8 cell
+                            atomicAdd(&A.C[q << 12 | (uint32_t)c << 4 | rt << 2 | rt], 255ull);
+                            *cell = 0;
+                        } else {
+                            *cell = (calcell_t)v;
+                        }
+                    } else {
+                        atomicAdd(&A.C[q << 12 | (uint32_t)c << 4 | rt << 2 | o], 1ull);
+                    }
                 }
             };
             if (direct)
@@ -346,10 +372,13 @@ __global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
             else
                 count_batch(sb, sb + A.SB, sb + 2 * A.SB - st_rs[sidx]);
         }
-        __syncthreads();                               // stage k fully consumed
-        if (tid == 0) m_n[sidx] = 0;
-        __syncthreads();
-        if (k + 1 < nbatch) stage_meta(k + 1);         // metadata for the next stage
+        if (k + 1 < nbatch) {
+            // batch k+1's buffers were last read by batch k-1 (before this iteration's barrier)
+            // and its counter m_n[(k+1)%3] was reset during batch k-1
+            const Meta m = nxt;
+            if (k + 2 < nbatch) nxt = meta_load(k + 2);
+            meta_commit(m, sidx ^ 1, (int)((k + 1) % 3));
+        }
     }
     if (err) atomicOr(A.err, err);
     __syncthreads();
