@@ -20,6 +20,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "oracle.c")
+_SRC_C = os.path.join(_HERE, "compress.c")          # output compression (§V-B, reading R12)
 _LIB = os.path.join(_HERE, "liboracle.so")
 
 GA1 = (0, 0, 0, 0, 1, 1, 1, 2, 2, 3)
@@ -28,9 +29,10 @@ GENOTYPES = ("AA", "AC", "AT", "AG", "CC", "CT", "CG", "TT", "TG", "GG")
 
 
 def build(force: bool = False) -> str:
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+    if force or not os.path.exists(_LIB) or any(os.path.getmtime(_LIB) < os.path.getmtime(s)
+                                                  for s in (_SRC, _SRC_C)):
         subprocess.check_call(["gcc", "-O2", "-fPIC", "-shared", "-ffp-contract=off",
-                               "-o", _LIB, _SRC, "-lm"])
+                               "-o", _LIB, _SRC, _SRC_C, "-lm"])
     return _LIB
 
 
@@ -102,6 +104,10 @@ def lib():
         L.or_call_window.argtypes = [PP, P, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64, P, P,
                                      P, ctypes.POINTER(_Reads), ctypes.c_uint64, ctypes.c_uint64,
                                      P, P, P, P, P, P]
+        L.oc_compress.restype = ctypes.c_uint64
+        L.oc_compress.argtypes = [P, ctypes.c_uint64, ctypes.c_uint32, P, ctypes.c_uint64]
+        L.oc_decompress.restype = ctypes.c_int64
+        L.oc_decompress.argtypes = [P, ctypes.c_uint64, P, ctypes.c_uint64]
         L.or_sizeof_record.restype = ctypes.c_int
         assert L.or_sizeof_record() == RECORD_DTYPE.itemsize
         _lib_cache = L
@@ -219,3 +225,24 @@ def call_window(P: Params, w: dict, p: np.ndarray, w0: int, w1: int, debug: bool
         dbg["keys"] = dbg["keys"][: dbg["off"][-1]]
         return rec, dbg
     return rec
+
+
+def compress(rec: np.ndarray, block_sites: int) -> np.ndarray:
+    """RLE-DICT column compression of records (§V-B, format R12 in compress.c).
+    Returns the stream as uint32 words."""
+    rec = np.ascontiguousarray(rec, RECORD_DTYPE)
+    need = lib().oc_compress(_p(rec), len(rec), block_sites, None, 0)
+    out = np.zeros(max(int(need), 1), np.uint32)
+    got = lib().oc_compress(_p(rec), len(rec), block_sites, _p(out), len(out))
+    assert got == need
+    return out[:need]
+
+
+def decompress(words: np.ndarray, n_max: int) -> np.ndarray:
+    """Inverse of compress(); raises ValueError on a malformed stream."""
+    words = np.ascontiguousarray(words, np.uint32)
+    rec = np.zeros(max(n_max, 1), RECORD_DTYPE)
+    n = lib().oc_decompress(_p(words), len(words), _p(rec), n_max)
+    if n < 0:
+        raise ValueError("malformed compressed stream")
+    return rec[:n]
