@@ -52,7 +52,8 @@ typedef int32_t gsnp_status;
 #define GSNP_STAGE_CALL 3         /* k_call_tile (a4..a8) */
 #define GSNP_STAGE_FINALIZE 4     /* host tables + upload (a2), wall time on the host */
 #define GSNP_STAGE_BIG 5          /* k_big_sites (sites with > 1024 unique keys) */
-#define GSNP_N_STAGES 6
+#define GSNP_STAGE_COMPRESS 6     /* k_cz_* (output compression, §V-B) */
+#define GSNP_N_STAGES 7
 
 typedef struct gsnp_ctx gsnp_ctx;  /* opaque; owned by the library until gsnp_destroy */
 
@@ -158,6 +159,28 @@ gsnp_status gsnp_debug_window(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w
  * dims (may be NULL) receives {L, adj_pcr, adj_g}. */
 gsnp_status gsnp_get_tables(gsnp_ctx* ctx, uint64_t* counts, double* p_matrix, double* T,
                             uint8_t* adj, uint32_t* dims);
+
+/* Output compression (§V-B): compress records rec[0 .. n) into a stream of uint32
+ * words, in blocks of block_sites consecutive records (1 .. 2^24; the paper compresses per window,
+ * P:L749).  The byte format is reading R17 of DESIGN.md: per block a header (magic "GSC1", n,
+ * pos of the first record, block words, block_sites), 2-bit planes of ref/base1/base2 + runs of
+ * N, exception lists for genotype/known/rank_p/post1, the sparse
+ * second-allele columns, and the six quality columns quality, avgq1, cnt_uni1,
+ * cnt_all1, depth, copy_num as RLE with both run arrays DICT-encoded.  Records are
+ * expected in ascending pos order with pos[i+1] = pos[i] + 1 inside a block (what gsnp_call
+ * writes); pos is not stored beyond the block's first record.
+ *   rec: host or device memory (device: used in place).  out: host or device memory.
+ *   out_cap: capacity in words.  *n_words: words of the stream (also on GSNP_E_CAPACITY, when
+ *   out_cap is too small; nothing is written then).  out may be NULL with out_cap 0 to query.
+ * Every step runs in the library's kernels (k_cz_*); the host only sums two sizes. */
+gsnp_status gsnp_compress(gsnp_ctx* ctx, const gsnp_record* rec, uint64_t n, uint32_t block_sites,
+                          uint32_t* out, uint64_t out_cap, uint64_t* n_words);
+
+/* gsnp_call followed by gsnp_compress of the window's records without the records leaving the
+ * device (a8 -> §V-B fused at the library level): the result is the compressed stream only. */
+gsnp_status gsnp_call_compressed(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1,
+                                 uint32_t block_sites, uint32_t* out, uint64_t out_cap,
+                                 uint64_t* n_words);
 
 /* Number of kernel launches this context has issued so far (for bench accounting). */
 uint64_t gsnp_launch_count(const gsnp_ctx* ctx);

@@ -20,7 +20,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "oracle.c")
-_SRC_C = os.path.join(_HERE, "compress.c")          # output compression (§V-B, reading R12)
+_SRC_C = os.path.join(_HERE, "compress.c")          # output compression (§V-B, reading R17)
 _LIB = os.path.join(_HERE, "liboracle.so")
 
 GA1 = (0, 0, 0, 0, 1, 1, 1, 2, 2, 3)
@@ -228,7 +228,7 @@ def call_window(P: Params, w: dict, p: np.ndarray, w0: int, w1: int, debug: bool
 
 
 def compress(rec: np.ndarray, block_sites: int) -> np.ndarray:
-    """RLE-DICT column compression of records (§V-B, format R12 in compress.c).
+    """RLE-DICT column compression of records (§V-B, format R17 in compress.c).
     Returns the stream as uint32 words."""
     rec = np.ascontiguousarray(rec, RECORD_DTYPE)
     need = lib().oc_compress(_p(rec), len(rec), block_sites, None, 0)

@@ -3,7 +3,7 @@
  * TEST INFRASTRUCTURE ONLY (same rules as oracle.c: tests/, smoke() and bench.py only; shares
  * no code with libgsnp).
  *
- * The paper describes the scheme in prose; the byte format below is the reading R12 of
+ * The paper describes the scheme in prose; the byte format below is the reading R17 of
  * DESIGN.md, one section per column family the paper names:
  *   - "sequence name and the number of sites"    -> block header (pos0, n)
  *   - "three columns containing four base types, two bits"     -> planes P (+ N runs)

@@ -7,7 +7,8 @@ import subprocess
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 SRC = os.path.join(HERE, "csrc", "gsnp.cu")
-DEPS = [SRC, os.path.join(HERE, "csrc", "gsnp_kernels.cuh"), os.path.join(ROOT, "include", "gsnp.h")]
+DEPS = [SRC, os.path.join(HERE, "csrc", "gsnp_kernels.cuh"),
+        os.path.join(HERE, "csrc", "gsnp_compress.cuh"), os.path.join(ROOT, "include", "gsnp.h")]
 LIB = os.path.join(HERE, "libgsnp.so")
 
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",

@@ -18,6 +18,7 @@
 
 #include "gsnp.h"
 #include "gsnp_kernels.cuh"
+#include "gsnp_compress.cuh"
 
 using namespace gsnp_dev;
 
@@ -84,6 +85,12 @@ struct gsnp_ctx {
     // debug
     DevBuf<uint32_t> dbg_u32a, dbg_u32b, dbg_u32c, dbg_u32d, dbg_u32e;
     DevBuf<double> dbg_f64a, dbg_f64b;
+    // output compression scratch (§V-B)
+    DevBuf<uint8_t> cz_cols;
+    DevBuf<uint32_t> cz_meta, cz_dD, cz_dict, cz_out;
+    DevBuf<uint64_t> cz_off;
+    DevBuf<gsnp_record> cz_rec;
+    uint64_t* h_cz_total = nullptr;     // pinned
     uint64_t launches = 0;
     // per-stage timing (GSNP_TIMING)
     struct Pending { int stage; cudaEvent_t a, b; };
@@ -510,6 +517,71 @@ gsnp_status finalize_impl(gsnp_ctx* ctx, const uint64_t* counts_host) {
     return GSNP_OK;
 }
 
+// §V-B output compression of device records d_rec[0, n) (format R17, kernels k_cz_*)
+gsnp_status compress_impl(gsnp_ctx* ctx, const gsnp_record* d_rec, uint64_t n, uint32_t B,
+                          uint32_t* out, uint64_t out_cap, uint64_t* n_words) {
+    using namespace gsnp_cz;
+    cudaStream_t s = ctx->stream;
+    const uint64_t nblk = (n + B - 1) / B;
+    if (nblk * NSEC > 0x7FFFFFFFull) return fail(ctx, GSNP_E_RANGE, "too many compression blocks");
+    const uint32_t DC = std::min<uint32_t>(DICT_MAX, B);
+    CK(ctx->cz_cols.ensure(32 * n));
+    CK(ctx->cz_meta.ensure(nblk * NSEC * 2));
+    CK(ctx->cz_dD.ensure(nblk * NDICT));
+    CK(ctx->cz_dict.ensure(nblk * NDICT * DC));
+    CK(ctx->cz_off.ensure(nblk * NSEC + 1));
+    if (!ctx->h_cz_total) CK(cudaMallocHost(&ctx->h_cz_total, 8));
+    CzArgs A;
+    memset(&A, 0, sizeof A);
+    A.rec = d_rec;
+    A.n = n;
+    A.B = B;
+    A.nblk = (uint32_t)nblk;
+    A.DC = DC;
+    uint8_t* base = ctx->cz_cols.p;                  // u32 columns, then u16, then u8
+    for (int k = 0; k < 4; ++k) A.col.u32[k] = reinterpret_cast<uint32_t*>(base + (size_t)4 * n * k);
+    for (int k = 0; k < 4; ++k) A.col.u16[k] = reinterpret_cast<uint16_t*>(base + 16 * n + (size_t)2 * n * k);
+    for (int k = 0; k < 8; ++k) A.col.u8[k] = base + 24 * n + (size_t)n * k;
+    A.meta = ctx->cz_meta.p;
+    A.dD = ctx->cz_dD.p;
+    A.dict = ctx->cz_dict.p;
+    A.off = ctx->cz_off.p;
+    const size_t sm_size = SMEM_SIZE_WORDS * 4, sm_write = SMEM_WRITE_WORDS * 4;
+    CK(cudaFuncSetAttribute(k_cz_sections<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_size));
+    CK(cudaFuncSetAttribute(k_cz_sections<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_write));
+    ctx->begin();
+    const unsigned g0 = (unsigned)std::min<uint64_t>((n + 255) / 256, (uint64_t)g_num_sms * 8);
+    k_cz_columns<<<g0, 256, 0, s>>>(d_rec, n, A.col);
+    k_cz_sections<false><<<(unsigned)(nblk * NSEC), gsnp_cz::NT, sm_size, s>>>(A);
+    k_cz_scan<<<1, 1024, 0, s>>>(ctx->cz_meta.p, nblk * NSEC, ctx->cz_off.p);
+    ctx->launches += 3;
+    CK(cudaGetLastError());
+    CK(cudaMemcpyAsync(ctx->h_cz_total, ctx->cz_off.p + nblk * NSEC, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    const uint64_t total = *ctx->h_cz_total;
+    if (n_words) *n_words = total;
+    if (total > out_cap) {
+        ctx->end(GSNP_STAGE_COMPRESS);
+        return fail(ctx, GSNP_E_CAPACITY, "compressed stream needs %llu words, out_cap %llu",
+                    (unsigned long long)total, (unsigned long long)out_cap);
+    }
+    const bool dev_out = is_device_ptr(out);
+    if (dev_out) {
+        A.out = out;
+    } else {
+        CK(ctx->cz_out.ensure(total));
+        A.out = ctx->cz_out.p;
+    }
+    k_cz_sections<true><<<(unsigned)(nblk * NSEC), gsnp_cz::NT, sm_write, s>>>(A);
+    ctx->launches += 1;
+    ctx->end(GSNP_STAGE_COMPRESS);
+    CK(cudaGetLastError());
+    if (!dev_out) CK(cudaMemcpyAsync(out, A.out, total * 4, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    ctx->flush();
+    return GSNP_OK;
+}
+
 }  // namespace
 
 // ============================================================================ public ABI
@@ -681,6 +753,43 @@ gsnp_status gsnp_call(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint6
     return read_err(ctx);
 }
 
+gsnp_status gsnp_compress(gsnp_ctx* ctx, const gsnp_record* rec, uint64_t n, uint32_t block_sites,
+                          uint32_t* out, uint64_t out_cap, uint64_t* n_words) {
+    if (!ctx) return GSNP_E_INVAL;
+    if (n_words) *n_words = 0;
+    if (cudaSetDevice(ctx->prm.device) != cudaSuccess) return fail(ctx, GSNP_E_CUDA, "set device");
+    if (block_sites < 1 || block_sites > (1u << 24)) return fail(ctx, GSNP_E_INVAL, "block_sites");
+    if (n == 0) return GSNP_OK;
+    if (!rec) return fail(ctx, GSNP_E_INVAL, "rec == NULL");
+    if (out_cap && !out) return fail(ctx, GSNP_E_INVAL, "out == NULL");
+    const gsnp_record* d_rec = rec;
+    if (!is_device_ptr(rec)) {
+        CK(ctx->cz_rec.ensure(n));
+        CK(cudaMemcpyAsync(ctx->cz_rec.p, rec, n * sizeof(gsnp_record), cudaMemcpyHostToDevice,
+                           ctx->stream));
+        d_rec = ctx->cz_rec.p;
+    }
+    return compress_impl(ctx, d_rec, n, block_sites, out, out_cap, n_words);
+}
+
+gsnp_status gsnp_call_compressed(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1,
+                                 uint32_t block_sites, uint32_t* out, uint64_t out_cap,
+                                 uint64_t* n_words) {
+    if (!ctx) return GSNP_E_INVAL;
+    if (n_words) *n_words = 0;
+    if (cudaSetDevice(ctx->prm.device) != cudaSuccess) return fail(ctx, GSNP_E_CUDA, "set device");
+    if (block_sites < 1 || block_sites > (1u << 24)) return fail(ctx, GSNP_E_INVAL, "block_sites");
+    if (out_cap && !out) return fail(ctx, GSNP_E_INVAL, "out == NULL");
+    if (w1 < w0) return fail(ctx, GSNP_E_RANGE, "window outside the reference");
+    const uint64_t S = w1 - w0;
+    if (S == 0) return check_window(ctx, reads, w0, w1);
+    CK(ctx->rec.ensure(S));
+    uint64_t nrec = 0;
+    gsnp_status st = gsnp_call(ctx, reads, w0, w1, ctx->rec.p, S, &nrec);
+    if (st) return st;
+    return compress_impl(ctx, ctx->rec.p, S, block_sites, out, out_cap, n_words);
+}
+
 gsnp_status gsnp_debug_window(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1,
                               uint32_t* off, uint32_t* keys_built, uint32_t* keys_sorted,
                               uint32_t* site_counters, double* L10, double* post10,
@@ -799,6 +908,9 @@ void gsnp_destroy(gsnp_ctx* ctx) {
     ctx->r_bases.release(); ctx->r_quals.release(); ctx->r_strand.release();
     ctx->dbg_u32a.release(); ctx->dbg_u32b.release(); ctx->dbg_u32c.release();
     ctx->dbg_u32d.release(); ctx->dbg_u32e.release(); ctx->dbg_f64a.release(); ctx->dbg_f64b.release();
+    ctx->cz_cols.release(); ctx->cz_meta.release(); ctx->cz_dD.release(); ctx->cz_dict.release();
+    ctx->cz_out.release(); ctx->cz_off.release(); ctx->cz_rec.release();
+    if (ctx->h_cz_total) cudaFreeHost(ctx->h_cz_total);
     if (ctx->h_T) cudaFreeHost(ctx->h_T);
     if (ctx->h_cnt_pinned) cudaFreeHost(ctx->h_cnt_pinned);
     for (auto& p : ctx->pending) { cudaEventDestroy(p.a); cudaEventDestroy(p.b); }

@@ -16,13 +16,15 @@ LIB_PATH = os.environ.get("GSNP_LIB") or os.path.join(_HERE, "libgsnp.so")   # G
 GSNP_ABI_VERSION = 1
 GSNP_RANK_SUM = 0x1
 GSNP_TIMING = 0x2
-STAGES = ("validate", "calib_count", "tile_ranges", "call_tile", "finalize", "big_sites")
+STAGES = ("validate", "calib_count", "tile_ranges", "call_tile", "finalize", "big_sites",
+          "compress")
 STATUS = {0: "GSNP_OK", -1: "GSNP_E_INVAL", -2: "GSNP_E_RANGE", -3: "GSNP_E_UNSORTED",
           -4: "GSNP_E_STATE", -5: "GSNP_E_NOMEM", -6: "GSNP_E_CUDA", -7: "GSNP_E_CAPACITY"}
 
 # exported symbols declared in include/gsnp.h
 SYMBOLS = ("gsnp_params_default", "gsnp_create", "gsnp_calibrate", "gsnp_calibrate_count",
            "gsnp_calibrate_finalize", "gsnp_call", "gsnp_debug_window", "gsnp_get_tables",
+           "gsnp_compress", "gsnp_call_compressed",
            "gsnp_launch_count", "gsnp_stage_times", "gsnp_strerror", "gsnp_last_error",
            "gsnp_destroy")
 
@@ -95,6 +97,11 @@ def lib():
         L.gsnp_debug_window.argtypes = [P, ctypes.POINTER(gsnp_reads), u64, u64] + [P] * 7
         L.gsnp_get_tables.restype = S
         L.gsnp_get_tables.argtypes = [P, P, P, P, P, P]
+        L.gsnp_compress.restype = S
+        L.gsnp_compress.argtypes = [P, P, u64, ctypes.c_uint32, P, u64, ctypes.POINTER(u64)]
+        L.gsnp_call_compressed.restype = S
+        L.gsnp_call_compressed.argtypes = [P, ctypes.POINTER(gsnp_reads), u64, u64,
+                                           ctypes.c_uint32, P, u64, ctypes.POINTER(u64)]
         L.gsnp_launch_count.restype = u64
         L.gsnp_launch_count.argtypes = [P]
         L.gsnp_stage_times.restype = S
@@ -237,6 +244,32 @@ class Context:
                self.h)
         return out
 
+    def compress(self, rec, block_sites: int = 65536, out=None):
+        """§V-B compression of records (numpy RECORD_DTYPE array, or a CUDA uint8 tensor of
+        40*n bytes).  out: None (numpy uint32 result, sized by a query call) or a uint32 buffer
+        (numpy or CUDA tensor); returns (out, n_words)."""
+        n = (rec.numel() // 40) if hasattr(rec, "numel") else len(rec)
+        nw = ctypes.c_uint64(0)
+        if out is None:
+            st = lib().gsnp_compress(self.h, _ptr(rec), n, block_sites, None, 0, ctypes.byref(nw))
+            if st not in (0, -7):
+                _check(st, self.h)
+            out = np.zeros(int(nw.value), np.uint32)
+        cap = out.numel() if hasattr(out, "numel") else len(out)
+        _check(lib().gsnp_compress(self.h, _ptr(rec), n, block_sites, _ptr(out), cap,
+                                   ctypes.byref(nw)), self.h)
+        return out[:int(nw.value)], int(nw.value)
+
+    def call_compressed(self, reads, w0: int, w1: int, out, block_sites: int = 65536):
+        """gsnp_call + gsnp_compress with the records kept on the device; out: uint32 buffer
+        (numpy or CUDA tensor).  Returns the number of words written."""
+        r = reads if isinstance(reads, gsnp_reads) else make_reads(reads)
+        cap = out.numel() if hasattr(out, "numel") else len(out)
+        nw = ctypes.c_uint64(0)
+        _check(lib().gsnp_call_compressed(self.h, ctypes.byref(r), w0, w1, block_sites, _ptr(out),
+                                          cap, ctypes.byref(nw)), self.h)
+        return int(nw.value)
+
     def debug_window(self, reads: dict, w0: int, w1: int):
         S = w1 - w0
         nb = int(np.asarray(reads["off"][-1]) - np.asarray(reads["off"][0])) \
@@ -304,6 +337,14 @@ def gsnp_calibrate_finalize(ctx: Context, counts):
 
 def gsnp_call(ctx: Context, reads, w0, w1, out=None):
     return ctx.call(reads, w0, w1, out)
+
+
+def gsnp_compress(ctx: Context, rec, block_sites=65536, out=None):
+    return ctx.compress(rec, block_sites, out)
+
+
+def gsnp_call_compressed(ctx: Context, reads, w0, w1, out, block_sites=65536):
+    return ctx.call_compressed(reads, w0, w1, out, block_sites)
 
 
 def gsnp_debug_window(ctx: Context, reads, w0, w1):

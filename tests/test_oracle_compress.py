@@ -1,5 +1,5 @@
 """Pins for the oracle's output compression (§V-B; byte format = reading
-R12, oracle/compress.c).  What fixes it independently of the encoder: a block whose every word
+R17, oracle/compress.c).  What fixes it independently of the encoder: a block whose every word
 was derived by hand from the format (tests/golden/compress_tiny.txt), exact round trip on
 adversarial tables (decode is a separate code path), and structural identities that follow
 from the definitions of RLE and DICT."""
