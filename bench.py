@@ -339,6 +339,29 @@ def run_gpu(args):
     e2e_val = total_sites / (float(te.item()) / 1e3)
     ok = bool(torch.equal(out_h, out.cpu()))
 
+    # ---- §8(f) NEXT #1, outside the step: RLE-DICT compression (§V-B) of this shard's records,
+    # device to device, blocks of 65536 records.  CUDA events on the library's stream.
+    CZ_B = 65536
+    nw = gsnp.ctypes.c_uint64(0)                       # size query (status CAPACITY expected)
+    gsnp.lib().gsnp_compress(ctx.h, gsnp._ptr(out), S, CZ_B, None, 0, gsnp.ctypes.byref(nw))
+    cz_words = int(nw.value)
+    cz_out = torch.empty(cz_words, dtype=torch.int32, device="cuda")
+    ctx.compress(out, CZ_B, cz_out)
+    ctx.stage_times(reset=True)
+    c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    n_cz = 5
+    c0.record(stream)
+    for _ in range(n_cz):
+        ctx.compress(out, CZ_B, cz_out)
+    c1.record(stream)
+    torch.cuda.synchronize()
+    cz_ms = c0.elapsed_time(c1) / n_cz
+    cz_kernel_ms = ctx.stage_times(reset=True)["compress"][0] / n_cz
+    compress = {"block_sites": CZ_B, "ms": cz_ms, "kernel_ms": cz_kernel_ms,
+                "records_per_s": S / (cz_ms / 1e3), "in_bytes": 40 * S, "out_bytes": 4 * cz_words,
+                "ratio": 40 * S / (4 * cz_words),
+                "note": "device records -> device stream; not part of the step (SURVEY §8(f) #1)"}
+
     if rank != 0:
         if dist is not None:
             dist.destroy_process_group()
@@ -401,6 +424,7 @@ def run_gpu(args):
                 "d2h_bytes_per_step": d2h, "ms_per_step": float(te.item()), "check": ok},
         "gpu_launches": launches,
         "clocks": clk.summary(),
+        "compress": compress,
     }
     print(json.dumps(line), flush=True)
     ctx.close()
