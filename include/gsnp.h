@@ -53,7 +53,8 @@ typedef int32_t gsnp_status;
 #define GSNP_STAGE_FINALIZE 4     /* host tables + upload (a2), wall time on the host */
 #define GSNP_STAGE_BIG 5          /* k_big_sites (sites with > 1024 unique keys) */
 #define GSNP_STAGE_COMPRESS 6     /* k_cz_* (output compression, §V-B) */
-#define GSNP_N_STAGES 7
+#define GSNP_STAGE_WARP 7         /* k_warp_sites (sites with more keys than the thread path) */
+#define GSNP_N_STAGES 8
 
 typedef struct gsnp_ctx gsnp_ctx;  /* opaque; owned by the library until gsnp_destroy */
 

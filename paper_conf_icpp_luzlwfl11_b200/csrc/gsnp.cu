@@ -7,6 +7,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <atomic>
 #include <chrono>
 #include <cmath>
 #include <cstdarg>
@@ -78,6 +79,7 @@ struct gsnp_ctx {
     DevBuf<gsnp_record> rec;
     DevBuf<BigSite> big;
     DevBuf<uint32_t> big_n;
+    DevBuf<uint32_t> wlist;
     // staged host reads
     DevBuf<uint64_t> r_pos, r_off;
     DevBuf<uint16_t> r_len, r_hits;
@@ -251,10 +253,10 @@ void estimate_p_q(const gsnp_params& prm, const uint64_t* C, double* p, int q) {
 // Alg. 3 score-table rows of quality qa: T[qa][c][b][n] = log10(0.5 p[qa][c][a1][b] +
 // 0.5 p[qa][c][a2][b]), the value Alg. 2 returns, built on the CPU (§IV-G).
 // Rows are stored with TROW (>= 10) doubles each; the padding stays zero.
-void build_T_q(int L, const double* p, double* T, int qa) {
+void build_T_q(int L, const double* p, double* T, int qa, int c_lo, int c_hi) {
     static const int A1[10] = {0, 0, 0, 0, 1, 1, 1, 2, 2, 3};
     static const int A2[10] = {0, 1, 2, 3, 1, 2, 3, 2, 3, 3};
-    for (int c = 0; c < L; ++c)
+    for (int c = c_lo; c < c_hi; ++c)
         for (int b = 0; b < 4; ++b)
             for (int n = 0; n < 10; ++n) {
                 int p1 = qa << 12 | c << 4 | A1[n] << 2 | b;
@@ -397,8 +399,9 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
     const size_t smem = call_smem_bytes(A.L, adj_smem ? adj_bytes : 0, cols, nullptr, nullptr);
     const uint32_t big_cap = (uint32_t)std::min<uint64_t>(w1 - w0, 1u << 22);
     CK(ctx->big.ensure(big_cap));
-    CK(ctx->big_n.ensure(2));
-    CK(cudaMemsetAsync(ctx->big_n.p, 0, 8, s));     // [0] big-site count, [1] work counter
+    CK(ctx->wlist.ensure(w1 - w0));                 // sites for k_warp_sites (at most all)
+    CK(ctx->big_n.ensure(3));
+    CK(cudaMemsetAsync(ctx->big_n.p, 0, 12, s));    // [0] big sites, [1] work counter, [2] wlist
     const bool dbg = A.count_only || A.dbg_off || A.dbg_counters || A.dbg_L10 || A.dbg_post10;
     auto kern = dbg ? (deep ? k_call_tile<true, COLS_DEEP> : k_call_tile<true, COLS>)
                     : (deep ? k_call_tile<false, COLS_DEEP> : k_call_tile<false, COLS>);
@@ -408,11 +411,23 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
     const uint64_t want = (uint64_t)g_num_sms * std::max(per_sm, 1);
     const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, n_tiles));
     ctx->begin();
-    kern<<<grid, NT, smem, s>>>(A, ctx->big.p, ctx->big_n.p, big_cap, ctx->big_n.p + 1, adj_smem);
+    kern<<<grid, NT, smem, s>>>(A, ctx->wlist.p, ctx->big_n.p + 2, ctx->big_n.p + 1, adj_smem);
     ctx->end(GSNP_STAGE_CALL);
     ctx->launches++;
     CK(cudaGetLastError());
     if (!A.count_only) {
+        // listed sites (n > 32 keys, or beyond the deep kernel's thread path): warp per site
+        auto wk = deep ? k_warp_sites<COLS_DEEP> : k_warp_sites<COLS>;
+        const size_t wsm = call_smem_bytes(A.L, 0, cols, nullptr, nullptr);
+        CK(cudaFuncSetAttribute(wk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)wsm));
+        int wper = 0;
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&wper, wk, NT, wsm));
+        ctx->begin();
+        wk<<<(unsigned)(g_num_sms * std::max(wper, 1)), NT, wsm, s>>>(A, ctx->wlist.p, ctx->big_n.p + 2,
+                                                                       ctx->big.p, ctx->big_n.p, big_cap);
+        ctx->end(GSNP_STAGE_WARP);
+        ctx->launches++;
+        CK(cudaGetLastError());
         // sites beyond 1024 unique keys: one CTA each, shared buffer of up to ~200 KB
         const uint32_t cap = (uint32_t)((200 * 1024 - (size_t)8 * A.L) / 4);
         const size_t bsm = 4 * (size_t)cap + (size_t)8 * A.L;
@@ -451,23 +466,24 @@ gsnp_status count_impl(gsnp_ctx* ctx, const gsnp_reads* reads) {
         A.n_sites = ctx->n_sites;
         A.L = (int)ctx->prm.max_read_len;
         A.q_max = (int)ctx->prm.q_max;
-        A.CT = (A.L + 1 + 31) / 32 * 32;              // one spare thread issues the copies
-        A.SB = 12 * 1024;                              // bases (and quals) per stage
-        A.RB = 4 * 1024 + 32;                          // reference window per stage
-        A.CB = std::max(1, std::min<int>(CAL_MAXB, (int)(A.SB - 32) / A.L));
         A.C = ctx->d_counts.p;
         A.err = ctx->d_err.p;
-        const size_t hist = (size_t)(A.q_max + 1) * 4 * A.L * sizeof(calcell_t), stages = 2 * (2 * (size_t)A.SB + A.RB);
-        A.G = CAL_GMAX;                                // as many histogram copies as fit
-        while (A.G > 1 && (align16(A.G * hist) + stages > 200 * 1024 || A.G * A.CT > 1024)) A.G >>= 1;
-        A.CB = std::min(A.CB, A.CT * A.G);             // one descriptor per thread
-        const size_t smem = align16(A.G * hist) + stages;
-        const int per_sm = 1;
-        unsigned grid = (unsigned)std::min<uint64_t>((uint64_t)g_num_sms * per_sm, (d.n + A.CB - 1) / A.CB);
+        // shared memory: u32 diagonal histogram [q][t][cycle] + two stages of (bases, quals,
+        // reference window).  Cycles beyond Lh (only for long reads at high q_max) use global REDs.
+        const size_t budget = 200 * 1024;
+        A.RB = 8 * 1024;                               // reference window per stage
+        A.SB = 24 * 1024;                              // bases (and quals) per stage
+        const size_t per_cyc = (size_t)(A.q_max + 1) * 4 * 4;
+        A.Lh = std::min<int>(A.L, (int)((budget - 2 * (2 * 4096 + A.RB) - 16) / per_cyc) & ~3);
+        const size_t hist = align16(per_cyc * ((A.Lh + 3) / 4 * 4));
+        while (A.SB > 4096 && hist + 2 * (2 * (size_t)A.SB + A.RB) + 16 > budget) A.SB -= 4096;
+        A.CB = std::max(1, std::min<int>(CAL_MAXB, (int)(A.SB - 32) / A.L));
+        const size_t smem = hist + 2 * (2 * (size_t)A.SB + A.RB) + 16;
+        unsigned grid = (unsigned)std::min<uint64_t>((uint64_t)g_num_sms, (d.n + A.CB - 1) / A.CB);
         grid = std::max(grid, 1u);
         CK(cudaFuncSetAttribute(k_calib_count, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         ctx->begin();
-        k_calib_count<<<grid, A.CT * A.G, smem, s>>>(A);
+        k_calib_count<<<grid, CAL_NT, smem, s>>>(A);
         ctx->end(GSNP_STAGE_CALIB);
         ctx->launches++;
         CK(cudaGetLastError());
@@ -494,16 +510,27 @@ gsnp_status finalize_impl(gsnp_ctx* ctx, const uint64_t* counts_host) {
     double* p = ctx->h_p.data();
     double* T = ctx->h_T;
     const gsnp_params prm = ctx->prm;
-    auto work = [&](int tid, int nt) {
-        for (int q = tid; q < 64; q += nt) {
+    // two phases over all host threads: p rows per quality, then T rows per (quality, cycle
+    // chunk) — the log10 calls of Alg. 2 dominate (built once on the CPU)
+    const int CCH = 10;                                  // cycles per T work item
+    const int nch = (L + CCH - 1) / CCH;
+    const int nT = qmax * nch;
+    std::atomic<int> next_p{0}, done_p{0}, next_t{0};
+    auto work = [&]() {
+        for (int q; (q = next_p.fetch_add(1)) < 64;) {
             estimate_p_q(prm, C, p, q);
-            if (q >= 1 && q <= qmax) build_T_q(L, p, T, q);
+            done_p.fetch_add(1);
+        }
+        while (done_p.load() < 64) std::this_thread::yield();
+        for (int it; (it = next_t.fetch_add(1)) < nT;) {
+            const int q = 1 + it / nch, c0 = (it % nch) * CCH;
+            build_T_q(L, p, T, q, c0, std::min(L, c0 + CCH));
         }
     };
-    const int nt = (int)std::max(1u, std::min(8u, std::thread::hardware_concurrency()));
+    const int nt = (int)std::max(1u, std::min(32u, std::thread::hardware_concurrency()));
     std::vector<std::thread> th;
-    for (int i = 1; i < nt; ++i) th.emplace_back(work, i, nt);
-    work(0, nt);
+    for (int i = 1; i < nt; ++i) th.emplace_back(work);
+    work();
     for (auto& t : th) t.join();
     CK(ctx->T.ensure(tn));
     CK(cudaMemcpyAsync(ctx->T.p, ctx->h_T, tn * 8, cudaMemcpyHostToDevice, ctx->stream));
@@ -903,7 +930,7 @@ void gsnp_destroy(gsnp_ctx* ctx) {
     ctx->ref.release(); ctx->known_pos.release(); ctx->known_lp.release();
     ctx->adj.release(); ctx->LP.release(); ctx->T.release(); ctx->d_err.release();
     ctx->d_counts.release(); ctx->tile_ra.release(); ctx->tile_rb.release(); ctx->rec.release();
-    ctx->big.release(); ctx->big_n.release();
+    ctx->big.release(); ctx->big_n.release(); ctx->wlist.release();
     ctx->r_pos.release(); ctx->r_off.release(); ctx->r_len.release(); ctx->r_hits.release();
     ctx->r_bases.release(); ctx->r_quals.release(); ctx->r_strand.release();
     ctx->dbg_u32a.release(); ctx->dbg_u32b.release(); ctx->dbg_u32c.release();

@@ -176,18 +176,19 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
 // ------------------------------------------------------------------------------------------
 // a1: calibration histogram C[q][cyc][t][o] (cal_p_matrix).
 // The CTA streams its share of the reads in batches: the batch's bases and qualities (one
-// contiguous byte range) arrive in shared memory by TMA bulk copies, double-buffered and
-// completed on an mbarrier, while the previous batch is counted.  Cycle-major counting: thread
-// c owns sequencing cycle c, so the diagonal cells (t == o, ~98% of bases) accumulate in a
-// shared [q][t][cycle] u16 histogram with plain read-modify-writes (flushed to the global u64
-// counts before any cell can overflow); mismatches go straight to global u64 REDs.
+// contiguous byte range) and the reference window under it arrive in shared memory by TMA bulk
+// copies, double-buffered and completed on an mbarrier, while the previous batch is counted.
+// Warp per read, four consecutive read positions per lane (one 32-bit shared load per array,
+// realigned with a funnel shift).  The diagonal cells (t == o, ~98% of bases) go to a shared
+// [q][t][cycle] u32 histogram with fire-and-forget shared reductions (lanes of a warp hit
+// consecutive cycles: distinct words, distinct banks); mismatches go to global u64 REDs; the
+// histogram is added into the global counts once at the end.
 struct CalibArgs {
     DevReads R;
     const uint8_t* ref;               // code | known << 3, indexed by site - origin (16 B padded)
     uint64_t origin, n_sites;
     int L, q_max;
-    int CT;                           // threads per group (>= L; thread CT-1 issues the copies)
-    int G;                            // groups per CTA (1, 2 or 4), one histogram copy each
+    int Lh;                           // cycles [0, Lh) counted in shared memory (Lh <= L)
     int CB;                           // reads per batch
     uint32_t SB;                      // bytes per stage buffer (bases; quals the same)
     uint32_t RB;                      // bytes per reference-window buffer
@@ -195,41 +196,20 @@ struct CalibArgs {
     int* err;
 };
 
+constexpr int CAL_NT = 1024;
+constexpr int CAL_NW = CAL_NT / 32;
 constexpr int CAL_MAXB = 512;         // max reads per batch (metadata arrays)
 
-#ifndef GSNP_CAL_U8
-#define GSNP_CAL_U8 1
-#endif
-// Histogram cells: u8 (a full cell hands 255 to the global count) lets 8 groups of 128 threads
-// share one SM's shared memory; u16 cells are flushed before they could overflow.
-#if GSNP_CAL_U8
-typedef uint8_t calcell_t;
-constexpr int CAL_GMAX = 8;           // thread groups per CTA (A.G), one histogram copy each
-#else
-typedef uint16_t calcell_t;
-constexpr int CAL_GMAX = 4;
-#endif
-
-// Add the G histogram copies of cycle c into the global counts and clear them (threads of
-// group 0; the caller synchronises before and after).
-__device__ __forceinline__ void calib_flush(const CalibArgs& A, calcell_t* h, int nbins, int c) {
-    if (c >= A.L || threadIdx.x >= (unsigned)A.CT) return;
-    const size_t copy = (size_t)nbins * A.L;
-    for (int k = 0; k < nbins; ++k) {                 // k = q*4 + t
-        uint32_t v = 0;
-        for (int g = 0; g < A.G; ++g) {
-            calcell_t* cell = h + g * copy + (size_t)k * A.L + c;
-            v += *cell;
-            *cell = 0;
-        }
-        if (v) {
-            const uint32_t q = k >> 2, t = k & 3;
-            atomicAdd(&A.C[q << 12 | (uint32_t)c << 4 | t << 2 | t], (unsigned long long)v);
-        }
-    }
+__device__ __forceinline__ void red_shared_add(uint32_t* p, uint32_t v) {
+    asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
+}
+// predicated shared increment (no branch around it)
+__device__ __forceinline__ void red_shared_inc_if(uint32_t saddr, uint32_t pred) {
+    asm volatile("{\n .reg .pred p;\n setp.ne.u32 p, %1, 0;\n @p red.shared.add.u32 [%0], 1;\n}"
+                 ::"r"(saddr), "r"(pred) : "memory");
 }
 
-__global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
+__global__ void __launch_bounds__(CAL_NT, 1) k_calib_count(CalibArgs A) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ uint64_t m_desc[2][CAL_MAXB];          // counted reads: rs | stage offset << 32
     __shared__ uint16_t m_ls[2][CAL_MAXB];            // len | strand << 9
@@ -238,19 +218,24 @@ __global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
     __shared__ uint64_t st_base[2];                   // global byte index of each stage's start
     __shared__ uint32_t st_rs[2];                     // reference index of each ref window's start
     __shared__ int st_direct[2];                      // too wide for the buffers: read global
-    const int nbins = (A.q_max + 1) * 4;
-    const int tid = threadIdx.x;
-    const int grp = tid / A.CT, c = tid % A.CT;       // group grp counts reads grp, grp+G, ...
-    const int L = A.L;
-    calcell_t* h0 = reinterpret_cast<calcell_t*>(smem);
-    calcell_t* h = h0 + (size_t)grp * nbins * L;      // this group's histogram copy
-    unsigned char* stage = smem + align16((size_t)A.G * nbins * L * sizeof(calcell_t));
+    // flat mode (every read of the batch has length Lb and the reads' bytes are contiguous):
+    // per read of the batch, uncompacted: reference offset in the stage window | minus << 31,
+    // or ~0 for a read that is not counted
+    __shared__ uint32_t m_flat[2][CAL_MAXB];
+    __shared__ uint32_t m_fl[2][3];                   // uniform flag, reads in batch, length Lb
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int L = A.L, Lh = A.Lh;
+    const uint32_t qmax = (uint32_t)A.q_max;
+    const int ncell = (A.q_max + 1) * 4 * Lh;
+    uint32_t* hist = reinterpret_cast<uint32_t*>(smem);               // [q*4 + t][cycle]
+    auto hidx = [&](uint32_t qt, uint32_t cyc) { return qt * (uint32_t)Lh + cyc; };
+    unsigned char* stage = smem + align16((size_t)ncell * 4);
     const size_t stage_bytes = 2 * (size_t)A.SB + A.RB;
-    for (int i = tid; i < A.G * nbins * L; i += blockDim.x) h0[i] = 0;
+    for (int i = tid; i < ncell; i += CAL_NT) hist[i] = 0;
     const uint64_t per = (A.R.n + gridDim.x - 1) / gridDim.x;
     const uint64_t ra = min(A.R.n, (uint64_t)blockIdx.x * per), rb = min(A.R.n, ra + per);
     const uint64_t nbatch = (rb - ra + A.CB - 1) / A.CB;
-    const int issuer = A.CT - 1;                      // beyond the last cycle when CT > L
+    const int issuer = CAL_NT - 1;
     if (tid == 0) { mbar_init(&bar[0], 1); mbar_init(&bar[1], 1); }
     __syncthreads();
     // thread `issuer`: bulk copies of batch k's bases, quals and reference window into stage k&1
@@ -276,15 +261,18 @@ __global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
         tma_g2s(sb + A.SB, A.R.quals + a0, bytes, &bar[sidx]);
         tma_g2s(sb + 2 * A.SB, A.ref + r0, rbytes, &bar[sidx]);
     };
-    // all threads: compact the counted reads of batch k (unique, inside the reference)
-    // Descriptor of read b0 + tid of batch k (CB <= blockDim), loaded into registers one batch
-    // ahead so its global latency overlaps the count of the batch before.
-    struct Meta { uint64_t p, o, base; uint32_t l, st, hit; bool in; };
+    // Descriptor of read b0 + tid of batch k, loaded into registers one batch ahead so its
+    // global latency overlaps the count of the batch before.
+    struct Meta { uint64_t p, o, base, ob0, p0; uint32_t l, st, hit, l0, nall; bool in; };
     auto meta_load = [&](uint64_t k) {
         Meta m;
         const uint64_t b0 = ra + k * A.CB, b1 = min(rb, b0 + A.CB), r = b0 + tid;
         m.in = tid < A.CB && r < b1;
-        m.base = (A.R.off[b0] - A.R.off0) & ~15ull;   // = st_base of batch k (see issue)
+        m.ob0 = A.R.off[b0];
+        m.base = (m.ob0 - A.R.off0) & ~15ull;         // = st_base of batch k (see issue)
+        m.p0 = A.R.pos[b0];
+        m.l0 = A.R.len[b0];
+        m.nall = (uint32_t)(b1 - b0);
         m.p = 0; m.o = 0; m.l = 0; m.st = 0; m.hit = 0;
         if (m.in) {
             m.p = A.R.pos[r]; m.o = A.R.off[r]; m.l = A.R.len[r];
@@ -292,7 +280,7 @@ __global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
         }
         return m;
     };
-    // Compact the counted reads of a batch into m_desc/m_ls[sidx], count in m_n[cidx].
+    // Compact the counted reads (unique, inside the reference) of a batch into m_desc/m_ls[sidx].
     auto meta_commit = [&](const Meta& m, int sidx, int cidx) {
         const bool keep = m.in && m.hit == 1 && m.p >= A.origin && m.p + m.l <= A.origin + A.n_sites &&
                           m.l >= 1 && m.l <= (uint32_t)L;
@@ -306,6 +294,21 @@ __global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
                               (uint64_t)(uint32_t)(m.o - A.R.off0 - m.base) << 32;
             m_ls[sidx][j] = (uint16_t)(m.l | m.st << 9);
         }
+        // flat-mode descriptors and the batch's uniformity (all threads take part)
+        const uint64_t r0 = m.p0 >= A.origin ? ((m.p0 - A.origin) & ~15ull) : 0;   // = st_rs
+        if (m.in)
+            m_flat[sidx][tid] = keep ? (uint32_t)(m.p - A.origin - r0) | m.st << 31 : 0xFFFFFFFFu;
+        const bool uni = !m.in || (m.l == m.l0 && m.o - m.ob0 == (uint64_t)tid * m.l0);
+        const int all_uni = __syncthreads_and(uni);
+        if (tid == 0) { m_fl[sidx][0] = all_uni; m_fl[sidx][1] = m.nall; m_fl[sidx][2] = m.l0; }
+    };
+    // one base: o observed, q quality, rt reference code | known << 3, cycle cyc
+    int err = 0;
+    auto count1 = [&](uint32_t o, uint32_t q, uint32_t rt, uint32_t cyc) {
+        err |= (o > 4 ? ERR_RANGE : 0) | (q > qmax ? ERR_QUAL : 0);
+        if (rt >= 4 || o >= 4 || q > qmax) return;                 // N, known SNP, bad
+        if (rt == o && cyc < (uint32_t)Lh) red_shared_add(&hist[hidx(q * 4 + rt, cyc)], 1u);
+        else atomicAdd(&A.C[q << 12 | cyc << 4 | rt << 2 | o], 1ull);
     };
     if (tid == 0) { m_n[0] = 0; m_n[1] = 0; m_n[2] = 0; }
     __syncthreads();
@@ -313,8 +316,6 @@ __global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
     Meta nxt{};
     if (nbatch > 0) meta_commit(meta_load(0), 0, 0);
     if (nbatch > 1) nxt = meta_load(1);
-    int err = 0;
-    uint32_t since_flush = 0;
     uint32_t phase0 = 0, phase1 = 0;                   // mbarrier parity per stage (TMA'd uses)
     for (uint64_t k = 0; k < nbatch; ++k) {
         const int sidx = (int)(k & 1);
@@ -322,55 +323,156 @@ __global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
         if (tid == issuer && k + 1 < nbatch) issue(k + 1);
         const uint32_t nr = m_n[k % 3];
         if (tid == 0) m_n[(k + 2) % 3] = 0;           // last read for batch k-1, before the barrier
-        const uint32_t per_grp = (nr + A.G - 1) / A.G;
-        if (!GSNP_CAL_U8 && since_flush + per_grp > 65535u) {   // u16 cells could overflow: flush
-            calib_flush(A, h0, nbins, c + grp * A.CT);
-            since_flush = 0;
-            __syncthreads();
-        }
-        since_flush += per_grp;
         const bool direct = st_direct[sidx] != 0;
+        const uint64_t* md = m_desc[sidx];
+        const uint16_t* ml = m_ls[sidx];
         if (!direct) {
             mbar_wait(&bar[sidx], sidx ? phase1 : phase0);
             if (sidx) phase1 ^= 1u; else phase0 ^= 1u;
         }
-        if (c < L) {
-            const unsigned char* sb = stage + (size_t)sidx * stage_bytes;
-            const uint64_t* md = m_desc[sidx];
-            const uint16_t* ml = m_ls[sidx];
-            // two instantiations: the staged loop's pointers are provably shared (LDS, not
-            // generic loads through a pointer that might be global)
-            auto count_batch = [&](const unsigned char* bq, const unsigned char* qq,
-                                   const unsigned char* rr) {
-#pragma unroll 4
-                for (uint32_t j = grp; j < nr; j += A.G) {
-                    const uint64_t d = md[j];
-                    const uint32_t ls = ml[j], l = ls & 511u;
-                    if ((uint32_t)c >= l) continue;
-                    const uint32_t i = (ls >> 9) ? l - 1 - c : (uint32_t)c;    // read position of cycle c
-                    const uint32_t bi = (uint32_t)(d >> 32) + i;
-                    const uint32_t o = bq[bi], q = qq[bi];
-                    const uint32_t rt = rr[(uint32_t)d + i];                    // code | known << 3
-                    err |= (o > 4 ? ERR_RANGE : 0) | (q > (uint32_t)A.q_max ? ERR_QUAL : 0);
-                    if (rt >= 4 || o >= 4 || q > (uint32_t)A.q_max) continue;   // N, known SNP, bad
-                    if (rt == o) {
-                        calcell_t* cell = h + (q * 4 + rt) * L + c;
-                        const uint32_t v = *cell + 1u;
-                        if (GSNP_CAL_U8 && v == 255u) {        // full u8 cell
-                            atomicAdd(&A.C[q << 12 | (uint32_t)c << 4 | rt << 2 | rt], 255ull);
-                            *cell = 0;
-                        } else {
-                            *cell = (calcell_t)v;
-                        }
+        const unsigned char* sb = stage + (size_t)sidx * stage_bytes;
+        const unsigned char* rr = sb + 2 * A.SB;
+        if (!direct && m_fl[sidx][0]) {
+            // flat: thread t takes bytes t, t + 1024, ... of the batch (consecutive threads,
+            // consecutive bytes: one read = Lb consecutive bytes; read j = x / Lb exactly by a
+            // multiply-high since x < 2^16 and Lb <= 256)
+            const uint32_t Lb = m_fl[sidx][2], nb = m_fl[sidx][1] * Lb;
+            const uint32_t magic = (uint32_t)(0xFFFFFFFFull / Lb + 1);
+            const uint32_t xb = (uint32_t)((A.R.off[ra + k * A.CB] - A.R.off0) & 15ull);
+            const unsigned char* fb = sb + xb;
+            const uint32_t* mf = m_flat[sidx];
+            bool eb = false, eq = false;
+            uint32_t ebw = 0, eqw = 0;                                 // error bits (fast path)
+            const uint32_t hbase = smem_u32(hist);
+            // one byte of the batch (edge words and words that straddle two reads)
+            auto one = [&](int64_t x) {
+                if (x < 0 || x >= (int64_t)nb) return;
+                const uint32_t j = __umulhi((uint32_t)x, magic), i = (uint32_t)x - j * Lb;
+                const uint32_t fd = mf[j];
+                if (fd == 0xFFFFFFFFu) return;                          // not a counted read
+                const uint32_t o = fb[x], q = fb[A.SB + x], rt = rr[(fd & 0xFFFFu) + i];
+                const uint32_t cyc = (fd >> 31) ? Lb - 1 - i : i;
+                eb |= o > 4;
+                eq |= q > qmax;
+                if (rt >= 4 || o >= 4 || q > qmax) return;               // N, known SNP, bad
+                if (rt == o && cyc < (uint32_t)Lh) red_shared_add(&hist[(q * 4 + rt) * (uint32_t)Lh + cyc], 1u);
+                else atomicAdd(&A.C[q << 12 | cyc << 4 | rt << 2 | o], 1ull);
+            };
+            // thread t: aligned stage words t, t + 1024, ...: four bases, four qualities and the
+            // four reference codes under them, checked byte-parallel in 32-bit registers
+            const uint32_t* sw = reinterpret_cast<const uint32_t*>(sb);
+            const uint32_t w_lo = xb >> 2, w_hi = (xb + nb + 3) >> 2;
+            const uint32_t qlim = (qmax + 1) * 0x01010101u;
+            for (uint32_t w = w_lo + tid; w < w_hi; w += CAL_NT) {
+                const int64_t x0 = (int64_t)(4 * w) - (int64_t)xb;
+                const uint32_t xc = x0 > 0 ? (uint32_t)x0 : 0u;
+                const uint32_t j = __umulhi(xc, magic), i0 = xc - j * Lb;
+                if (x0 < 0 || x0 + 4 > (int64_t)nb || i0 + 4 > Lb) {    // edge / read boundary
+                    for (int u = 0; u < 4; ++u) one(x0 + u);
+                    continue;
+                }
+                const uint32_t fd = mf[j];
+                if (fd == 0xFFFFFFFFu) continue;                        // not a counted read
+                const uint32_t bw = sw[w], qw = sw[(A.SB >> 2) + w];
+                const uint32_t ro = (fd & 0xFFFFu) + i0;
+                const uint32_t* rw2 = reinterpret_cast<const uint32_t*>(rr + (ro & ~3u));
+                const uint32_t rw = __funnelshift_r(rw2[0], rw2[1], (ro & 3u) * 8);
+                // per byte, bit 7: b > 4 / q > qmax (errors), byte non-zero tests
+                const uint32_t H = 0x80808080u, M = 0x7F7F7F7Fu;
+                const uint32_t badb = (((bw | H) - 0x05050505u) | bw) & H;
+                const uint32_t badq = (((qw | H) - qlim) | qw) & H;
+                ebw |= badb;
+                eqw |= badq;
+                const uint32_t xd = (rw ^ bw) | (rw & 0xFCFCFCFCu);      // 0 <=> diagonal, t < 4
+                const uint32_t xu = (rw | bw) & 0xFCFCFCFCu;             // 0 <=> t < 4 and o < 4
+                const uint32_t diag = ~(((xd & M) + M) | xd) & H & ~badq;
+                const uint32_t used = ~(((xu & M) + M) | xu) & H & ~badq;
+                const uint32_t qt = ((qw & 0x3F3F3F3Fu) << 2) | (rw & 0x03030303u);
+                const bool minus = (fd >> 31) != 0;
+                const uint32_t c0 = minus ? Lb - 1 - i0 : i0;
+                if (Lh == L) {
+                    const int dir = minus ? -1 : 1;
+#pragma unroll
+                    for (int u = 0; u < 4; ++u)
+                        red_shared_inc_if(hbase + 4u * (((qt >> (8 * u)) & 255u) * (uint32_t)Lh +
+                                                        (uint32_t)((int)c0 + u * dir)),
+                                          diag & (0x80u << (8 * u)));
+                    uint32_t mis = used & ~diag;                      // ~2% of bases: global
+                    while (mis) {
+                        const int u = (__ffs(mis) - 1) >> 3;
+                        mis &= mis - 1;
+                        const uint32_t cyc = minus ? c0 - u : c0 + u;
+                        atomicAdd(&A.C[((qw >> (8 * u)) & 63u) << 12 | cyc << 4 |
+                                       ((rw >> (8 * u)) & 3u) << 2 | ((bw >> (8 * u)) & 3u)], 1ull);
+                    }
+                } else {
+                    for (int u = 0; u < 4; ++u) one(x0 + u);
+                }
+            }
+            err |= (eb || ebw ? ERR_RANGE : 0) | (eq || eqw ? ERR_QUAL : 0);
+        } else if (!direct) {
+            const uint32_t rs = st_rs[sidx];
+            // staged: lane covers read positions 4*lane .. 4*lane+3 (+128 per pass)
+            for (uint32_t j = warp; j < nr; j += CAL_NW) {
+                const uint64_t d = md[j];
+                const uint32_t ls = ml[j], l = ls & 511u, minus = ls >> 9;
+                const uint32_t bo = (uint32_t)(d >> 32), ro = (uint32_t)d - rs;
+                for (uint32_t i0 = 4 * lane; i0 < l; i0 += 128) {
+                    const uint32_t ob = bo + i0, orf = ro + i0;
+                    const uint32_t* wb = reinterpret_cast<const uint32_t*>(sb + (ob & ~3u));
+                    const uint32_t* wq = reinterpret_cast<const uint32_t*>(sb + A.SB + (ob & ~3u));
+                    const uint32_t* wr = reinterpret_cast<const uint32_t*>(rr + (orf & ~3u));
+                    const uint32_t sh = (ob & 3u) * 8, shr = (orf & 3u) * 8;
+                    const uint32_t bw = __funnelshift_r(wb[0], wb[1], sh);
+                    const uint32_t qw = __funnelshift_r(wq[0], wq[1], sh);
+                    const uint32_t rw = __funnelshift_r(wr[0], wr[1], shr);
+                    // byte-parallel (SIMD-in-register) checks of the four bases
+                    const uint32_t nv = min(l - i0, 4u);                       // valid bytes
+                    const uint32_t vm = nv >= 4 ? 0xFFFFFFFFu : (1u << (8 * nv)) - 1u;
+                    const uint32_t badb = __vcmpgtu4(bw, 0x04040404u) & vm;
+                    const uint32_t badq = __vcmpgtu4(qw, qmax * 0x01010101u) & vm;
+                    err |= (badb ? ERR_RANGE : 0) | (badq ? ERR_QUAL : 0);
+                    const uint32_t ok = __vcmpltu4(rw, 0x04040404u) & __vcmpltu4(bw, 0x04040404u) &
+                                        ~__vcmpgtu4(qw, qmax * 0x01010101u) & vm;
+                    const uint32_t diag = ok & __vcmpeq4(rw, bw);
+                    // byte u: (q << 2 | t), the histogram row (q <= 63: no carry between bytes)
+                    const uint32_t qt = ((qw & 0x3F3F3F3Fu) << 2) | (rw & 0x03030303u);
+                    const int c0 = minus ? (int)(l - 1 - i0) : (int)i0, dir = minus ? -1 : 1;
+                    if (Lh == L) {
+#pragma unroll
+                        for (int u = 0; u < 4; ++u)
+                            if (diag & (1u << (8 * u)))
+                                red_shared_add(&hist[hidx((qt >> (8 * u)) & 255u, c0 + u * dir)], 1u);
                     } else {
-                        atomicAdd(&A.C[q << 12 | (uint32_t)c << 4 | rt << 2 | o], 1ull);
+#pragma unroll
+                        for (int u = 0; u < 4; ++u)
+                            if ((diag & (1u << (8 * u))) && (uint32_t)(c0 + u * dir) < (uint32_t)Lh)
+                                red_shared_add(&hist[hidx((qt >> (8 * u)) & 255u, c0 + u * dir)], 1u);
+                    }
+                    // the rest goes to global REDs: mismatches (~2% of bases) and, when the shared
+                    // histogram stops at Lh < L, the diagonal cells of cycles >= Lh
+                    uint32_t mis = Lh == L ? ok & ~diag : ok;
+                    while (mis) {
+                        const int u = (__ffs(mis) - 1) >> 3;
+                        mis &= ~(0xFFu << (8 * u));
+                        const uint32_t cyc = (uint32_t)(c0 + u * dir);
+                        const uint32_t o = (bw >> (8 * u)) & 255u, rt = (rw >> (8 * u)) & 255u;
+                        if (rt == o && cyc < (uint32_t)Lh) continue;           // counted in shared
+                        count1(o, (qw >> (8 * u)) & 255u, rt, cyc);
                     }
                 }
-            };
-            if (direct)
-                count_batch(A.R.bases + st_base[sidx], A.R.quals + st_base[sidx], A.ref);
-            else
-                count_batch(sb, sb + A.SB, sb + 2 * A.SB - st_rs[sidx]);
+            }
+        } else {
+            // direct: byte loads from global (batch too wide for the stage buffers)
+            const unsigned char* gb = A.R.bases + st_base[sidx];
+            const unsigned char* gq = A.R.quals + st_base[sidx];
+            for (uint32_t j = warp; j < nr; j += CAL_NW) {
+                const uint64_t d = md[j];
+                const uint32_t ls = ml[j], l = ls & 511u, minus = ls >> 9;
+                const uint32_t bo = (uint32_t)(d >> 32);
+                for (uint32_t i = lane; i < l; i += 32)
+                    count1(gb[bo + i], gq[bo + i], A.ref[(uint32_t)d + i], minus ? l - 1 - i : i);
+            }
         }
         if (k + 1 < nbatch) {
             // batch k+1's buffers were last read by batch k-1 (before this iteration's barrier)
@@ -382,7 +484,13 @@ __global__ void __launch_bounds__(1024) k_calib_count(CalibArgs A) {
     }
     if (err) atomicOr(A.err, err);
     __syncthreads();
-    calib_flush(A, h0, nbins, c + grp * A.CT);
+    for (int i = tid; i < ncell; i += CAL_NT) {
+        const uint32_t v = hist[i];
+        if (v) {
+            const uint32_t qt = (uint32_t)(i / Lh), c = (uint32_t)(i % Lh), q = qt >> 2, t = qt & 3;
+            atomicAdd(&A.C[q << 12 | c << 4 | t << 2 | t], (unsigned long long)v);
+        }
+    }
 }
 // ------------------------------------------------------------------------------------------
 // a3: read ranges.  For each group of 32 consecutive sites [s0, s0+32) (one warp of
@@ -404,7 +512,7 @@ __global__ void k_tile_ranges(const uint64_t* pos, uint64_t n, uint64_t w0, uint
 constexpr int TS = NT;
 constexpr int COLS = 32;              // key slots per site, shallow kernel (thread path n <= 32)
 #ifndef GSNP_GB
-#define GSNP_GB 4
+#define GSNP_GB 2
 #endif
 constexpr int GB = GSNP_GB;           // reads whose bytes are in flight together in the gather
 constexpr int COLS_DEEP = 128;        // key slots per site, deep kernel (thread path n <= 128)
@@ -1325,12 +1433,11 @@ struct BigSite {
 // thread-per-site sort + likelihood + posterior + record; its sites with more than 32 keys
 // follow on the warp paths; beyond 1024 keys they go to k_big_sites.
 #ifndef GSNP_CALL_MINB
-#define GSNP_CALL_MINB 2
+#define GSNP_CALL_MINB 3
 #endif
 template <bool DBG, int CC>
 __global__ void __launch_bounds__(NT, GSNP_CALL_MINB)
-k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_t* work,
-            uint32_t adj_smem) {
+k_call_tile(CallArgs A, uint32_t* wlist, uint32_t* wlist_n, uint32_t* work, uint32_t adj_smem) {
     extern __shared__ __align__(16) unsigned char smem[];
     TileSmem sm;
     const size_t adj_bytes = adj_smem ? (size_t)64 * A.adjP * A.adjG : 0;
@@ -1338,8 +1445,6 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     for (size_t i = tid; i < adj_bytes; i += NT) sm.adj[i] = A.adj[i];
     const uint8_t* adj = adj_smem ? sm.adj : A.adj;
-    uint8_t* myslot = sm.slotcnt + warp * 8 * A.L;
-    for (int i = lane; i < 2 * A.L; i += 32) reinterpret_cast<uint32_t*>(myslot)[i] = 0;
     uint32_t* colp = sm.col + tid;                           // this lane's column
     __syncthreads();
     const uint64_t n_groups = (A.w1 - A.w0 + 31) / 32;
@@ -1483,32 +1588,72 @@ k_call_tile(CallArgs A, BigSite* big, uint32_t* big_n, uint32_t big_cap, uint32_
     }
     __syncwarp();
 
-    // ---- this warp's deeper sites: warp paths (n <= 1024) or the k_big_sites list
-    uint32_t ovf = __ballot_sync(FULL, active && n > COLS && !mid);
-    while (ovf) {
-        const int l = __ffs(ovf) - 1;
-        ovf &= ovf - 1;
-        const uint32_t nn = __shfl_sync(FULL, n, l);
-        const uint32_t c0 = __shfl_sync(FULL, ca0, l), c1 = __shfl_sync(FULL, ca1, l);
-        const uint32_t c2 = __shfl_sync(FULL, ca2, l), c3 = __shfl_sync(FULL, ca3, l);
-        const uint32_t rp = __shfl_sync(FULL, rep, l);
-        const uint64_t s = g0 + l;
-        if (nn > 32 * CC) {
-            if (lane == l) {
-                const uint32_t j = atomicAdd(big_n, 1u);
-                if (j < big_cap) big[j] = BigSite{s, nn, c0, c1, c2, c3, rp};
+    // ---- this warp's deeper sites go to the list that k_warp_sites works through (warp paths,
+    // or k_big_sites beyond the warp buffer): their code stays out of this kernel's registers
+    const bool deep = active && n > COLS && !mid;
+    const uint32_t dv = __ballot_sync(FULL, deep);
+    if (dv) {
+        uint32_t base = 0;
+        if (lane == 0) base = atomicAdd(wlist_n, (uint32_t)__popc(dv));
+        base = __shfl_sync(FULL, base, 0);
+        if (deep) wlist[base + __popc(dv & lanemask_lt())] = (uint32_t)(site - A.w0);
+    }
+    }  // persistent loop
+}
+
+// Sites listed by k_call_tile (n > COLS keys, or n > CC / '-' ends out of order on the deep
+// kernel): one warp per site.  The warp recounts the site's all-hits counters over its group's
+// read range, re-gathers the unique keys into its slice of the col region and runs the warp
+// paths (n <= 32*CC) or hands the site to k_big_sites.
+template <int CC>
+__global__ void __launch_bounds__(NT) k_warp_sites(CallArgs A, const uint32_t* wlist,
+                                                   const uint32_t* wlist_n, BigSite* big,
+                                                   uint32_t* big_n, uint32_t big_cap) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    TileSmem sm;
+    call_smem_bytes(A.L, 0, CC, &sm, smem);
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    uint8_t* myslot = sm.slotcnt + warp * 8 * A.L;
+    for (int i = lane; i < 2 * A.L; i += 32) reinterpret_cast<uint32_t*>(myslot)[i] = 0;
+    __syncwarp();
+    const uint32_t count = *wlist_n;
+    for (uint32_t j = blockIdx.x * NW + warp; j < count; j += gridDim.x * NW) {
+        const uint64_t s = A.w0 + wlist[j];
+        const uint64_t grp = (s - A.w0) / 32;
+        const uint64_t ra = A.tile_ra[grp], rb = A.tile_rb[grp];
+        uint32_t c[4] = {0, 0, 0, 0}, rp = 0;
+        for (uint64_t r = ra + lane; r < rb; r += 32) {
+            const uint64_t i = s - A.R.pos[r];                   // huge when the read starts later
+            if (i < A.R.len[r]) {
+                const uint32_t b = A.R.bases[A.R.off[r] - A.R.off0 + i];
+                if (b < 4) {
+#pragma unroll
+                    for (int x = 0; x < 4; ++x) c[x] += b == (uint32_t)x;
+                    rp += A.R.hits[r];
+                }
+            }
+        }
+#pragma unroll
+        for (int d = 16; d > 0; d >>= 1) {
+#pragma unroll
+            for (int x = 0; x < 4; ++x) c[x] += __shfl_xor_sync(FULL, c[x], d);
+            rp += __shfl_xor_sync(FULL, rp, d);
+        }
+        const uint32_t m = warp_gather(A, sm.col, warp, s, ra, rb);
+        if (m > 32u * CC) {
+            if (lane == 0) {
+                const uint32_t k = atomicAdd(big_n, 1u);
+                if (k < big_cap) big[k] = BigSite{s, m, c[0], c[1], c[2], c[3], rp};
                 else atomicOr(A.err, ERR_DEEP);
             }
             continue;
         }
-        const uint32_t m = warp_gather(A, sm.col, warp, s, wra, wrb);
-        if (m <= 64) warp_site<2>(A, sm.col, warp, m, s, c0, c1, c2, c3, rp, myslot);
-        else if (m <= 128) warp_site<4>(A, sm.col, warp, m, s, c0, c1, c2, c3, rp, myslot);
-        else if (m <= 256) warp_site<8>(A, sm.col, warp, m, s, c0, c1, c2, c3, rp, myslot);
-        else warp_deep_site(A, sm.col, warp, m, s, c0, c1, c2, c3, rp, myslot);
+        if (m <= 64) warp_site<2>(A, sm.col, warp, m, s, c[0], c[1], c[2], c[3], rp, myslot);
+        else if (m <= 128) warp_site<4>(A, sm.col, warp, m, s, c[0], c[1], c[2], c[3], rp, myslot);
+        else if (m <= 256) warp_site<8>(A, sm.col, warp, m, s, c[0], c[1], c[2], c[3], rp, myslot);
+        else warp_deep_site(A, sm.col, warp, m, s, c[0], c[1], c[2], c[3], rp, myslot);
         __syncwarp();
     }
-    }  // persistent loop
 }
 
 // Sites with more than 1024 unique keys: one CTA per site (persistent loop over the list),

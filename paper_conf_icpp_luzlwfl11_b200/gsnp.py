@@ -17,7 +17,7 @@ GSNP_ABI_VERSION = 1
 GSNP_RANK_SUM = 0x1
 GSNP_TIMING = 0x2
 STAGES = ("validate", "calib_count", "tile_ranges", "call_tile", "finalize", "big_sites",
-          "compress")
+          "compress", "warp_sites")
 STATUS = {0: "GSNP_OK", -1: "GSNP_E_INVAL", -2: "GSNP_E_RANGE", -3: "GSNP_E_UNSORTED",
           -4: "GSNP_E_STATE", -5: "GSNP_E_NOMEM", -6: "GSNP_E_CUDA", -7: "GSNP_E_CAPACITY"}
 
