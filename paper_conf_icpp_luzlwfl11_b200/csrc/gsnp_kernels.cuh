@@ -512,7 +512,7 @@ __global__ void k_tile_ranges(const uint64_t* pos, uint64_t n, uint64_t w0, uint
 constexpr int TS = NT;
 constexpr int COLS = 32;              // key slots per site, shallow kernel (thread path n <= 32)
 #ifndef GSNP_GB
-#define GSNP_GB 2
+#define GSNP_GB 1
 #endif
 constexpr int GB = GSNP_GB;           // reads whose bytes are in flight together in the gather
 constexpr int COLS_DEEP = 128;        // key slots per site, deep kernel (thread path n <= 128)
@@ -548,7 +548,7 @@ constexpr uint32_t KEY_BSLOT = (3u << 15) | 511u;                               
 #define GSNP_T_NOALLOC 0
 #endif
 #ifndef GSNP_P2_UNROLL
-#define GSNP_P2_UNROLL 2
+#define GSNP_P2_UNROLL 1
 #endif
 constexpr int kP2Unroll = GSNP_P2_UNROLL;      // rows in flight per thread in likelihood pass 2
 #ifndef GSNP_FUSED_PASS

@@ -1,13 +1,17 @@
-// l2_gather_peak.cu — measured ceiling for k_call_tile's dominant access: random 80-byte rows
-// (5 x 16-byte loads) gathered from an L2-resident table of the score-table's size.
-// Prints one JSON line: {"l2_gather_gbs": ..., "rows_per_s": ..., "table_bytes": ...}.
+// l2_gather_peak.cu — measured ceiling for k_call_tile's dominant access: random score-table
+// rows (10 doubles = 80 algorithmic bytes each) gathered from an L2-resident table of the score
+// table's size.  Two layouts are timed and the best is reported:
+//   80 B rows, 5 x LDG.128 (unpadded);  96 B rows padded to 3 sectors, 3 x LDG.256 (the layout
+//   k_call_tile uses, GSNP_T256).  Grids of 2/4/8 CTAs of 256 threads per SM, best of 5 runs.
+// Prints one JSON line: {"l2_gather_gbs": ..., "rows_per_s": ..., ...}; GB/s counts 80 B per row.
 //   nvcc -O3 -gencode arch=compute_100a,code=sm_100a -o tools/l2_gather_peak tools/l2_gather_peak.cu
 #include <cstdio>
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
-__global__ void __launch_bounds__(256) gather(const double2* __restrict__ T, uint32_t rows,
-                                              uint32_t iters, uint32_t seed, double* out) {
+__global__ void __launch_bounds__(256) gather80(const double2* __restrict__ T, uint32_t rows,
+                                                uint32_t iters, uint32_t seed, double* out) {
     uint32_t x = seed ^ (blockIdx.x * 256u + threadIdx.x) * 2654435761u;
     double a0 = 0, a1 = 0, a2 = 0, a3 = 0, a4 = 0, a5 = 0, a6 = 0, a7 = 0, a8 = 0, a9 = 0;
 #pragma unroll 4
@@ -23,37 +27,71 @@ __global__ void __launch_bounds__(256) gather(const double2* __restrict__ T, uin
     if (s == 12345.678) out[0] = s;  // keep the loads alive
 }
 
+__device__ __forceinline__ void ld256(const double* p, double& a, double& b, double& c, double& d) {
+    asm volatile("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];"
+                 : "=d"(a), "=d"(b), "=d"(c), "=d"(d) : "l"(p));
+}
+
+__global__ void __launch_bounds__(256) gather96(const double* __restrict__ T, uint32_t rows,
+                                                uint32_t iters, uint32_t seed, double* out) {
+    uint32_t x = seed ^ (blockIdx.x * 256u + threadIdx.x) * 2654435761u;
+    double a0 = 0, a1 = 0, a2 = 0, a3 = 0, a4 = 0, a5 = 0, a6 = 0, a7 = 0, a8 = 0, a9 = 0;
+#pragma unroll 2
+    for (uint32_t i = 0; i < iters; ++i) {
+        x = x * 1664525u + 1013904223u;
+        const double* r = T + (size_t)(x % rows) * 12;
+        double v0, v1, v2, v3, v4, v5, v6, v7, v8, v9, p0, p1;
+        ld256(r, v0, v1, v2, v3);
+        ld256(r + 4, v4, v5, v6, v7);
+        ld256(r + 8, v8, v9, p0, p1);
+        a0 += v0; a1 += v1; a2 += v2; a3 += v3; a4 += v4;
+        a5 += v5; a6 += v6; a7 += v7; a8 += v8; a9 += v9;
+    }
+    double s = a0 + a1 + a2 + a3 + a4 + a5 + a6 + a7 + a8 + a9;
+    if (s == 12345.678) out[0] = s;
+}
+
 int main(int argc, char** argv) {
-    const uint32_t rows = argc > 1 ? (uint32_t)atoi(argv[1]) : 64 * 100 * 4;   // 2 MB table
+    const uint32_t rows = argc > 1 ? (uint32_t)atoi(argv[1]) : 64 * 100 * 4;   // the T row count
     const uint32_t iters = 4096;
     int sms = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
-    double2* T;
+    double* T;
     double* out;
-    cudaMalloc(&T, (size_t)rows * 80);
-    cudaMemset(T, 0, (size_t)rows * 80);
+    cudaMalloc(&T, (size_t)rows * 96);
+    cudaMemset(T, 0, (size_t)rows * 96);
     cudaMalloc(&out, 8);
     double best = 0;
-    for (int occ = 4; occ <= 8; occ += 4) {
-        const unsigned grid = (unsigned)(sms * occ);
-        gather<<<grid, 256>>>(T, rows, 64, 1, out);
-        cudaEvent_t a, b;
-        cudaEventCreate(&a);
-        cudaEventCreate(&b);
-        for (int rep = 0; rep < 5; ++rep) {
-            cudaEventRecord(a);
-            gather<<<grid, 256>>>(T, rows, iters, 7 + rep, out);
-            cudaEventRecord(b);
-            cudaEventSynchronize(b);
-            float ms = 0;
-            cudaEventElapsedTime(&ms, a, b);
-            const double nrows = (double)grid * 256 * iters;
-            const double gbs = nrows * 80 / (ms * 1e-3) / 1e9;
-            if (gbs > best) best = gbs;
+    const char* best_how = "";
+    cudaEvent_t a, b;
+    cudaEventCreate(&a);
+    cudaEventCreate(&b);
+    for (int layout = 0; layout < 2; ++layout)
+        for (int occ = 2; occ <= 8; occ *= 2) {
+            const unsigned grid = (unsigned)(sms * occ);
+            for (int rep = 0; rep < 6; ++rep) {
+                cudaEventRecord(a);
+                if (layout == 0)
+                    gather80<<<grid, 256>>>(reinterpret_cast<const double2*>(T), rows,
+                                            rep ? iters : 64, 7 + rep, out);
+                else
+                    gather96<<<grid, 256>>>(T, rows, rep ? iters : 64, 7 + rep, out);
+                cudaEventRecord(b);
+                cudaEventSynchronize(b);
+                if (rep == 0) continue;                      // warm-up
+                float ms = 0;
+                cudaEventElapsedTime(&ms, a, b);
+                const double nrows = (double)grid * 256 * iters;
+                const double gbs = nrows * 80 / (ms * 1e-3) / 1e9;
+                if (gbs > best) {
+                    best = gbs;
+                    best_how = layout == 0 ? "80 B rows, 5 x LDG.128" : "96 B padded rows, 3 x LDG.256";
+                }
+            }
         }
-    }
-    printf("{\"l2_gather_gbs\": %.1f, \"rows_per_s\": %.4g, \"row_bytes\": 80, \"table_bytes\": %llu, "
-           "\"how\": \"random 80-byte rows (5 x LDG.128) from an L2-resident table, best of 5 x 2 grids\"}\n",
-           best, best * 1e9 / 80, (unsigned long long)rows * 80);
+    printf("{\"l2_gather_gbs\": %.1f, \"rows_per_s\": %.4g, \"row_bytes\": 80, \"table_rows\": %u, "
+           "\"best\": \"%s\", \"how\": \"random score-table rows from an L2-resident table; 80 B/row "
+           "counted; best of 2 layouts x grids of 2/4/8 CTAs/SM x 5 runs\"}\n",
+           best, best * 1e9 / 80, rows, best_how);
     return 0;
 }
