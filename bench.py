@@ -268,24 +268,30 @@ def run_gpu(args):
     value = total_sites / (ms_step / 1e3)
 
     # ---- e2e: the same step through the public API with pinned host inputs and outputs, the
-    # host->device copy of the reads and the device->host copy of the records inside the timed
+    # host->device copy of the reads and the device->host copy of the result inside the timed
     # region.  Transfers overlap compute: reads go up in chunks on a copy stream while the
-    # calibration counts each chunk that has arrived; records come down per window chunk while
-    # the next chunk is being called.
+    # calibration counts each chunk that has arrived; the result of each window chunk comes down
+    # while the next chunk is being called.  Two results: the 40-byte records (gsnp_call), and the
+    # paper's output form, the RLE-DICT-compressed records (gsnp_call_compressed, §V-B) — the
+    # headline e2e.
     K = 8
+    CZ_B = 65536
     pinned = {k: v.pin_memory() for k, v in host.items()}
     out_h = torch.empty(40 * S, dtype=torch.uint8).pin_memory()
     dev2 = {k: torch.empty_like(v, device="cuda") for k, v in host.items()}
     h2d = sum(v.numel() * v.element_size() for v in pinned.values())
-    d2h = out_h.numel()
     nr_all = int(len(w["pos"]))
     rcut = [nr_all * i // K for i in range(K + 1)]
     ocut = [int(w["off"][r]) for r in rcut]
     wcut = [w0 + S * i // K for i in range(K + 1)]
     copy_stream = torch.cuda.Stream()
     part = torch.zeros_like(counts)
+    zcap = 11 * (S // K + 1) + 4096                 # words per chunk (> raw 10 words/record)
+    zdev = torch.empty(K * zcap, dtype=torch.int32, device="cuda")
+    zh = torch.empty(K * zcap, dtype=torch.int32).pin_memory()
+    znw = [0] * K
 
-    def e2e_step():
+    def e2e_step(compressed):
         evs = []
         with torch.cuda.stream(copy_stream):
             for i in range(K):
@@ -312,36 +318,59 @@ def run_gpu(args):
             all_reduce_(counts.view(torch.int64))
         ctx.calibrate_finalize(counts)
         rd2 = gsnp.make_reads(dev2)
-        for j in range(K):                    # call window chunk j, then ship its records
+        for j in range(K):                    # call window chunk j, then ship its result
             lo, hi = wcut[j], wcut[j + 1]
-            ctx.call_reads(rd2, lo, hi, out[40 * (lo - w0):40 * (hi - w0)])
+            if compressed:
+                znw[j] = ctx.call_compressed(rd2, lo, hi, zdev[j * zcap:(j + 1) * zcap], CZ_B)
+                src, dst = zdev[j * zcap:j * zcap + znw[j]], zh[j * zcap:j * zcap + znw[j]]
+            else:
+                src = out[40 * (lo - w0):40 * (hi - w0)]
+                ctx.call_reads(rd2, lo, hi, src)
+                dst = out_h[40 * (lo - w0):40 * (hi - w0)]
             e = torch.cuda.Event()
             e.record(stream)
             copy_stream.wait_event(e)
             with torch.cuda.stream(copy_stream):
-                out_h[40 * (lo - w0):40 * (hi - w0)].copy_(out[40 * (lo - w0):40 * (hi - w0)],
-                                                           non_blocking=True)
+                dst.copy_(src, non_blocking=True)
         stream.wait_stream(copy_stream)
 
-    for _ in range(max(1, args.warmup // 2)):
-        e2e_step()
-    torch.cuda.synchronize()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    n_e2e = max(2, min(args.steps, 5))
-    e0.record(stream)
-    for _ in range(n_e2e):
-        e2e_step()
-    e1.record(stream)
-    torch.cuda.synchronize()
-    te = torch.tensor([e0.elapsed_time(e1) / n_e2e], dtype=torch.float64, device="cuda")
-    if dist is not None:
-        all_reduce_(te, dist.ReduceOp.MAX)
-    e2e_val = total_sites / (float(te.item()) / 1e3)
-    ok = bool(torch.equal(out_h, out.cpu()))
+    def time_e2e(compressed):
+        for _ in range(max(1, args.warmup // 2)):
+            e2e_step(compressed)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        n_e2e = max(2, min(args.steps, 5))
+        e0.record(stream)
+        for _ in range(n_e2e):
+            e2e_step(compressed)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        te = torch.tensor([e0.elapsed_time(e1) / n_e2e], dtype=torch.float64, device="cuda")
+        if dist is not None:
+            all_reduce_(te, dist.ReduceOp.MAX)
+        return float(te.item())
+
+    te_rec = time_e2e(False)
+    ok_rec = bool(torch.equal(out_h, out.cpu()))
+    te_cz = time_e2e(True)
+    # the shipped streams == the device compressor run on the device-timed step's records
+    ok_cz = True
+    for j in range(K):
+        lo, hi = wcut[j], wcut[j + 1]
+        ref, nw = ctx.compress(out[40 * (lo - w0):40 * (hi - w0)], CZ_B,
+                               torch.empty(zcap, dtype=torch.int32, device="cuda"))
+        ok_cz &= nw == znw[j] and bool(torch.equal(ref.cpu(), zh[j * zcap:j * zcap + nw]))
+    d2h_cz = 4 * sum(znw)
+    e2e = {"value": total_sites / (te_cz / 1e3), "unit": UNIT, "h2d_bytes_per_step": h2d,
+           "d2h_bytes_per_step": d2h_cz, "ms_per_step": te_cz, "check": ok_cz,
+           "result": "RLE-DICT-compressed records (gsnp_call_compressed, §V-B), %d window chunks "
+                     "overlapped with the transfers" % K,
+           "records": {"value": total_sites / (te_rec / 1e3), "ms_per_step": te_rec,
+                       "d2h_bytes_per_step": out_h.numel(), "check": ok_rec,
+                       "result": "40-byte records (gsnp_call)"}}
 
     # ---- §8(f) NEXT #1, outside the step: RLE-DICT compression (§V-B) of this shard's records,
     # device to device, blocks of 65536 records.  CUDA events on the library's stream.
-    CZ_B = 65536
     nw = gsnp.ctypes.c_uint64(0)                       # size query (status CAPACITY expected)
     gsnp.lib().gsnp_compress(ctx.h, gsnp._ptr(out), S, CZ_B, None, 0, gsnp.ctypes.byref(nw))
     cz_words = int(nw.value)
@@ -360,7 +389,8 @@ def run_gpu(args):
     compress = {"block_sites": CZ_B, "ms": cz_ms, "kernel_ms": cz_kernel_ms,
                 "records_per_s": S / (cz_ms / 1e3), "in_bytes": 40 * S, "out_bytes": 4 * cz_words,
                 "ratio": 40 * S / (4 * cz_words),
-                "note": "device records -> device stream; not part of the step (SURVEY §8(f) #1)"}
+                "note": "device records -> device stream, whole shard; not part of the step "
+                        "(SURVEY §8(f) #1)"}
 
     if rank != 0:
         if dist is not None:
@@ -420,8 +450,7 @@ def run_gpu(args):
                                   "frac": hbm_achieved / peak, "alg_bytes_per_launch": alg_bytes}},
         "cpu_baseline": ({"value": cpu_v, "unit": UNIT, "cores": 1, "kind": "oracle",
                           "sample": cpu_desc} if cpu_v else None),
-        "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": h2d,
-                "d2h_bytes_per_step": d2h, "ms_per_step": float(te.item()), "check": ok},
+        "e2e": e2e,
         "gpu_launches": launches,
         "clocks": clk.summary(),
         "compress": compress,
