@@ -290,6 +290,7 @@ def run_gpu(args):
     zdev = torch.empty(K * zcap, dtype=torch.int32, device="cuda")
     zh = torch.empty(K * zcap, dtype=torch.int32).pin_memory()
     znw = [0] * K
+    gofs = [0] * ws                           # global word offset of each rank's compressed output
 
     def e2e_step(compressed):
         evs = []
@@ -332,6 +333,9 @@ def run_gpu(args):
             copy_stream.wait_event(e)
             with torch.cuda.stream(copy_stream):
                 dst.copy_(src, non_blocking=True)
+        if compressed and dist is not None:   # §8(e) collective 2: where each rank's stream goes
+            gofs[:] = shard.gather_output_offsets(
+                dist, sum(znw), "cuda" if backend == "nccl" else "cpu")[0]
         stream.wait_stream(copy_stream)
 
     def time_e2e(compressed):
@@ -368,6 +372,8 @@ def run_gpu(args):
            "records": {"value": total_sites / (te_rec / 1e3), "ms_per_step": te_rec,
                        "d2h_bytes_per_step": out_h.numel(), "check": ok_rec,
                        "result": "40-byte records (gsnp_call)"}}
+    if ws > 1:
+        e2e["rank_offsets_words"] = gofs      # all-gathered per-rank compressed sizes (§8(e))
 
     # ---- §8(f) NEXT #1, outside the step: RLE-DICT compression (§V-B) of this shard's records,
     # device to device, blocks of 65536 records.  CUDA events on the library's stream.

@@ -66,3 +66,26 @@ def take_reads(w: dict, ra: int, rb: int) -> dict:
                hits=w["hits"][ra:rb], off=(np.asarray(w["off"][ra:rb + 1]) - np.uint64(o0)),
                bases=w["bases"][o0:o1], quals=w["quals"][o0:o1])
     return out
+
+
+def output_offsets(sizes) -> list[int]:
+    """Exclusive prefix sum of per-rank output sizes: where each rank's output starts in the
+    whole-genome output (records, or words of its compressed stream)."""
+    out, acc = [], 0
+    for s in sizes:
+        out.append(acc)
+        acc += int(s)
+    return out
+
+
+def gather_output_offsets(dist, n_local: int, device=None) -> tuple[list[int], int]:
+    """SURVEY.md §8(e) collective 2: all-gather every rank's output size (one uint64 each) and
+    return (per-rank start offsets, total).  `dist` is torch.distributed with an initialised
+    group; `device` is where the one-element tensors live (cuda for NCCL, cpu for gloo)."""
+    import torch
+    ws = dist.get_world_size()
+    mine = torch.tensor([int(n_local)], dtype=torch.int64, device=device)
+    allv = torch.empty(ws, dtype=torch.int64, device=device)
+    dist.all_gather_into_tensor(allv, mine)
+    sizes = [int(x) for x in allv.cpu().tolist()]
+    return output_offsets(sizes), sum(sizes)

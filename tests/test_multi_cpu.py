@@ -44,8 +44,11 @@ def _rank_main(rank, world, port, q):
     p = oracle.p_matrix(P, t.numpy().astype(np.uint64).reshape(64, 256, 4, 4))
     ca, cb = shard.call_reads(w["pos"], lo, hi, w["read_len"])
     rec = oracle.call_window(P, shard.take_reads(w, ca, cb), p, lo, hi)
+    # collective 2: per-rank record counts -> global output offsets
+    offs, total = shard.gather_output_offsets(dist, len(rec))
+    assert total == GENOME["n_sites"] and offs[rank] == lo
     out = [None] * world
-    dist.all_gather_object(out, (t.numpy(), rec.tobytes()))
+    dist.all_gather_object(out, (t.numpy(), rec.tobytes(), offs))
     if rank == 0:
         q.put(out)
     dist.destroy_process_group()
@@ -69,10 +72,20 @@ def test_two_rank_shards_equal_single_process():
     C = oracle.calib_counts(P, w)
     p = oracle.p_matrix(P, C)
     rec = oracle.call_window(P, w, p, 0, GENOME["n_sites"])
-    for counts, _ in out:
+    for counts, _, _ in out:
         assert np.array_equal(counts.reshape(64, 256, 4, 4).astype(np.uint64), C)
-    merged = b"".join(r for _, r in out)
-    assert merged == rec.tobytes()
+    # every rank writes its records at its gathered offset of one whole-genome output
+    offs = out[0][2]
+    assert all(o[2] == offs for o in out)
+    merged = bytearray(len(rec.tobytes()))
+    for r, (_, b, _) in enumerate(out):
+        merged[40 * offs[r]:40 * offs[r] + len(b)] = b
+    assert bytes(merged) == rec.tobytes()
+
+
+def test_output_offsets():
+    assert shard.output_offsets([3, 0, 5, 2]) == [0, 3, 3, 8]
+    assert shard.output_offsets([]) == []
 
 
 def test_plan_by_bases_balances_and_covers():
