@@ -398,6 +398,45 @@ def run_gpu(args):
                 "note": "device records -> device stream, whole shard; not part of the step "
                         "(SURVEY §8(f) #1)"}
 
+    # ---- §8(f) NEXT #3, outside the step: the dense ablation (Fig. 5) — SOAPsnp's
+    # Alg. 1 over per-site dense base_occ arrays (gsnp_call_dense) vs the sparse path, same
+    # sub-window of this shard, same records.  CUDA events on the library's stream.
+    dense = None
+    if not args.no_dense:
+        dlo = w0 + min(S // 4, 8_000_000)
+        dhi = min(w1, dlo + (1 << 22))
+        nd = dhi - dlo
+        dout = torch.empty(40 * nd, dtype=torch.uint8, device="cuda")
+        sout = torch.empty(40 * nd, dtype=torch.uint8, device="cuda")
+        DCH = 16384
+
+        def t_dense():
+            ctx.call_dense(rd, dlo, dhi, dout, chunk_sites=DCH)
+
+        def t_sparse():
+            ctx.call_reads(rd, dlo, dhi, sout)
+        res = {}
+        for name, fn in (("dense", t_dense), ("sparse", t_sparse)):
+            fn()
+            torch.cuda.synchronize()
+            ctx.stage_times(reset=True)
+            d0, d1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            d0.record(stream)
+            for _ in range(3):
+                fn()
+            d1.record(stream)
+            torch.cuda.synchronize()
+            res[name] = (d0.elapsed_time(d1) / 3, ctx.stage_times(reset=True))
+        dst = res["dense"][1]
+        dense = {"sites": nd, "window": [dlo, dhi], "chunk_sites": DCH,
+                 "dense_ms": res["dense"][0], "sparse_ms": res["sparse"][0],
+                 "dense_over_sparse": res["dense"][0] / res["sparse"][0],
+                 "dense_stage_ms": {k: round(dst[k][0] / 3, 3) for k in
+                                    ("dense_count", "dense_lik", "dense_recycle")},
+                 "same_records": bool(torch.equal(dout, sout)),
+                 "note": "paper: GPU dense 14-17x slower than GSNP on an M2050 (P:L915-917)"}
+        del dout, sout
+
     if rank != 0:
         if dist is not None:
             dist.destroy_process_group()
@@ -460,6 +499,7 @@ def run_gpu(args):
         "gpu_launches": launches,
         "clocks": clk.summary(),
         "compress": compress,
+        "dense_ablation": dense,
     }
     print(json.dumps(line), flush=True)
     ctx.close()
@@ -483,6 +523,7 @@ def main():
     ap.add_argument("--no-cpu", action="store_true",
                     help="skip the cpu_baseline leg and the live L2-gather microbenchmark")
     ap.add_argument("--ref-budget", type=float, default=15.0)
+    ap.add_argument("--no-dense", action="store_true", help="skip the dense-ablation leg")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)

@@ -44,6 +44,10 @@ typedef int32_t gsnp_status;
 
 #define GSNP_RANK_SUM 0x1u    /* apply the rank-sum test to heterozygous calls (reading R8) */
 #define GSNP_TIMING 0x2u      /* record per-stage device times with CUDA events (see below) */
+/* Prior variants (reading R18; P:L216 names only known-SNP priors): */
+#define GSNP_MONOPLOID 0x4u   /* heterozygous genotypes get prior 0 at every site (known rows too) */
+#define GSNP_TITV 0x8u        /* novel priors weighted for transition:transversion 2:1: the
+                                 transition allele of ref (A<->G, C<->T) x2, transversions x1/2 */
 
 /* stages reported by gsnp_stage_times */
 #define GSNP_STAGE_VALIDATE 0     /* k_validate_reads */
@@ -54,7 +58,10 @@ typedef int32_t gsnp_status;
 #define GSNP_STAGE_BIG 5          /* k_big_sites (sites with > 1024 unique keys) */
 #define GSNP_STAGE_COMPRESS 6     /* k_cz_* (output compression, §V-B) */
 #define GSNP_STAGE_WARP 7         /* k_warp_sites (sites with more keys than the thread path) */
-#define GSNP_N_STAGES 8
+#define GSNP_STAGE_DENSE_COUNT 8    /* k_dense_count (dense ablation, gsnp_call_dense) */
+#define GSNP_STAGE_DENSE_LIK 9      /* k_dense_sites (dense Alg. 1 + posterior + record) */
+#define GSNP_STAGE_DENSE_RECYCLE 10 /* re-zeroing base_occ after each chunk (memset) */
+#define GSNP_N_STAGES 11
 
 typedef struct gsnp_ctx gsnp_ctx;  /* opaque; owned by the library until gsnp_destroy */
 
@@ -116,6 +123,15 @@ typedef struct {              /* 40 bytes: one output row (f
 /* Fill *out with the defaults listed above. */
 gsnp_status gsnp_params_default(gsnp_params* out);
 
+/* Known-SNP priors from allele frequencies (reading R18; the known-SNP file of P:L216 as
+ * SOAPsnp's per-site A/C/T/G frequencies): Hardy-Weinberg genotype frequencies f_a^2 (a/a) and
+ * 2 f_a f_b (a/b) of the row-normalised frequencies, each floored at floor_prior (> 0) so every
+ * prior is positive, as gsnp_priors requires.  freq: n x 4 (A, C, T, G; >= 0, row sum > 0), host;
+ * prior10: n x 10 out, host, genotype order n = 0..9.  A bad row -> GSNP_E_RANGE (rows before it
+ * are written).  Host arithmetic only; no context needed. */
+gsnp_status gsnp_priors_from_freq(const double* freq, uint64_t n, double floor_prior,
+                                  double* prior10);
+
 /* Create a context on params->device: copies the reference and known-SNP list to the device and
  * builds the adjust table (R3) on the host.  priors may be NULL (no known SNPs). */
 gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
@@ -139,6 +155,19 @@ gsnp_status gsnp_calibrate_finalize(gsnp_ctx* ctx, const uint64_t* counts);
  * device memory.  out_cap < w1-w0 -> GSNP_E_CAPACITY with *n_out = w1-w0. */
 gsnp_status gsnp_call(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1,
                       gsnp_record* out, uint64_t out_cap, uint64_t* n_out);
+
+/* the dense ablation (Fig. 5): the same records as
+ * gsnp_call, computed the way SOAPsnp's Alg. 1 does on the GPU: per site a dense
+ * base_occ[4][64][256][2] of 1-byte occurrence counts (131,072 B, index base<<15 | score<<9 |
+ * coord<<1 | strand) is filled (`counting`), walked in full loop-nest order
+ * (`likelihood`: base 0..3, score q_max..0, coord 0..L-1, strand 0..1) and re-zeroed
+ * (`recycle`), chunk_sites sites at a time (the paper's window of sites).  Arguments
+ * as gsnp_call; chunk_sites: a multiple of 32 in [32, 2^20] (device memory chunk_sites x 128 KiB,
+ * owned by the context).  A cell reaching 256 occurrences (more than 255 identical unique bases
+ * at one site: the paper's 1-byte cell) -> GSNP_E_CAPACITY. */
+gsnp_status gsnp_call_dense(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1,
+                            uint32_t chunk_sites, gsnp_record* out, uint64_t out_cap,
+                            uint64_t* n_out);
 
 /* Debug dump of the same pipeline for [w0, w1) into HOST buffers (any may be NULL):
  *   off[S+1]        u32 CSR offsets of each site's unique keys (S = w1-w0)

@@ -40,7 +40,8 @@ class _Params(ctypes.Structure):
     _fields_ = [("max_read_len", ctypes.c_uint32), ("q_max", ctypes.c_uint32),
                 ("het_novel", ctypes.c_double), ("althom_novel", ctypes.c_double),
                 ("global_dep", ctypes.c_double), ("pcr_dep", ctypes.c_double),
-                ("calib_min_count", ctypes.c_uint32), ("rank_sum", ctypes.c_uint32)]
+                ("calib_min_count", ctypes.c_uint32), ("rank_sum", ctypes.c_uint32),
+                ("prior_mode", ctypes.c_uint32)]
 
 
 class _Reads(ctypes.Structure):
@@ -70,10 +71,13 @@ class Params:
     pcr_dep: float = 0.5
     calib_min_count: int = 10
     rank_sum: bool = True
+    monoploid: bool = False      # R18: heterozygous genotypes get prior 0
+    titv: bool = False           # R18: novel transition:transversion 2:1
 
     def c(self) -> _Params:
         return _Params(self.max_read_len, self.q_max, self.het_novel, self.althom_novel,
-                       self.global_dep, self.pcr_dep, self.calib_min_count, int(self.rank_sum))
+                       self.global_dep, self.pcr_dep, self.calib_min_count, int(self.rank_sum),
+                       int(self.monoploid) | 2 * int(self.titv))
 
 
 _lib_cache = None
@@ -104,6 +108,8 @@ def lib():
         L.or_call_window.argtypes = [PP, P, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64, P, P,
                                      P, ctypes.POINTER(_Reads), ctypes.c_uint64, ctypes.c_uint64,
                                      P, P, P, P, P, P]
+        L.or_priors_from_freq.restype = ctypes.c_int
+        L.or_priors_from_freq.argtypes = [P, ctypes.c_uint64, ctypes.c_double, P]
         L.oc_compress.restype = ctypes.c_uint64
         L.oc_compress.argtypes = [P, ctypes.c_uint64, ctypes.c_uint32, P, ctypes.c_uint64]
         L.oc_decompress.restype = ctypes.c_int64
@@ -225,6 +231,15 @@ def call_window(P: Params, w: dict, p: np.ndarray, w0: int, w1: int, debug: bool
         dbg["keys"] = dbg["keys"][: dbg["off"][-1]]
         return rec, dbg
     return rec
+
+
+def priors_from_freq(freq, floor_prior: float = 5e-7) -> np.ndarray:
+    """R18: Hardy-Weinberg known-SNP prior rows (n x 10) from allele frequencies (n x 4)."""
+    f = np.ascontiguousarray(freq, np.float64).reshape(-1, 4)
+    out = np.zeros((len(f), 10), np.float64)
+    if lib().or_priors_from_freq(_p(f), len(f), float(floor_prior), _p(out)) != 0:
+        raise ValueError("allele frequencies must be >= 0 with a positive row sum")
+    return out
 
 
 def compress(rec: np.ndarray, block_sites: int) -> np.ndarray:

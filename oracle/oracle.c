@@ -27,6 +27,7 @@ typedef struct {
     double pcr_dep;          /* R3 PCR dependency coefficient (linear) */
     uint32_t calib_min_count;/* R1 tau */
     uint32_t rank_sum;       /* R8: 1 = apply the rank-sum test to het calls */
+    uint32_t prior_mode;     /* R18: bit 0 monoploid, bit 1 ti/tv 2:1 */
 } or_params;
 
 typedef struct {
@@ -271,16 +272,50 @@ int or_dense_likelihood(const or_params* P, const double* p, uint64_t n, const u
  * C6 — priors ("prior probability for known SNPs"; the novel prior is PAPER SILENT,
  * reading R6).  Returns log10 prior of genotype n at a site with reference base ref.
  */
+/* R18 prior variants (P:L216 names only "prior probability for known
+ * SNPs", so every variant is a reading):
+ *  - ti/tv (prior_mode bit 1): the transition:transversion ratio of novel alleles is 2:1.  Of the
+ *    three alternative alleles of ref, one is the transition (A<->G, C<->T: code XOR 3) and two are
+ *    transversions; per-allele weights with mean 1 and ratio 2:1 overall are w_ti = 2,
+ *    w_tv = 1/2.  ref/x het: het_novel w(x); x/x: althom_novel w(x); x/y: het_novel althom_novel
+ *    w(x) w(y).  No effect at ref N.
+ *  - monoploid (bit 0): heterozygous genotypes have prior 0 (log10 = -inf) at every site,
+ *    known SNP rows included. */
+static double titv_w(const or_params* P, int ref, int x) {
+    if (!(P->prior_mode & 2u)) return 1.0;
+    return (ref ^ x) == 3 ? 2.0 : 0.5;
+}
+
 static double log10_prior(const or_params* P, int ref, int n, const double* known_row) {
+    int a1 = GA1[n], a2 = GA2[n];
+    if ((P->prior_mode & 1u) && a1 != a2) return log10(0.0);   /* -inf */
     if (known_row) return log10(known_row[n]);
     if (ref == 4) return 0.0;
-    int a1 = GA1[n], a2 = GA2[n];
     double pr;
     if (a1 == ref && a2 == ref) pr = 1.0;
-    else if (a1 == ref || a2 == ref) pr = P->het_novel;
-    else if (a1 == a2) pr = P->althom_novel;
-    else pr = P->het_novel * P->althom_novel;
+    else if (a1 == ref) pr = P->het_novel * titv_w(P, ref, a2);
+    else if (a2 == ref) pr = P->het_novel * titv_w(P, ref, a1);
+    else if (a1 == a2) pr = P->althom_novel * titv_w(P, ref, a1);
+    else pr = P->het_novel * P->althom_novel * titv_w(P, ref, a1) * titv_w(P, ref, a2);
     return log10(pr);
+}
+
+/* R18 known-SNP priors from allele frequencies (the known-SNP file of P:L216 as SOAPsnp's:
+ * per-site frequencies of A, C, T, G): Hardy-Weinberg genotype frequencies, f_a^2 for a/a and
+ * 2 f_a f_b for a/b (frequencies normalised to sum 1), each floored at floor_prior > 0 so every
+ * prior stays positive.  freq: n x 4; prior10: n x 10.  Returns -1 if a row sums to <= 0. */
+int or_priors_from_freq(const double* freq, uint64_t n, double floor_prior, double* prior10) {
+    for (uint64_t i = 0; i < n; ++i) {
+        const double* f = freq + 4 * i;
+        double tot = f[0] + f[1] + f[2] + f[3];
+        if (!(tot > 0) || f[0] < 0 || f[1] < 0 || f[2] < 0 || f[3] < 0) return -1;
+        for (int k = 0; k < 10; ++k) {
+            double fa = f[GA1[k]] / tot, fb = f[GA2[k]] / tot;
+            double v = GA1[k] == GA2[k] ? fa * fa : 2.0 * fa * fb;
+            prior10[10 * i + k] = v > floor_prior ? v : floor_prior;
+        }
+    }
+    return 0;
 }
 
 /* C8 — Wilcoxon rank-sum, normal approximation with tie correction (PAPER SILENT, reading R8).

@@ -8,7 +8,8 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 SRC = os.path.join(HERE, "csrc", "gsnp.cu")
 DEPS = [SRC, os.path.join(HERE, "csrc", "gsnp_kernels.cuh"),
-        os.path.join(HERE, "csrc", "gsnp_compress.cuh"), os.path.join(ROOT, "include", "gsnp.h")]
+        os.path.join(HERE, "csrc", "gsnp_compress.cuh"), os.path.join(HERE, "csrc", "gsnp_dense.cuh"),
+        os.path.join(ROOT, "include", "gsnp.h")]
 LIB = os.path.join(HERE, "libgsnp.so")
 
 NVCC_FLAGS = ["-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",

@@ -20,6 +20,7 @@
 #include "gsnp.h"
 #include "gsnp_kernels.cuh"
 #include "gsnp_compress.cuh"
+#include "gsnp_dense.cuh"
 
 using namespace gsnp_dev;
 
@@ -80,6 +81,9 @@ struct gsnp_ctx {
     DevBuf<BigSite> big;
     DevBuf<uint32_t> big_n;
     DevBuf<uint32_t> wlist;
+    // dense ablation (§8(f) NEXT #3): base_occ of one chunk of sites + per-site all-hits counters
+    DevBuf<uint8_t> dense_occ;
+    DevBuf<uint32_t> dense_cnt;
     // staged host reads
     DevBuf<uint64_t> r_pos, r_off;
     DevBuf<uint16_t> r_len, r_hits;
@@ -320,6 +324,8 @@ gsnp_status map_err(gsnp_ctx* ctx, int e) {
     if (e & ERR_UNSORTED) return fail(ctx, GSNP_E_UNSORTED, "read positions decrease");
     if (e & (ERR_RANGE | ERR_QUAL))
         return fail(ctx, GSNP_E_RANGE, "read value out of range (len/base/qual/strand/hits/pos)");
+    if (e & ERR_DENSE_SAT)
+        return fail(ctx, GSNP_E_CAPACITY, "a dense base_occ count exceeds 255 (1-byte cells, P:L390)");
     if (e & ERR_DEEP)
         return fail(ctx, GSNP_E_CAPACITY, "a site's unique depth exceeds the shared-memory key buffer");
     return fail(ctx, GSNP_E_CUDA, "device error flag %d", e);
@@ -339,12 +345,11 @@ gsnp_status launch_validate(gsnp_ctx* ctx, const DevReads& d) {
 
 int g_num_sms = 0;
 
-gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w1,
-                       gsnp_record* d_out, CallArgs& A) {
+// a3: per-32-site-group read ranges of [w0, w1) (k_tile_ranges) and the kernels' arguments
+gsnp_status prep_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w1,
+                        gsnp_record* d_out, CallArgs& A) {
     cudaStream_t s = ctx->stream;
-    const uint64_t n_tiles = (w1 - w0 + TS - 1) / TS;
     const uint64_t n_groups = (w1 - w0 + 31) / 32;
-    if (n_tiles == 0) return GSNP_OK;
     CK(ctx->tile_ra.ensure(n_groups));
     CK(ctx->tile_rb.ensure(n_groups));
     if (d.n) {
@@ -379,6 +384,17 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
     A.tile_rb = ctx->tile_rb.p;
     A.out = d_out;
     A.err = ctx->d_err.p;
+    return GSNP_OK;
+}
+
+gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w1,
+                       gsnp_record* d_out, CallArgs& A) {
+    cudaStream_t s = ctx->stream;
+    const uint64_t n_tiles = (w1 - w0 + TS - 1) / TS;
+    if (n_tiles == 0) return GSNP_OK;
+    gsnp_status st = prep_window(ctx, d, w0, w1, d_out, A);
+    if (st) return st;
+    const uint64_t n_groups = (w1 - w0 + 31) / 32;
     // persistent CTAs; warps pull 32-site groups from a counter.  The adjust table rides in
     // shared memory when small (it is 64 x 7 x 37 bytes at the default coefficients).
     const size_t adj_bytes = (size_t)64 * A.adjP * A.adjG;
@@ -631,6 +647,26 @@ gsnp_status gsnp_params_default(gsnp_params* out) {
     return GSNP_OK;
 }
 
+gsnp_status gsnp_priors_from_freq(const double* freq, uint64_t n, double floor_prior,
+                                  double* prior10) {
+    static const int A1[10] = {0, 0, 0, 0, 1, 1, 1, 2, 2, 3};
+    static const int A2[10] = {0, 1, 2, 3, 1, 2, 3, 2, 3, 3};
+    if (n && (!freq || !prior10)) return GSNP_E_INVAL;
+    if (!(floor_prior > 0)) return GSNP_E_INVAL;
+    for (uint64_t i = 0; i < n; ++i) {
+        const double* f = freq + 4 * i;
+        const double tot = f[0] + f[1] + f[2] + f[3];
+        if (!(tot > 0) || !(f[0] >= 0) || !(f[1] >= 0) || !(f[2] >= 0) || !(f[3] >= 0))
+            return GSNP_E_RANGE;
+        for (int k = 0; k < 10; ++k) {
+            const double fa = f[A1[k]] / tot, fb = f[A2[k]] / tot;
+            const double v = A1[k] == A2[k] ? fa * fa : 2.0 * fa * fb;
+            prior10[10 * i + k] = v > floor_prior ? v : floor_prior;
+        }
+    }
+    return GSNP_OK;
+}
+
 gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
                         const gsnp_params* params, gsnp_ctx** out) {
     if (!out) return GSNP_E_INVAL;
@@ -675,16 +711,25 @@ gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
     double LP[50];
     static const int A1[10] = {0, 0, 0, 0, 1, 1, 1, 2, 2, 3};
     static const int A2[10] = {0, 1, 2, 3, 1, 2, 3, 2, 3, 3};
+    // R18 variants: ti/tv 2:1 weights of the alternative alleles; monoploid zeroes het priors
+    const bool mono = (params->flags & GSNP_MONOPLOID) != 0, titv = (params->flags & GSNP_TITV) != 0;
+    auto wt = [&](int r, int x) { return !titv ? 1.0 : (r ^ x) == 3 ? 2.0 : 0.5; };
     for (int r = 0; r < 5; ++r)
         for (int n = 0; n < 10; ++n) {
             double v;
+            if (mono && A1[n] != A2[n]) { LP[r * 10 + n] = log10(0.0); continue; }
             if (r == 4) { LP[r * 10 + n] = kLog10Zero; continue; }
             if (A1[n] == r && A2[n] == r) v = 1.0;
-            else if (A1[n] == r || A2[n] == r) v = params->het_novel;
-            else if (A1[n] == A2[n]) v = params->althom_novel;
-            else v = params->het_novel * params->althom_novel;
+            else if (A1[n] == r) v = params->het_novel * wt(r, A2[n]);
+            else if (A2[n] == r) v = params->het_novel * wt(r, A1[n]);
+            else if (A1[n] == A2[n]) v = params->althom_novel * wt(r, A1[n]);
+            else v = params->het_novel * params->althom_novel * wt(r, A1[n]) * wt(r, A2[n]);
             LP[r * 10 + n] = log10(v);
         }
+    if (mono)
+        for (uint64_t k = 0; k < nk; ++k)
+            for (int n = 0; n < 10; ++n)
+                if (A1[n] != A2[n]) lp[k * 10 + n] = log10(0.0);
     if ((st = build_adj(ctx))) return bail(st);
     gsnp_ctx* c = ctx;
 #define CKC(x) do { if ((x) != cudaSuccess) { cudaGetLastError(); return bail(fail(c, GSNP_E_CUDA, "%s", #x)); } } while (0)
@@ -778,6 +823,71 @@ gsnp_status gsnp_call(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint6
     if (!dev_out)
         CK(cudaMemcpyAsync(out, d_out, S * sizeof(gsnp_record), cudaMemcpyDeviceToHost, ctx->stream));
     return read_err(ctx);
+}
+
+gsnp_status gsnp_call_dense(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1,
+                            uint32_t chunk_sites, gsnp_record* out, uint64_t out_cap,
+                            uint64_t* n_out) {
+    if (!ctx) return GSNP_E_INVAL;
+    if (cudaSetDevice(ctx->prm.device) != cudaSuccess) return fail(ctx, GSNP_E_CUDA, "set device");
+    gsnp_status st = check_window(ctx, reads, w0, w1);
+    if (st) return st;
+    if (chunk_sites < 32 || chunk_sites % 32 || chunk_sites > (1u << 20))
+        return fail(ctx, GSNP_E_INVAL, "chunk_sites must be a multiple of 32 in [32, 2^20]");
+    const uint64_t S = w1 - w0;
+    if (n_out) *n_out = S;
+    if (out_cap < S) return fail(ctx, GSNP_E_CAPACITY, "out_cap %llu < %llu", (unsigned long long)out_cap,
+                                 (unsigned long long)S);
+    if (S && !out) return fail(ctx, GSNP_E_INVAL, "out == NULL");
+    if (S == 0) return GSNP_OK;
+    cudaStream_t s = ctx->stream;
+    DevReads d;
+    if ((st = stage_reads(ctx, reads, d))) return st;
+    CK(cudaMemsetAsync(ctx->d_err.p, 0, sizeof(int), s));
+    if ((st = launch_validate(ctx, d))) return st;
+    const bool dev_out = is_device_ptr(out);
+    gsnp_record* d_out = out;
+    if (!dev_out) {
+        CK(ctx->rec.ensure(S));
+        d_out = ctx->rec.p;
+    }
+    DenseArgs D;
+    memset(&D, 0, sizeof D);
+    if ((st = prep_window(ctx, d, w0, w1, d_out, D.A))) return st;
+    const uint64_t chunk = std::min<uint64_t>(chunk_sites, S);
+    const bool fresh = ctx->dense_occ.n < chunk * DENSE_SITE_BYTES;
+    CK(ctx->dense_occ.ensure(chunk * DENSE_SITE_BYTES));
+    CK(ctx->dense_cnt.ensure(chunk * 5));
+    if (fresh) CK(cudaMemsetAsync(ctx->dense_occ.p, 0, chunk * DENSE_SITE_BYTES, s));
+    D.occ = ctx->dense_occ.p;
+    D.cnt = ctx->dense_cnt.p;
+    for (uint64_t c0 = w0; c0 < w1; c0 += chunk) {
+        D.c0 = c0;
+        D.c1 = std::min(w1, c0 + chunk);
+        const uint64_t n = D.c1 - D.c0;
+        CK(cudaMemsetAsync(D.cnt, 0, n * 5 * 4, s));
+        if (d.n) {
+            ctx->begin();
+            k_dense_count<<<(unsigned)(g_num_sms * 8), DENSE_NT, 0, s>>>(D);
+            ctx->end(GSNP_STAGE_DENSE_COUNT);
+            ctx->launches++;
+            CK(cudaGetLastError());
+        }
+        ctx->begin();
+        k_dense_sites<<<(unsigned)std::min<uint64_t>((n + 7) / 8, (uint64_t)g_num_sms * 8), DENSE_NT, 0, s>>>(D);
+        ctx->end(GSNP_STAGE_DENSE_LIK);
+        ctx->launches++;
+        CK(cudaGetLastError());
+        ctx->begin();                       // recycle: re-zero the whole dense array
+        CK(cudaMemsetAsync(D.occ, 0, n * DENSE_SITE_BYTES, s));
+        ctx->end(GSNP_STAGE_DENSE_RECYCLE);
+    }
+    if (!dev_out)
+        CK(cudaMemcpyAsync(out, d_out, S * sizeof(gsnp_record), cudaMemcpyDeviceToHost, s));
+    st = read_err(ctx);
+    if (st == GSNP_E_CAPACITY)              // a saturated cell leaves residue behind: start clean
+        cudaMemsetAsync(ctx->dense_occ.p, 0, ctx->dense_occ.n, s);
+    return st;
 }
 
 gsnp_status gsnp_compress(gsnp_ctx* ctx, const gsnp_record* rec, uint64_t n, uint32_t block_sites,
@@ -931,6 +1041,7 @@ void gsnp_destroy(gsnp_ctx* ctx) {
     ctx->adj.release(); ctx->LP.release(); ctx->T.release(); ctx->d_err.release();
     ctx->d_counts.release(); ctx->tile_ra.release(); ctx->tile_rb.release(); ctx->rec.release();
     ctx->big.release(); ctx->big_n.release(); ctx->wlist.release();
+    ctx->dense_occ.release(); ctx->dense_cnt.release();
     ctx->r_pos.release(); ctx->r_off.release(); ctx->r_len.release(); ctx->r_hits.release();
     ctx->r_bases.release(); ctx->r_quals.release(); ctx->r_strand.release();
     ctx->dbg_u32a.release(); ctx->dbg_u32b.release(); ctx->dbg_u32c.release();

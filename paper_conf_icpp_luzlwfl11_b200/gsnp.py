@@ -16,15 +16,17 @@ LIB_PATH = os.environ.get("GSNP_LIB") or os.path.join(_HERE, "libgsnp.so")   # G
 GSNP_ABI_VERSION = 1
 GSNP_RANK_SUM = 0x1
 GSNP_TIMING = 0x2
+GSNP_MONOPLOID = 0x4
+GSNP_TITV = 0x8
 STAGES = ("validate", "calib_count", "tile_ranges", "call_tile", "finalize", "big_sites",
-          "compress", "warp_sites")
+          "compress", "warp_sites", "dense_count", "dense_lik", "dense_recycle")
 STATUS = {0: "GSNP_OK", -1: "GSNP_E_INVAL", -2: "GSNP_E_RANGE", -3: "GSNP_E_UNSORTED",
           -4: "GSNP_E_STATE", -5: "GSNP_E_NOMEM", -6: "GSNP_E_CUDA", -7: "GSNP_E_CAPACITY"}
 
 # exported symbols declared in include/gsnp.h
 SYMBOLS = ("gsnp_params_default", "gsnp_create", "gsnp_calibrate", "gsnp_calibrate_count",
            "gsnp_calibrate_finalize", "gsnp_call", "gsnp_debug_window", "gsnp_get_tables",
-           "gsnp_compress", "gsnp_call_compressed",
+           "gsnp_compress", "gsnp_call_compressed", "gsnp_call_dense", "gsnp_priors_from_freq",
            "gsnp_launch_count", "gsnp_stage_times", "gsnp_strerror", "gsnp_last_error",
            "gsnp_destroy")
 
@@ -102,6 +104,11 @@ def lib():
         L.gsnp_call_compressed.restype = S
         L.gsnp_call_compressed.argtypes = [P, ctypes.POINTER(gsnp_reads), u64, u64,
                                            ctypes.c_uint32, P, u64, ctypes.POINTER(u64)]
+        L.gsnp_call_dense.restype = S
+        L.gsnp_call_dense.argtypes = [P, ctypes.POINTER(gsnp_reads), u64, u64, ctypes.c_uint32,
+                                      P, u64, ctypes.POINTER(u64)]
+        L.gsnp_priors_from_freq.restype = S
+        L.gsnp_priors_from_freq.argtypes = [P, u64, ctypes.c_double, P]
         L.gsnp_launch_count.restype = u64
         L.gsnp_launch_count.argtypes = [P]
         L.gsnp_stage_times.restype = S
@@ -244,6 +251,19 @@ class Context:
                self.h)
         return out
 
+    def call_dense(self, reads, w0: int, w1: int, out=None, chunk_sites: int = 16384):
+        """The dense ablation (gsnp_call_dense): same records as call(),
+        through per-site dense base_occ arrays, chunk_sites sites at a time."""
+        S = w1 - w0
+        if out is None:
+            out = np.zeros(S, RECORD_DTYPE)
+        cap = (out.numel() // 40) if hasattr(out, "numel") else len(out)
+        r = reads if isinstance(reads, gsnp_reads) else make_reads(reads)
+        n = ctypes.c_uint64(0)
+        _check(lib().gsnp_call_dense(self.h, ctypes.byref(r), w0, w1, chunk_sites, _ptr(out), cap,
+                                     ctypes.byref(n)), self.h)
+        return out
+
     def compress(self, rec, block_sites: int = 65536, out=None):
         """§V-B compression of records (numpy RECORD_DTYPE array, or a CUDA uint8 tensor of
         40*n bytes).  out: None (numpy uint32 result, sized by a query call) or a uint32 buffer
@@ -345,6 +365,18 @@ def gsnp_compress(ctx: Context, rec, block_sites=65536, out=None):
 
 def gsnp_call_compressed(ctx: Context, reads, w0, w1, out, block_sites=65536):
     return ctx.call_compressed(reads, w0, w1, out, block_sites)
+
+
+def gsnp_call_dense(ctx: Context, reads, w0, w1, out=None, chunk_sites=16384):
+    return ctx.call_dense(reads, w0, w1, out, chunk_sites)
+
+
+def gsnp_priors_from_freq(freq, floor_prior: float = 5e-7) -> np.ndarray:
+    """Known-SNP prior rows (n x 10) from allele frequencies (n x 4, A C T G), reading R18."""
+    f = np.ascontiguousarray(freq, np.float64).reshape(-1, 4)
+    out = np.zeros((len(f), 10), np.float64)
+    _check(lib().gsnp_priors_from_freq(_ptr(f), len(f), float(floor_prior), _ptr(out)), None)
+    return out
 
 
 def gsnp_debug_window(ctx: Context, reads, w0, w1):

@@ -1,0 +1,70 @@
+"""GPU parity for the prior variants (reading R18): monoploid and
+ti/tv 2:1 novel priors, and known-SNP rows from allele frequencies — CUDA path vs the oracle."""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from paper_conf_icpp_luzlwfl11_b200 import gsnp
+from tests._parity import compare
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.parametrize("mono,titv", [(True, False), (False, True), (True, True)])
+def test_prior_variants_parity(mono, titv):
+    w = synth.generate("C1", n_sites=8_000, depth=12.0, seed=41)
+    P = oracle.Params(monoploid=mono, titv=titv)
+    C = oracle.calib_counts(P, w)
+    p = oracle.p_matrix(P, C)
+    rec_o, dbg = oracle.call_window(P, w, p, 0, 8_000, debug=True)
+    flags = gsnp.GSNP_RANK_SUM | (gsnp.GSNP_MONOPLOID if mono else 0) | (gsnp.GSNP_TITV if titv else 0)
+    with gsnp.Context.from_workload(w, flags=flags) as ctx:
+        ctx.calibrate(w)
+        rec_g = ctx.call(w, 0, 8_000)
+        dg = ctx.debug_window(w, 0, 8_000)
+        rec_d = ctx.call_dense(w, 0, 8_000, chunk_sites=2048)
+    assert rec_g.tobytes() == dg["records"].tobytes() == rec_d.tobytes()
+    # L10 is prior-free: bit-exact; posteriors within 1e-9 relative; every record field equal
+    assert np.array_equal(dg["L10"], dbg["L10"])
+    pg, po = dg["post10"], dbg["post10"]
+    big = np.maximum(np.abs(pg), np.abs(po)) > 1e-300
+    assert np.all(np.abs(pg - po)[big] <= 1e-9 * np.maximum(np.abs(pg), np.abs(po))[big])
+    assert np.all((pg == 0) == (po == 0))
+    srt = np.sort(po, 1)
+    near_tie = srt[:, -1] - srt[:, -2] <= 1e-9 * srt[:, -1]      # listed, not mismatches
+    for f in rec_o.dtype.names:
+        if f in ("rank_p", "post1"):
+            assert np.allclose(rec_g[f][~near_tie], rec_o[f][~near_tie], rtol=1e-6, atol=0), f
+        elif f == "quality":        # exact but for 10Δ+10log10(p) at an integer boundary
+            d = np.abs(rec_g[f].astype(int) - rec_o[f].astype(int))[~near_tie]
+            assert d.max(initial=0) <= 1 and (d > 0).sum() <= 2, f
+        elif f == "genotype":
+            assert np.array_equal(rec_g[f][~near_tie], rec_o[f][~near_tie]), f
+        else:
+            assert np.array_equal(rec_g[f], rec_o[f]), f
+    if mono:
+        assert not np.isin(rec_g["genotype"], [1, 2, 3, 5, 6, 8]).any()
+
+
+def test_priors_from_freq_library_equals_oracle_and_calls():
+    rng = np.random.default_rng(7)
+    f = rng.dirichlet(np.ones(4) * 0.3, 500)
+    f[::7, 1] = 0.0
+    assert np.array_equal(gsnp.gsnp_priors_from_freq(f, 5e-7), oracle.priors_from_freq(f, 5e-7))
+    with pytest.raises(gsnp.GsnpError):
+        gsnp.gsnp_priors_from_freq([[0.0, 0, 0, 0]])
+    # known-SNP rows from frequencies drive the call like any caller-supplied prior10
+    w = synth.generate("C1", n_sites=6_000, depth=10.0, seed=43)
+    kp = np.asarray(w["known_pos"], np.uint64)
+    freq = rng.dirichlet(np.ones(4), len(kp))
+    w = dict(w, known_prior10=gsnp.gsnp_priors_from_freq(freq))
+    P = oracle.Params()
+    p = oracle.p_matrix(P, oracle.calib_counts(P, w))
+    rec_o, dbg = oracle.call_window(P, w, p, 0, 6_000, debug=True)
+    with gsnp.Context.from_workload(w) as ctx:
+        ctx.calibrate(w)
+        rec_g = ctx.call(w, 0, 6_000)
+    compare(w, rec_g, rec_o, dbg["L10"])
