@@ -437,6 +437,43 @@ def run_gpu(args):
                  "note": "paper: GPU dense 14-17x slower than GSNP on an M2050 (P:L915-917)"}
         del dout, sout
 
+    # ---- §8(f) NEXT #2, outside the step: input packing on the GPU — this shard's reads as SOAP
+    # alignment text (resident in HBM), parsed into the gsnp_reads arrays (gsnp_parse_soap).
+    parse = None
+    if not args.no_parse:
+        import synth
+        text = synth.soap_text(w, "chr21", 33)
+        tdev = torch.frombuffer(bytearray(text), dtype=torch.uint8).cuda()
+        del text
+        pout = {k: torch.empty_like(v) for k, v in dev.items()}
+        pout["off"] = torch.empty_like(dev["off"])
+        lb = int(w["origin"])
+        ctx.parse_soap(tdev, "chr21", 33, lb, out=pout)
+        torch.cuda.synchronize()
+        ctx.stage_times(reset=True)
+        p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        n_p = 5
+        p0.record(stream)
+        for _ in range(n_p):
+            got = ctx.parse_soap(tdev, "chr21", 33, lb, out=pout)
+        p1.record(stream)
+        torch.cuda.synchronize()
+        p_ms = p0.elapsed_time(p1) / n_p
+        p_kms = ctx.stage_times(reset=True)["parse"][0] / n_p
+        sv = {torch.uint16: torch.int16, torch.uint64: torch.int64}
+
+        def _sg(t):
+            return t.view(sv.get(t.dtype, t.dtype))
+        off0 = _sg(dev["off"])[0]
+        ok = all(torch.equal(_sg(got[k]), _sg(dev[k]) - off0 if k == "off" else _sg(dev[k]))
+                 for k in got)
+        nbt = int(tdev.numel())
+        parse = {"text_bytes": nbt, "reads": int(len(w["pos"])), "ms": p_ms, "kernel_ms": p_kms,
+                 "text_GB_per_s": nbt / (p_ms / 1e3) / 1e9, "reads_per_s": len(w["pos"]) / (p_ms / 1e3),
+                 "check": bool(ok),
+                 "note": "SOAP text in HBM -> gsnp_reads arrays; not part of the step (SURVEY §8(f) #2)"}
+        del tdev, pout, got
+
     if rank != 0:
         if dist is not None:
             dist.destroy_process_group()
@@ -500,6 +537,7 @@ def run_gpu(args):
         "clocks": clk.summary(),
         "compress": compress,
         "dense_ablation": dense,
+        "parse": parse,
     }
     print(json.dumps(line), flush=True)
     ctx.close()
@@ -524,6 +562,7 @@ def main():
                     help="skip the cpu_baseline leg and the live L2-gather microbenchmark")
     ap.add_argument("--ref-budget", type=float, default=15.0)
     ap.add_argument("--no-dense", action="store_true", help="skip the dense-ablation leg")
+    ap.add_argument("--no-parse", action="store_true", help="skip the SOAP-text parsing leg")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)

@@ -61,7 +61,8 @@ typedef int32_t gsnp_status;
 #define GSNP_STAGE_DENSE_COUNT 8    /* k_dense_count (dense ablation, gsnp_call_dense) */
 #define GSNP_STAGE_DENSE_LIK 9      /* k_dense_sites (dense Alg. 1 + posterior + record) */
 #define GSNP_STAGE_DENSE_RECYCLE 10 /* re-zeroing base_occ after each chunk (memset) */
-#define GSNP_N_STAGES 11
+#define GSNP_STAGE_PARSE 11         /* k_nl_tiles, k_parse_meta, k_sel_*, k_parse_emit (gsnp_parse_soap) */
+#define GSNP_N_STAGES 12
 
 typedef struct gsnp_ctx gsnp_ctx;  /* opaque; owned by the library until gsnp_destroy */
 
@@ -148,6 +149,29 @@ gsnp_status gsnp_calibrate(gsnp_ctx* ctx, const gsnp_reads* reads);
  * score table T (Alg. 3) and the priors on the host and uploads them. */
 gsnp_status gsnp_calibrate_count(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t* counts);
 gsnp_status gsnp_calibrate_finalize(gsnp_ctx* ctx, const uint64_t* counts);
+
+/* input packing on the GPU: SOAP alignment text (input file 1,
+ * P:L206-212, in SOAPsnp's format; reading R19) -> the gsnp_reads arrays.  One
+ * alignment per '\n'-terminated line (the last line may be unterminated; empty lines are
+ * skipped), tab-separated fields
+ *   id  seq  qual  n_hits  a/b  len  strand(+/-)  chr  location(1-based)  [further fields ignored]
+ * seq in reference-forward orientation, ACGTN (either case) -> 0 1 2 3 4; qual characters minus
+ * q_offset (33 or 64), each 0..63; n_hits >= 1 (saturates at 65535); len == |seq| == |qual|,
+ * 1..256.  Lines whose chr differs from chr_name (NULL or "" = any) are skipped; the others, in
+ * input order, become reads with pos = location - 1 + loc_base.
+ *   text: n_bytes bytes, host or device (device text is used in place when 16-byte aligned).
+ *   outputs: reads_cap entries of pos/len/strand/hits, reads_cap+1 of off (off[0] = 0),
+ *   bases_cap of bases/quals; all host or all device (judged by pos).
+ *   *n_reads / *n_bases: the selected reads and their bases — also set on GSNP_E_CAPACITY (caps
+ *   too small; nothing written), so a call with caps 0 and NULL outputs is a size query.
+ * A malformed selected line (missing fields, bad number, |seq| != len, strand not +/-, a base
+ * or quality character out of range) -> GSNP_E_RANGE naming the first bad line.  Sortedness
+ * and the reference range are checked later, by gsnp_calibrate / gsnp_call. */
+gsnp_status gsnp_parse_soap(gsnp_ctx* ctx, const char* text, uint64_t n_bytes, const char* chr_name,
+                            uint32_t q_offset, uint64_t loc_base, uint64_t* pos, uint16_t* len,
+                            uint64_t* off, uint8_t* bases, uint8_t* quals, uint8_t* strand,
+                            uint16_t* hits, uint64_t reads_cap, uint64_t bases_cap,
+                            uint64_t* n_reads, uint64_t* n_bases);
 
 /* Call sites [w0, w1) (global coordinates inside the reference): one gsnp_record per site,
  * written to out[0 .. w1-w0).  reads must include every read overlapping the window (the

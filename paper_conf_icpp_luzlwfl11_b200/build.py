@@ -9,6 +9,7 @@ ROOT = os.path.dirname(HERE)
 SRC = os.path.join(HERE, "csrc", "gsnp.cu")
 DEPS = [SRC, os.path.join(HERE, "csrc", "gsnp_kernels.cuh"),
         os.path.join(HERE, "csrc", "gsnp_compress.cuh"), os.path.join(HERE, "csrc", "gsnp_dense.cuh"),
+        os.path.join(HERE, "csrc", "gsnp_parse.cuh"),
         os.path.join(ROOT, "include", "gsnp.h")]
 LIB = os.path.join(HERE, "libgsnp.so")
 

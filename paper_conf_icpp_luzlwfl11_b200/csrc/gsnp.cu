@@ -21,6 +21,7 @@
 #include "gsnp_kernels.cuh"
 #include "gsnp_compress.cuh"
 #include "gsnp_dense.cuh"
+#include "gsnp_parse.cuh"
 
 using namespace gsnp_dev;
 
@@ -84,6 +85,9 @@ struct gsnp_ctx {
     // dense ablation (§8(f) NEXT #3): base_occ of one chunk of sites + per-site all-hits counters
     DevBuf<uint8_t> dense_occ;
     DevBuf<uint32_t> dense_cnt;
+    // SOAP text parsing (§8(f) NEXT #2)
+    DevBuf<uint8_t> p_text, p_chr;
+    DevBuf<uint64_t> p_cnt, p_ls, p_meta, p_pos, p_ridx, p_boff, p_part, p_scal;
     // staged host reads
     DevBuf<uint64_t> r_pos, r_off;
     DevBuf<uint16_t> r_len, r_hits;
@@ -890,6 +894,153 @@ gsnp_status gsnp_call_dense(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0,
     return st;
 }
 
+gsnp_status gsnp_parse_soap(gsnp_ctx* ctx, const char* text, uint64_t n_bytes, const char* chr_name,
+                            uint32_t q_offset, uint64_t loc_base, uint64_t* pos, uint16_t* len,
+                            uint64_t* off, uint8_t* bases, uint8_t* quals, uint8_t* strand,
+                            uint16_t* hits, uint64_t reads_cap, uint64_t bases_cap,
+                            uint64_t* n_reads, uint64_t* n_bases) {
+    if (!ctx) return GSNP_E_INVAL;
+    if (n_reads) *n_reads = 0;
+    if (n_bases) *n_bases = 0;
+    if (cudaSetDevice(ctx->prm.device) != cudaSuccess) return fail(ctx, GSNP_E_CUDA, "set device");
+    if (n_bytes && !text) return fail(ctx, GSNP_E_INVAL, "text == NULL");
+    if (q_offset > 255) return fail(ctx, GSNP_E_INVAL, "q_offset > 255");
+    const size_t chr_len = chr_name ? strlen(chr_name) : 0;
+    if (chr_len > 4096) return fail(ctx, GSNP_E_INVAL, "chr_name longer than 4096");
+    cudaStream_t s = ctx->stream;
+    // the text on the device, 16-byte aligned (host text or an unaligned device pointer: copied)
+    const uint8_t* t = reinterpret_cast<const uint8_t*>(text);
+    const bool dev_text = is_device_ptr(text);
+    if (!dev_text || (reinterpret_cast<uintptr_t>(text) & 15)) {
+        CK(ctx->p_text.ensure(n_bytes + 16));
+        CK(cudaMemcpyAsync(ctx->p_text.p, text, n_bytes, dev_text ? cudaMemcpyDeviceToDevice
+                                                                    : cudaMemcpyHostToDevice, s));
+        t = ctx->p_text.p;
+    }
+    uint8_t last = '\n';
+    if (n_bytes) {
+        if (dev_text) CK(cudaMemcpyAsync(&last, t + n_bytes - 1, 1, cudaMemcpyDeviceToHost, s));
+        else last = (uint8_t)text[n_bytes - 1];
+    }
+    CK(ctx->p_chr.ensure(chr_len + 1));
+    if (chr_len) CK(cudaMemcpyAsync(ctx->p_chr.p, chr_name, chr_len, cudaMemcpyHostToDevice, s));
+    CK(ctx->p_scal.ensure(8));
+    CK(cudaMemsetAsync(ctx->d_err.p, 0, sizeof(int), s));
+    CK(cudaMemsetAsync(ctx->p_scal.p, 0xFF, 8, s));                 // bad_line = max
+    // newlines: per-tile counts -> scan -> line starts
+    const uint64_t n_tiles = (n_bytes + PTILE - 1) / PTILE;
+    CK(ctx->p_cnt.ensure(n_tiles + 1));
+    uint64_t n_nl = 0;
+    if (n_tiles) {
+        ctx->begin();
+        k_nl_tiles<false><<<(unsigned)n_tiles, PNT, 0, s>>>(t, n_bytes, ctx->p_cnt.p, nullptr);
+        k_scan_partials<<<1, PNT, 0, s>>>(ctx->p_cnt.p, n_tiles);
+        ctx->end(GSNP_STAGE_PARSE);
+        ctx->launches += 2;
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(&n_nl, ctx->p_cnt.p + n_tiles, 8, cudaMemcpyDeviceToHost, s));
+    }
+    CK(cudaStreamSynchronize(s));
+    const uint64_t n_lines = n_nl + ((n_bytes && last != '\n') ? 1 : 0);
+    CK(ctx->p_ls.ensure(n_nl + 2));
+    uint64_t ls_end = n_bytes + 1;                                    // end of an unterminated line
+    if (n_tiles) {
+        ctx->begin();
+        k_nl_tiles<true><<<(unsigned)n_tiles, PNT, 0, s>>>(t, n_bytes, ctx->p_cnt.p, ctx->p_ls.p);
+        ctx->end(GSNP_STAGE_PARSE);
+        ctx->launches++;
+        CK(cudaGetLastError());
+    }
+    if (n_lines > n_nl) CK(cudaMemcpyAsync(ctx->p_ls.p + n_lines, &ls_end, 8, cudaMemcpyHostToDevice, s));
+    uint64_t tot[2] = {0, 0};
+    ParseArgs P;
+    memset(&P, 0, sizeof P);
+    P.text = t; P.n_bytes = n_bytes; P.n_lines = n_lines; P.ls = ctx->p_ls.p;
+    P.chr = ctx->p_chr.p; P.chr_len = (uint32_t)chr_len; P.q_offset = q_offset; P.loc_base = loc_base;
+    P.err = ctx->d_err.p; P.bad_line = reinterpret_cast<unsigned long long*>(ctx->p_scal.p);
+    const uint64_t n_sel_tiles = (n_lines + SEL_TILE - 1) / SEL_TILE;
+    if (n_lines) {
+        CK(ctx->p_meta.ensure(n_lines));
+        CK(ctx->p_pos.ensure(n_lines));
+        CK(ctx->p_ridx.ensure(n_lines));
+        CK(ctx->p_boff.ensure(n_lines));
+        CK(ctx->p_part.ensure(2 * (n_sel_tiles + 1)));
+        P.meta = ctx->p_meta.p; P.pos = ctx->p_pos.p; P.ridx = ctx->p_ridx.p; P.boff = ctx->p_boff.p;
+        const unsigned wgrid = (unsigned)std::min<uint64_t>((n_lines + 7) / 8, (uint64_t)g_num_sms * 16);
+        uint64_t* part_n = ctx->p_part.p;
+        uint64_t* part_b = ctx->p_part.p + n_sel_tiles + 1;
+        ctx->begin();
+        k_parse_meta<<<wgrid, PNT, 0, s>>>(P);
+        k_sel_tiles<<<(unsigned)n_sel_tiles, PNT, 0, s>>>(P.meta, n_lines, part_n, part_b);
+        k_scan_partials<<<1, PNT, 0, s>>>(part_n, n_sel_tiles);
+        k_scan_partials<<<1, PNT, 0, s>>>(part_b, n_sel_tiles);
+        ctx->end(GSNP_STAGE_PARSE);
+        ctx->launches += 4;
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(&tot[0], part_n + n_sel_tiles, 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(&tot[1], part_b + n_sel_tiles, 8, cudaMemcpyDeviceToHost, s));
+    }
+    int herr = 0;
+    unsigned long long bad = 0;
+    CK(cudaMemcpyAsync(&herr, ctx->d_err.p, sizeof(int), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(&bad, ctx->p_scal.p, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    ctx->flush();
+    if (herr) return fail(ctx, GSNP_E_RANGE, "malformed SOAP alignment line %llu (0-based)", bad);
+    if (n_reads) *n_reads = tot[0];
+    if (n_bases) *n_bases = tot[1];
+    if (reads_cap < tot[0] || bases_cap < tot[1])
+        return fail(ctx, GSNP_E_CAPACITY, "need %llu reads / %llu bases", (unsigned long long)tot[0],
+                    (unsigned long long)tot[1]);
+    if (!pos || !len || !off || !bases || !quals || !strand || !hits)
+        return fail(ctx, GSNP_E_INVAL, "NULL output array");
+    // outputs: device arrays written in place, host arrays through the staging buffers
+    const bool dev_out = is_device_ptr(pos);
+    P.o_pos = pos; P.o_len = len; P.o_off = off; P.o_bases = bases; P.o_quals = quals;
+    P.o_strand = strand; P.o_hits = hits;
+    if (!dev_out) {
+        CK(ctx->r_pos.ensure(tot[0] + 1)); CK(ctx->r_off.ensure(tot[0] + 1));
+        CK(ctx->r_len.ensure(tot[0] + 1)); CK(ctx->r_hits.ensure(tot[0] + 1));
+        CK(ctx->r_strand.ensure(tot[0] + 1));
+        CK(ctx->r_bases.ensure(tot[1] + 1)); CK(ctx->r_quals.ensure(tot[1] + 1));
+        P.o_pos = ctx->r_pos.p; P.o_len = ctx->r_len.p; P.o_off = ctx->r_off.p;
+        P.o_bases = ctx->r_bases.p; P.o_quals = ctx->r_quals.p; P.o_strand = ctx->r_strand.p;
+        P.o_hits = ctx->r_hits.p;
+    }
+    if (tot[0] == 0) {
+        const uint64_t z = 0;
+        CK(cudaMemcpyAsync(P.o_off, &z, 8, cudaMemcpyHostToDevice, s));
+        CK(cudaStreamSynchronize(s));
+    } else {
+        const uint64_t* part_n = ctx->p_part.p;
+        const uint64_t* part_b = ctx->p_part.p + n_sel_tiles + 1;
+        ctx->begin();
+        k_sel_apply<<<(unsigned)n_sel_tiles, PNT, 0, s>>>(P, part_n, part_b);
+        k_parse_emit<<<(unsigned)std::min<uint64_t>((n_lines + 7) / 8, (uint64_t)g_num_sms * 16), PNT, 0, s>>>(
+            P, tot[0], tot[1]);
+        ctx->end(GSNP_STAGE_PARSE);
+        ctx->launches += 2;
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(&herr, ctx->d_err.p, sizeof(int), cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(&bad, ctx->p_scal.p, 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        ctx->flush();
+        if (herr) return fail(ctx, GSNP_E_RANGE, "bad base or quality character on line %llu", bad);
+    }
+    if (!dev_out) {
+        const uint64_t nr = tot[0], nb = tot[1];
+        CK(cudaMemcpyAsync(pos, P.o_pos, nr * 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(len, P.o_len, nr * 2, cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(off, P.o_off, (nr + 1) * 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(strand, P.o_strand, nr, cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(hits, P.o_hits, nr * 2, cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(bases, P.o_bases, nb, cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(quals, P.o_quals, nb, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+    }
+    return GSNP_OK;
+}
+
 gsnp_status gsnp_compress(gsnp_ctx* ctx, const gsnp_record* rec, uint64_t n, uint32_t block_sites,
                           uint32_t* out, uint64_t out_cap, uint64_t* n_words) {
     if (!ctx) return GSNP_E_INVAL;
@@ -1042,6 +1193,9 @@ void gsnp_destroy(gsnp_ctx* ctx) {
     ctx->d_counts.release(); ctx->tile_ra.release(); ctx->tile_rb.release(); ctx->rec.release();
     ctx->big.release(); ctx->big_n.release(); ctx->wlist.release();
     ctx->dense_occ.release(); ctx->dense_cnt.release();
+    ctx->p_text.release(); ctx->p_chr.release(); ctx->p_cnt.release(); ctx->p_ls.release();
+    ctx->p_meta.release(); ctx->p_pos.release(); ctx->p_ridx.release(); ctx->p_boff.release();
+    ctx->p_part.release(); ctx->p_scal.release();
     ctx->r_pos.release(); ctx->r_off.release(); ctx->r_len.release(); ctx->r_hits.release();
     ctx->r_bases.release(); ctx->r_quals.release(); ctx->r_strand.release();
     ctx->dbg_u32a.release(); ctx->dbg_u32b.release(); ctx->dbg_u32c.release();

@@ -19,14 +19,14 @@ GSNP_TIMING = 0x2
 GSNP_MONOPLOID = 0x4
 GSNP_TITV = 0x8
 STAGES = ("validate", "calib_count", "tile_ranges", "call_tile", "finalize", "big_sites",
-          "compress", "warp_sites", "dense_count", "dense_lik", "dense_recycle")
+          "compress", "warp_sites", "dense_count", "dense_lik", "dense_recycle", "parse")
 STATUS = {0: "GSNP_OK", -1: "GSNP_E_INVAL", -2: "GSNP_E_RANGE", -3: "GSNP_E_UNSORTED",
           -4: "GSNP_E_STATE", -5: "GSNP_E_NOMEM", -6: "GSNP_E_CUDA", -7: "GSNP_E_CAPACITY"}
 
 # exported symbols declared in include/gsnp.h
 SYMBOLS = ("gsnp_params_default", "gsnp_create", "gsnp_calibrate", "gsnp_calibrate_count",
            "gsnp_calibrate_finalize", "gsnp_call", "gsnp_debug_window", "gsnp_get_tables",
-           "gsnp_compress", "gsnp_call_compressed", "gsnp_call_dense", "gsnp_priors_from_freq",
+           "gsnp_compress", "gsnp_call_compressed", "gsnp_call_dense", "gsnp_priors_from_freq", "gsnp_parse_soap",
            "gsnp_launch_count", "gsnp_stage_times", "gsnp_strerror", "gsnp_last_error",
            "gsnp_destroy")
 
@@ -109,6 +109,9 @@ def lib():
                                       P, u64, ctypes.POINTER(u64)]
         L.gsnp_priors_from_freq.restype = S
         L.gsnp_priors_from_freq.argtypes = [P, u64, ctypes.c_double, P]
+        L.gsnp_parse_soap.restype = S
+        L.gsnp_parse_soap.argtypes = [P, P, u64, ctypes.c_char_p, ctypes.c_uint32, u64] + [P] * 7 + \
+            [u64, u64, ctypes.POINTER(u64), ctypes.POINTER(u64)]
         L.gsnp_launch_count.restype = u64
         L.gsnp_launch_count.argtypes = [P]
         L.gsnp_stage_times.restype = S
@@ -264,6 +267,42 @@ class Context:
                                      ctypes.byref(n)), self.h)
         return out
 
+    def parse_soap(self, text, chr_name=None, q_offset: int = 33, loc_base: int = 0,
+                   device: bool = True, out: dict | None = None):
+        """SOAP alignment text -> reads dict (gsnp_parse_soap).  text: bytes /
+        numpy uint8 (host) or a CUDA uint8 tensor.  Returns CUDA tensors (device=True) or numpy
+        arrays, trimmed to the parsed sizes; out: preallocated arrays to fill instead (sizes are
+        then the caller's, e.g. from a previous parse)."""
+        if isinstance(text, (bytes, bytearray)):
+            text = np.frombuffer(bytes(text), np.uint8)
+        nb = int(text.numel() if hasattr(text, "numel") else len(text))
+        chr_b = chr_name.encode() if chr_name else None
+        nr, nbs = ctypes.c_uint64(0), ctypes.c_uint64(0)
+        if out is None:
+            st = lib().gsnp_parse_soap(self.h, _ptr(text), nb, chr_b, q_offset, loc_base,
+                                       *([None] * 7), 0, 0, ctypes.byref(nr), ctypes.byref(nbs))
+            if st not in (0, -7):
+                _check(st, self.h)
+            R, B = int(nr.value), int(nbs.value)
+            spec = dict(pos=(R, "uint64"), len=(R, "uint16"), off=(R + 1, "uint64"),
+                        bases=(B, "uint8"), quals=(B, "uint8"), strand=(R, "uint8"),
+                        hits=(R, "uint16"))
+            if device:
+                import torch
+                out = {k: torch.empty(max(n, 1), dtype=getattr(torch, d), device="cuda")
+                       for k, (n, d) in spec.items()}
+            else:
+                out = {k: np.zeros(max(n, 1), d) for k, (n, d) in spec.items()}
+        cap_r = int(out["pos"].numel() if hasattr(out["pos"], "numel") else len(out["pos"]))
+        cap_b = int(out["bases"].numel() if hasattr(out["bases"], "numel") else len(out["bases"]))
+        _check(lib().gsnp_parse_soap(self.h, _ptr(text), nb, chr_b, q_offset, loc_base,
+                                     *[_ptr(out[k]) for k in ("pos", "len", "off", "bases", "quals",
+                                                              "strand", "hits")],
+                                     cap_r, cap_b, ctypes.byref(nr), ctypes.byref(nbs)), self.h)
+        R, B = int(nr.value), int(nbs.value)
+        return {k: v[:(R + 1 if k == "off" else B if k in ("bases", "quals") else R)]
+                for k, v in out.items()}
+
     def compress(self, rec, block_sites: int = 65536, out=None):
         """§V-B compression of records (numpy RECORD_DTYPE array, or a CUDA uint8 tensor of
         40*n bytes).  out: None (numpy uint32 result, sized by a query call) or a uint32 buffer
@@ -377,6 +416,10 @@ def gsnp_priors_from_freq(freq, floor_prior: float = 5e-7) -> np.ndarray:
     out = np.zeros((len(f), 10), np.float64)
     _check(lib().gsnp_priors_from_freq(_ptr(f), len(f), float(floor_prior), _ptr(out)), None)
     return out
+
+
+def gsnp_parse_soap(ctx: Context, text, chr_name=None, q_offset=33, loc_base=0, device=True):
+    return ctx.parse_soap(text, chr_name, q_offset, loc_base, device)
 
 
 def gsnp_debug_window(ctx: Context, reads, w0, w1):

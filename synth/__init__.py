@@ -94,6 +94,9 @@ def _lib():
     lib.syn_plan.argtypes = [ctypes.POINTER(_Cfg), P, P, P, P]
     lib.syn_fill.restype = ctypes.c_uint64
     lib.syn_fill.argtypes = [ctypes.POINTER(_Cfg), P, P, P, P] + [P] * 7
+    lib.syn_soap_text.restype = ctypes.c_uint64
+    lib.syn_soap_text.argtypes = [ctypes.c_uint64] + [P] * 7 + [ctypes.c_char_p, ctypes.c_uint32,
+                                                               ctypes.c_uint64, P]
     lib.syn_known.restype = ctypes.c_uint64
     lib.syn_known.argtypes = [ctypes.POINTER(_Cfg), P, P, P, P, P]
     return lib
@@ -170,3 +173,26 @@ def slice_reads(w: dict, ra: int, rb: int) -> dict:
                hits=w["hits"][ra:rb], off=(w["off"][ra:rb + 1] - np.uint64(o0)),
                bases=w["bases"][o0:o1], quals=w["quals"][o0:o1])
     return out
+
+
+def soap_text(w: dict, chr_name: str = "chr1", q_offset: int = 33, loc_base: int | None = None,
+              ra: int = 0, rb: int | None = None) -> bytes:
+    """Reads [ra, rb) of a workload as SOAP alignment text (reading R19): one tab-separated line
+    per read — id, seq, qual, n_hits, a/b, len, strand, chr, 1-based location, n_mismatch.
+    location = pos - loc_base + 1 (loc_base defaults to the workload's origin)."""
+    lib = _lib()
+    rb = len(w["pos"]) if rb is None else rb
+    lb = int(w["origin"]) if loc_base is None else loc_base
+    arr = dict(pos=np.ascontiguousarray(w["pos"][ra:rb], np.uint64),
+               len=np.ascontiguousarray(w["len"][ra:rb], np.uint16),
+               off=np.ascontiguousarray(w["off"][ra:rb + 1], np.uint64),
+               strand=np.ascontiguousarray(w["strand"][ra:rb], np.uint8),
+               hits=np.ascontiguousarray(w["hits"][ra:rb], np.uint16))
+    bases = np.ascontiguousarray(w["bases"], np.uint8)
+    quals = np.ascontiguousarray(w["quals"], np.uint8)
+    a = [rb - ra, _p(arr["pos"]), _p(arr["len"]), _p(arr["off"]), _p(bases), _p(quals),
+         _p(arr["strand"]), _p(arr["hits"]), chr_name.encode(), q_offset, lb]
+    n = lib.syn_soap_text(*a, None)
+    out = np.empty(n, np.uint8)
+    lib.syn_soap_text(*a, _p(out))
+    return out.tobytes()

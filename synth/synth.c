@@ -332,3 +332,50 @@ uint64_t syn_known(const syn_config* c, const uint8_t* ref, const uint8_t* snp, 
     }
     return k;
 }
+
+/* ------------------------------------------------------------------------------------------
+ * SOAP alignment text (input file 1 of P:L206-212 in SOAPsnp's format; reading R19 of
+ * DESIGN.md): one line per read, tab-separated
+ *   id  seq  qual  n_hits  a  len  strand  chr  location(1-based)  n_mismatch
+ * seq in reference-forward orientation (ACGTN), qual = chr(q + q_offset).  Writes the lines of
+ * reads [0, n) to out (NULL: size query); returns the number of bytes.
+ */
+static uint32_t put_u64(char* o, uint64_t v) {
+    char t[24];
+    uint32_t k = 0;
+    do { t[k++] = (char)('0' + v % 10); v /= 10; } while (v);
+    for (uint32_t i = 0; i < k; ++i) o[i] = t[k - 1 - i];
+    return k;
+}
+
+uint64_t syn_soap_text(uint64_t n, const uint64_t* pos, const uint16_t* len, const uint64_t* off,
+                       const uint8_t* bases, const uint8_t* quals, const uint8_t* strand,
+                       const uint16_t* hits, const char* chr, uint32_t q_offset,
+                       uint64_t loc_base, char* out) {
+    static const char B[5] = {'A', 'C', 'T', 'G', 'N'};
+    char buf[1024];
+    uint64_t tot = 0;
+    size_t cl = strlen(chr);
+    for (uint64_t r = 0; r < n; ++r) {
+        char* o = buf;
+        *o++ = 'r';
+        o += put_u64(o, r);
+        *o++ = '\t';
+        for (uint32_t i = 0; i < len[r]; ++i) *o++ = B[bases[off[r] + i] > 4 ? 4 : bases[off[r] + i]];
+        *o++ = '\t';
+        for (uint32_t i = 0; i < len[r]; ++i) *o++ = (char)(quals[off[r] + i] + q_offset);
+        *o++ = '\t';
+        o += put_u64(o, hits[r]);
+        *o++ = '\t'; *o++ = (r & 1) ? 'b' : 'a'; *o++ = '\t';
+        o += put_u64(o, len[r]);
+        *o++ = '\t'; *o++ = strand[r] ? '-' : '+'; *o++ = '\t';
+        memcpy(o, chr, cl); o += cl;
+        *o++ = '\t';
+        o += put_u64(o, pos[r] - loc_base + 1);
+        *o++ = '\t'; *o++ = '0'; *o++ = '\n';
+        uint64_t k = (uint64_t)(o - buf);
+        if (out) memcpy(out + tot, buf, k);
+        tot += k;
+    }
+    return tot;
+}
