@@ -49,7 +49,8 @@ __global__ void __launch_bounds__(DENSE_NT) k_dense_count(DenseArgs D) {
             const uint64_t site = p + i;
             if (site < D.c0 || site >= D.c1) continue;
             const uint32_t b = A.R.bases[o + i];
-            if (b >= 4) continue;                                   // N: not aligned
+            if (b > 4 || A.R.quals[o + i] > (uint32_t)A.q_max) { err |= ERR_RANGE; continue; }
+            if (b == 4) continue;                                   // N: not aligned
             const uint64_t s = site - D.c0;
             atomicAdd(D.cnt + s * 5 + b, 1u);
             atomicAdd(D.cnt + s * 5 + 4, hk);

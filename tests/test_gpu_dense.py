@@ -78,3 +78,15 @@ def test_dense_device_io_and_bad_chunk():
         for bad in (0, 31, 33):
             with pytest.raises(gsnp.GsnpError):
                 ctx.call_dense(w, 0, 2_000, chunk_sites=bad)
+
+
+def test_dense_out_of_range_quality_is_status():
+    w = synth.generate("C1", n_sites=2_000, depth=10.0, seed=10)
+    with gsnp.Context.from_workload(w) as ctx:
+        ctx.calibrate(w)
+        bad = dict(w, quals=w["quals"].copy())
+        bad["quals"][7] = 50                                   # > q_max (40)
+        with pytest.raises(gsnp.GsnpError) as e:
+            ctx.call_dense(bad, 0, 2_000, chunk_sites=512)
+        assert e.value.status == -2
+        assert ctx.call_dense(w, 0, 2_000, chunk_sites=512).tobytes() == ctx.call(w, 0, 2_000).tobytes()
