@@ -488,6 +488,7 @@ gsnp_status count_impl(gsnp_ctx* ctx, const gsnp_reads* reads) {
         A.q_max = (int)ctx->prm.q_max;
         A.C = ctx->d_counts.p;
         A.err = ctx->d_err.p;
+        A.tma_ok = ((reinterpret_cast<uintptr_t>(d.bases) | reinterpret_cast<uintptr_t>(d.quals)) & 15) == 0;
         // shared memory: u32 diagonal histogram [q][t][cycle] + two stages of (bases, quals,
         // reference window).  Cycles beyond Lh (only for long reads at high q_max) use global REDs.
         const size_t budget = 200 * 1024;

@@ -194,6 +194,7 @@ struct CalibArgs {
     uint32_t RB;                      // bytes per reference-window buffer
     unsigned long long* C;            // [64][256][4][4]
     int* err;
+    int tma_ok;                       // bases and quals 16-byte aligned (TMA bulk copies allowed)
 };
 
 constexpr int CAL_NT = 1024;
@@ -249,8 +250,11 @@ __global__ void __launch_bounds__(CAL_NT, 1) k_calib_count(CalibArgs A) {
         const uint64_t r0 = p0 >= A.origin ? ((p0 - A.origin) & ~15ull) : 0;
         const uint64_t r1 = ((p1 + L - A.origin) + 15) & ~15ull;
         st_rs[sidx] = (uint32_t)r0;
-        const bool fits = a1 - a0 <= A.SB && p0 >= A.origin && p1 + L <= A.origin + A.n_sites &&
-                          r1 - r0 <= A.RB;
+        // the rounded-up copy must stay inside the caller's arrays (their last valid byte is
+        // off[n] - 1): a batch at the very end whose 16-byte round-up would overrun reads global
+        const uint64_t end = A.R.off[A.R.n] - A.R.off0;
+        const bool fits = A.tma_ok && a1 <= end && a1 - a0 <= A.SB && p0 >= A.origin &&
+                          p1 + L <= A.origin + A.n_sites && r1 - r0 <= A.RB;
         st_direct[sidx] = fits ? 0 : 1;
         if (!fits) return;
         unsigned char* sb = stage + (size_t)sidx * stage_bytes;

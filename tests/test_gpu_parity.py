@@ -268,3 +268,22 @@ def test_long_reads_full_quality_range_parity(read_len):
         assert np.array_equal(counts.reshape(64, 256, 4, 4), C)
         ctx.calibrate_finalize(counts)
         _check_window(ctx, w, 0, 4_000, C, p, P)
+
+
+def test_unaligned_device_reads_calibrate_and_call(c1):
+    """Device byte arrays at an odd address: the calibration's TMA stages must fall back to
+    global loads (bulk copies need 16-byte alignment) and give the same counts and records."""
+    import torch
+    w, C, p, rec, _ = c1
+    dev = {k: torch.from_numpy(np.ascontiguousarray(w[k])).cuda()
+           for k in ("pos", "len", "off", "strand", "hits")}
+    for k in ("bases", "quals"):
+        buf = torch.zeros(len(w[k]) + 3, dtype=torch.uint8, device="cuda")
+        buf[3:] = torch.from_numpy(np.ascontiguousarray(w[k])).cuda()
+        dev[k] = buf[3:]
+    with _ctx(w) as ctx:
+        counts = ctx.calibrate_count(dev)
+        assert np.array_equal(counts.reshape(64, 256, 4, 4), C)
+        ctx.calibrate_finalize(counts)
+        got = ctx.call(dev, int(w["origin"]), int(w["origin"]) + len(w["ref"]))
+    compare(w, got, rec, c1[4]["L10"])
