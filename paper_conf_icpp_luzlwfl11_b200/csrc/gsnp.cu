@@ -967,7 +967,8 @@ gsnp_status gsnp_parse_soap(gsnp_ctx* ctx, const char* text, uint64_t n_bytes, c
         CK(ctx->p_boff.ensure(n_lines));
         CK(ctx->p_part.ensure(2 * (n_sel_tiles + 1)));
         P.meta = ctx->p_meta.p; P.pos = ctx->p_pos.p; P.ridx = ctx->p_ridx.p; P.boff = ctx->p_boff.p;
-        const unsigned wgrid = (unsigned)std::min<uint64_t>((n_lines + 7) / 8, (uint64_t)g_num_sms * 16);
+        const unsigned wgrid = (unsigned)std::min<uint64_t>((n_lines + PGROUPS - 1) / PGROUPS,
+                                                            (uint64_t)g_num_sms * 8);
         uint64_t* part_n = ctx->p_part.p;
         uint64_t* part_b = ctx->p_part.p + n_sel_tiles + 1;
         ctx->begin();
@@ -993,6 +994,8 @@ gsnp_status gsnp_parse_soap(gsnp_ctx* ctx, const char* text, uint64_t n_bytes, c
     if (reads_cap < tot[0] || bases_cap < tot[1])
         return fail(ctx, GSNP_E_CAPACITY, "need %llu reads / %llu bases", (unsigned long long)tot[0],
                     (unsigned long long)tot[1]);
+    if (!pos && !len && !off && !bases && !quals && !strand && !hits && tot[0] == 0)
+        return GSNP_OK;                                               // size query of an empty parse
     if (!pos || !len || !off || !bases || !quals || !strand || !hits)
         return fail(ctx, GSNP_E_INVAL, "NULL output array");
     // outputs: device arrays written in place, host arrays through the staging buffers
@@ -1017,7 +1020,7 @@ gsnp_status gsnp_parse_soap(gsnp_ctx* ctx, const char* text, uint64_t n_bytes, c
         const uint64_t* part_b = ctx->p_part.p + n_sel_tiles + 1;
         ctx->begin();
         k_sel_apply<<<(unsigned)n_sel_tiles, PNT, 0, s>>>(P, part_n, part_b);
-        k_parse_emit<<<(unsigned)std::min<uint64_t>((n_lines + 7) / 8, (uint64_t)g_num_sms * 16), PNT, 0, s>>>(
+        k_parse_emit<<<(unsigned)std::min<uint64_t>((n_lines + PGROUPS - 1) / PGROUPS, (uint64_t)g_num_sms * 8), PNT, 0, s>>>(
             P, tot[0], tot[1]);
         ctx->end(GSNP_STAGE_PARSE);
         ctx->launches += 2;

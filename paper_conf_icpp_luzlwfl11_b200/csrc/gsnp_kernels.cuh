@@ -515,9 +515,6 @@ __global__ void k_tile_ranges(const uint64_t* pos, uint64_t n, uint64_t w0, uint
 // parallelisation).  Shared-memory layout (host: call_smem_bytes()).
 constexpr int TS = NT;
 constexpr int COLS = 32;              // key slots per site, shallow kernel (thread path n <= 32)
-#ifndef GSNP_G_PF
-#define GSNP_G_PF 0
-#endif
 #ifndef GSNP_GB
 #define GSNP_GB 1
 #endif
@@ -600,16 +597,6 @@ __device__ __forceinline__ void add_row(const double* __restrict__ T, int L, uin
     acc[0] += v0.x; acc[1] += v0.y; acc[2] += v1.x; acc[3] += v1.y; acc[4] += v2.x;
     acc[5] += v2.y; acc[6] += v3.x; acc[7] += v3.y; acc[8] += v4.x; acc[9] += v4.y;
 #endif
-}
-
-#ifndef GSNP_P2_PF
-#define GSNP_P2_PF 0
-#endif
-__device__ __forceinline__ void prefetch_row(const double* __restrict__ T, uint32_t L, uint32_t qa,
-                                             uint32_t cyc, uint32_t b) {
-    const double* row = T + ((size_t)(qa * L + cyc) * 4u + b) * TROW;
-    asm volatile("prefetch.global.L1 [%0];" ::"l"(row));
-    asm volatile("prefetch.global.L1 [%0];" ::"l"(row + 11));
 }
 
 // adjust(score, dep_count) through the host-built table (R3): adj[q][min(pcr,P)-1][min(g,G-1)]
@@ -942,13 +929,6 @@ __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* ad
 #pragma unroll kP2Unroll
     for (uint32_t j = 0; j < n; ++j) {
         const uint32_t kk = colp[j * TS];
-#if GSNP_P2_PF
-        // L1 prefetch of the row GSNP_P2_PF keys ahead: no registers held across the add
-        if (j + GSNP_P2_PF < n) {
-            const uint32_t kp = colp[(j + GSNP_P2_PF) * TS];
-            prefetch_row(T, L, kp >> 17, key_cyc(kp), key_base(kp));
-        }
-#endif
         add_row(T, (int)L, kk >> 17, key_cyc(kk), key_base(kk), acc);
     }
 #endif
@@ -1533,19 +1513,6 @@ k_call_tile(CallArgs A, uint32_t* wlist, uint32_t* wlist_n, uint32_t* work, uint
         const int nr = (int)min((uint64_t)32, wrb - r0);
         uint32_t cpack = 0;                                    // 4 x 8-bit base counts this batch
         for (int k0 = 0; k0 < nr; k0 += GB) {
-#if GSNP_G_PF
-            {   // L1 prefetch of the bytes of the read GSNP_G_PF ahead (no registers held)
-                const int kq = (k0 + GSNP_G_PF) & 31;
-                const int pq = __shfl_sync(FULL, pr, kq);
-                const uint32_t oq = __shfl_sync(FULL, o, kq);
-                const uint32_t mq = __shfl_sync(FULL, meta, kq);
-                const uint32_t iq = (uint32_t)(lane_rel - pq);
-                if (k0 + GSNP_G_PF < nr && iq < (mq & 511u)) {
-                    asm volatile("prefetch.global.L1 [%0];" ::"l"(wbases + oq + iq));
-                    asm volatile("prefetch.global.L1 [%0];" ::"l"(wquals + oq + iq));
-                }
-            }
-#endif
             int pk[GB];
             uint32_t ii[GB], mk[GB], bb[GB], qq[GB];
 #pragma unroll

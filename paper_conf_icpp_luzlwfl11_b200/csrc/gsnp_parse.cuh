@@ -5,13 +5,15 @@
 //   k_nl_tiles<false>  per 16 KiB tile of text: number of '\n' (16-byte vector loads)
 //   k_scan_partials    exclusive scan of the tile counts (one CTA)
 //   k_nl_tiles<true>   per tile: block scans give every newline its line number; line_start[]
-//   k_parse_meta       one warp per line: tab positions by ballot over 32-byte steps, the numeric
-//                      fields (n_hits, len, location) by a warp-parallel decimal reduction, the
-//                      chromosome compare, field validation -> packed per-line metadata
+//   k_parse_meta       one 8-lane group per line (4 lines in flight per warp): the line staged in
+//                      shared memory by 16-byte loads, tabs found 32 bytes per lane per step with
+//                      a group prefix sum, numeric fields (n_hits, len, location) by a group-
+//                      parallel decimal reduction, chromosome compare, validation -> packed
+//                      per-line metadata
 //   k_sel_tiles / k_scan_partials / k_sel_apply   read index and base offset of every selected
 //                      line (exclusive scans of 1 and len over the lines of the wanted chr)
-//   k_parse_emit       one warp per selected line: pos/len/strand/hits, off[], and the sequence /
-//                      quality characters converted to codes (coalesced byte lanes)
+//   k_parse_emit       one 8-lane group per selected line: pos/len/strand/hits, off[], and the
+//                      sequence / quality characters converted to codes (16 bytes per lane)
 #pragma once
 
 namespace gsnp_dev {
@@ -126,88 +128,160 @@ __device__ __constant__ uint64_t kPow10[20] = {
     100000000000000ull, 1000000000000000ull, 10000000000000000ull, 100000000000000000ull,
     1000000000000000000ull, 10000000000000000000ull};
 
-// decimal field text[a, b) -> value (warp-parallel; b - a <= 19 digits); ok = all digits
-__device__ __forceinline__ uint64_t warp_decimal(const uint8_t* text, uint64_t a, uint64_t b,
-                                                 int lane, bool& ok) {
-    const uint32_t nd = (uint32_t)(b - a);
-    ok = nd >= 1 && nd <= 19;
-    if (!ok) return 0;
-    uint64_t v = 0;
-    bool good = true;
-    if ((uint32_t)lane < nd) {
-        const uint32_t c = text[a + lane];
-        good = c >= '0' && c <= '9';
-        v = (uint64_t)(c - '0') * kPow10[nd - 1 - lane];
-    }
-    ok = __all_sync(FULL, good);
+// Lines are handled by groups of PG = 8 lanes (four lines in flight per warp).  A group stages
+// its line's bytes in shared memory with 16-byte loads (lines up to PSTAGE - 15 bytes; longer
+// lines are read from global memory byte by byte — same code, slower source).
+constexpr int PG = 8;
+constexpr int PSTAGE = 640;                     // staging bytes per group
+constexpr int PGROUPS = PNT / PG;               // groups per CTA
+
+__device__ __forceinline__ uint32_t group_mask(int lane) { return 0xFFu << (lane & ~(PG - 1)); }
+
+// group sum (lanes of one 8-lane group)
+__device__ __forceinline__ uint64_t group_sum(uint64_t v) {
 #pragma unroll
-    for (int d = 16; d; d >>= 1) v += __shfl_xor_sync(FULL, v, d);
+    for (int d = PG / 2; d; d >>= 1) v += __shfl_xor_sync(FULL, v, d);
     return v;
 }
 
 __global__ void __launch_bounds__(PNT) k_parse_meta(ParseArgs P) {
-    const int lane = threadIdx.x & 31;
-    const uint64_t nw = (uint64_t)gridDim.x * (PNT / 32);
-    for (uint64_t l = (uint64_t)blockIdx.x * (PNT / 32) + (threadIdx.x >> 5); l < P.n_lines; l += nw) {
-        const uint64_t a = P.ls[l];
-        uint64_t b = P.ls[l + 1] - 1;                    // the '\n' (or n_bytes for the last line)
-        if (b > P.n_bytes) b = P.n_bytes;
+    __shared__ __align__(16) uint8_t stage_s[PGROUPS][PSTAGE];
+    __shared__ uint64_t tab_s[PGROUPS][9];
+    const int lane = threadIdx.x & 31, sub = lane & (PG - 1), g = threadIdx.x / PG;
+    const int gbase = lane & ~(PG - 1);                       // first lane of this group
+    uint8_t* buf = stage_s[g];
+    uint64_t* tabs = tab_s[g];
+    const uint64_t ngroups = (uint64_t)gridDim.x * PGROUPS;
+    // warp-uniform rounds; in each, group g takes line l0 + g
+    for (uint64_t l0 = (uint64_t)blockIdx.x * PGROUPS + (threadIdx.x / 32) * (32 / PG);
+         __any_sync(FULL, l0 + (lane / PG) < P.n_lines); l0 += ngroups) {
+        const uint64_t l = l0 + (lane / PG);
+        const bool act = l < P.n_lines;
+        uint64_t a = 0, b = 0;
+        if (act) {
+            a = P.ls[l];
+            b = P.ls[l + 1] - 1;                                 // the '\n' (or n_bytes)
+            if (b > P.n_bytes) b = P.n_bytes;
+            if (b < a) b = a;
+        }
+        const uint64_t A0 = a & ~15ull;
+        const uint32_t nchunk = (uint32_t)((b - A0 + 15) / 16);
+        const bool fast = nchunk * 16 <= PSTAGE;
+        // stage the line: chunk c = sub + 8k, five 16-byte loads per lane at most
+        uint4 v[PSTAGE / 16 / PG];
+#pragma unroll
+        for (int k = 0; k < PSTAGE / 16 / PG; ++k) {
+            const uint32_t c = sub + PG * k;
+            v[k] = make_uint4(0, 0, 0, 0);
+            if (act && fast && c < nchunk) {
+                const uint64_t q = A0 + 16 * (uint64_t)c;
+                if (q + 16 <= P.n_bytes) v[k] = *reinterpret_cast<const uint4*>(P.text + q);
+                else {                                         // the text's last, partial chunk
+                    uint32_t w[4] = {0, 0, 0, 0};
+                    for (uint64_t i = q; i < P.n_bytes; ++i) w[(i - q) >> 2] |= (uint32_t)P.text[i] << (8 * ((i - q) & 3));
+                    v[k] = make_uint4(w[0], w[1], w[2], w[3]);
+                }
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < PSTAGE / 16 / PG; ++k) {
+            const uint32_t c = sub + PG * k;
+            if (act && fast && c < nchunk) *reinterpret_cast<uint4*>(buf + 16 * c) = v[k];
+        }
+        __syncwarp();
+        auto at = [&](uint64_t p) -> uint32_t { return fast ? buf[p - A0] : P.text[p]; };
+        // tabs in order: each lane scans 32 bytes per step; group prefix of the counts
+        uint32_t ntab = 0;
+        for (uint64_t p0 = A0; __any_sync(FULL, act && p0 < b && ntab < 9); p0 += 32 * PG) {
+            const uint64_t q0 = p0 + 32 * (uint64_t)sub;
+            uint32_t m = 0;
+            if (act && p0 < b && ntab < 9) {
+                if (fast && q0 < b) {
+                    const uint4 x = *reinterpret_cast<const uint4*>(buf + (q0 - A0));
+                    const uint4 y = *reinterpret_cast<const uint4*>(buf + (q0 - A0) + 16);
+                    const uint32_t w[8] = {x.x, x.y, x.z, x.w, y.x, y.y, y.z, y.w};
+#pragma unroll
+                    for (int k = 0; k < 32; ++k)
+                        m |= (((w[k >> 2] >> (8 * (k & 3))) & 255u) == 9u) ? 1u << k : 0u;
+                } else if (!fast) {
+                    for (int k = 0; k < 32; ++k)
+                        if (q0 + k < b && P.text[q0 + k] == '\t') m |= 1u << k;
+                }
+                // keep bytes inside [a, b)
+                for (int k = 0; k < 32; ++k)
+                    if (q0 + k < a || q0 + k >= b) m &= ~(1u << k);
+            }
+            uint32_t cnt = __popc(m), inc = cnt;
+#pragma unroll
+            for (int d = 1; d < PG; d <<= 1) {
+                const uint32_t y = __shfl_up_sync(FULL, inc, d);
+                if (sub >= d) inc += y;
+            }
+            uint32_t idx = ntab + inc - cnt;
+            for (; m && idx < 9; m &= m - 1, ++idx) tabs[idx] = q0 + (uint64_t)(__ffs(m) - 1);
+            ntab += __shfl_sync(FULL, inc, gbase + PG - 1);
+        }
+        __syncwarp();
+        uint64_t tab[9];
+#pragma unroll
+        for (int k = 0; k < 9; ++k) tab[k] = (uint32_t)k < ntab ? tabs[k] : b;
+        bool ok = ntab >= 8;                                     // 9 fields: id .. location
+        bool want = act && b > a && ok;
+        // chromosome (field 8: tab[6]+1 .. tab[7])
+        bool eq = true;
+        if (want && P.chr_len) {
+            const uint64_t ca = tab[6] + 1;
+            eq = tab[7] - ca == P.chr_len;
+            if (eq)
+                for (uint32_t i = sub; i < P.chr_len; i += PG) eq &= at(ca + i) == P.chr[i];
+        }
+        want = want && (__ballot_sync(FULL, !eq) & group_mask(lane)) == 0;
+        // numeric fields n_hits (3), len (5), location (8): digits spread over the group
+        uint64_t fa[3] = {tab[2] + 1, tab[4] + 1, tab[7] + 1};
+        uint64_t fb[3] = {tab[3], tab[5], ntab >= 9 ? tab[8] : b};
+        uint64_t val[3];
+        bool dig_ok = true;
+#pragma unroll
+        for (int f = 0; f < 3; ++f) {
+            const uint64_t nd = want ? fb[f] - fa[f] : 0;
+            uint64_t v = 0;
+            if (want && (nd < 1 || nd > 19)) dig_ok = false;
+            if (want && nd >= 1 && nd <= 19)
+                for (uint32_t i = sub; i < nd; i += PG) {
+                    const uint32_t c = at(fa[f] + i);
+                    dig_ok &= c >= '0' && c <= '9';
+                    v += (uint64_t)(c - '0') * kPow10[nd - 1 - i];
+                }
+            val[f] = group_sum(v);
+        }
+        const bool digits = (__ballot_sync(FULL, !dig_ok) & group_mask(lane)) == 0;
         uint64_t meta = 0, pos = 0;
-        if (b > a) {                                     // empty lines are skipped
-            // tab positions t[0..8] (fields 1..9 start after them)
-            uint64_t tab[9];
-#pragma unroll
-            for (int k = 0; k < 9; ++k) tab[k] = b;
-            uint32_t ntab = 0;
-            for (uint64_t p0 = a; p0 < b && ntab < 9; p0 += 32) {
-                const uint64_t p = p0 + lane;
-                const bool is_tab = p < b && P.text[p] == '\t';
-                uint32_t m = __ballot_sync(FULL, is_tab);
-                while (m && ntab < 9) {
-                    const uint64_t tp = p0 + (uint64_t)(__ffs(m) - 1);
-#pragma unroll
-                    for (int k = 0; k < 9; ++k) tab[k] = (k == (int)ntab) ? tp : tab[k];
-                    ++ntab;
-                    m &= m - 1;
-                }
+        bool bad = act && b > a && !ok;
+        if (want) {
+            const uint64_t hits = val[0], len = val[1], loc = val[2];
+            const uint64_t seq_a = tab[0] + 1, seq_len = tab[1] - seq_a;
+            const uint64_t qual_len = tab[2] - (tab[1] + 1);
+            const uint32_t sc = tab[6] - tab[5] == 2 ? at(tab[5] + 1) : 0u;
+            const bool good = digits && hits >= 1 && len >= 1 && len <= 256 && seq_len == len &&
+                              qual_len == len && loc >= 1 && (sc == '+' || sc == '-') &&
+                              seq_a - a < (1ull << 32);
+            if (good) {
+                const uint64_t h = hits > 65535 ? 65535 : hits;
+                meta = len | (uint64_t)(sc == '-') << 9 | 1ull << 10 | h << 11 | (seq_a - a) << 32;
+                pos = loc - 1 + P.loc_base;
+            } else {
+                bad = true;
             }
-            bool ok = ntab >= 8;                          // 9 fields: id .. location
-            const uint64_t f9_end = ntab >= 9 ? tab[8] : b;
-            // chromosome (field 8: tab[6]+1 .. tab[7])
-            bool want = ok;
-            if (ok && P.chr_len) {
-                const uint64_t ca = tab[6] + 1, cl = tab[7] - ca;
-                bool eq = cl == P.chr_len;
-                if (eq)
-                    for (uint32_t i = lane; i < P.chr_len; i += 32) eq &= P.text[ca + i] == P.chr[i];
-                want = __all_sync(FULL, eq);
-            }
-            if (want) {
-                bool o1, o2, o3;
-                const uint64_t hits = warp_decimal(P.text, tab[2] + 1, tab[3], lane, o1);
-                const uint64_t len = warp_decimal(P.text, tab[4] + 1, tab[5], lane, o2);
-                const uint64_t loc = warp_decimal(P.text, tab[7] + 1, f9_end, lane, o3);
-                const uint64_t seq_a = tab[0] + 1, seq_len = tab[1] - seq_a;
-                const uint64_t qual_len = tab[2] - (tab[1] + 1);
-                const uint32_t sc = tab[6] - tab[5] == 2 ? P.text[tab[5] + 1] : 0u;
-                ok = o1 && o2 && o3 && hits >= 1 && len >= 1 && len <= 256 && seq_len == len &&
-                     qual_len == len && loc >= 1 && (sc == '+' || sc == '-') && seq_a - a < (1ull << 32);
-                if (ok) {
-                    const uint64_t h = hits > 65535 ? 65535 : hits;
-                    meta = len | (uint64_t)(sc == '-') << 9 | 1ull << 10 | h << 11 |
-                           (seq_a - a) << 32;
-                    pos = loc - 1 + P.loc_base;
-                }
-            }
-            if (!ok && lane == 0) {
+        }
+        if (act && sub == 0) {
+            P.meta[l] = meta;
+            P.pos[l] = pos;
+            if (bad) {
                 atomicOr(P.err, ERR_PARSE);
                 atomicMin(P.bad_line, (unsigned long long)l);
             }
         }
-        if (lane == 0) {
-            P.meta[l] = meta;
-            P.pos[l] = pos;
-        }
+        __syncwarp();
     }
 }
 
@@ -252,20 +326,21 @@ __global__ void __launch_bounds__(PNT) k_sel_apply(ParseArgs P, const uint64_t* 
     }
 }
 
-// one warp per selected line: the gsnp_reads arrays
+// one 8-lane group per selected line (four lines in flight per warp): the gsnp_reads arrays.
+// Lane `sub` converts bytes [16 sub + 128 k, +16) of the sequence and of the quality string.
 __global__ void __launch_bounds__(PNT) k_parse_emit(ParseArgs P, uint64_t n_sel, uint64_t n_bases) {
-    const int lane = threadIdx.x & 31;
-    const uint64_t nw = (uint64_t)gridDim.x * (PNT / 32);
+    const int lane = threadIdx.x & 31, sub = lane & (PG - 1);
+    const uint64_t ngroups = (uint64_t)gridDim.x * PGROUPS;
     int err = 0;
     unsigned long long bad = ~0ull;
-    for (uint64_t l = (uint64_t)blockIdx.x * (PNT / 32) + (threadIdx.x >> 5); l < P.n_lines; l += nw) {
+    for (uint64_t l = (uint64_t)blockIdx.x * PGROUPS + threadIdx.x / PG; l < P.n_lines; l += ngroups) {
         const uint64_t m = P.meta[l];
         if (!sel_of(m)) continue;
         const uint64_t r = P.ridx[l], o = P.boff[l];
         const uint32_t len = (uint32_t)len_of(m);
         const uint8_t* seq = P.text + P.ls[l] + (m >> 32);
         const uint8_t* qual = seq + len + 1;
-        if (lane == 0) {
+        if (sub == 0) {
             P.o_pos[r] = P.pos[l];
             P.o_len[r] = (uint16_t)len;
             P.o_off[r] = o;
@@ -274,18 +349,28 @@ __global__ void __launch_bounds__(PNT) k_parse_emit(ParseArgs P, uint64_t n_sel,
             if (r + 1 == n_sel) P.o_off[n_sel] = n_bases;
         }
         bool good = true;
-        for (uint32_t i = lane; i < len; i += 32) {
-            const uint32_t c = seq[i] & 0xDFu;            // upper case
-            const uint32_t code = c == 'A' ? 0u : c == 'C' ? 1u : c == 'T' ? 2u : c == 'G' ? 3u
-                                : c == 'N' ? 4u : 255u;
-            const uint32_t qc = qual[i];
-            good &= code != 255u && qc >= P.q_offset && qc - P.q_offset <= 63u;
-            P.o_bases[o + i] = (uint8_t)code;
-            P.o_quals[o + i] = (uint8_t)(qc - P.q_offset);
+        for (uint32_t i0 = 16 * sub; i0 < len; i0 += 16 * PG) {
+            uint8_t cs[16], cq[16];
+#pragma unroll
+            for (int k = 0; k < 16; ++k) {
+                cs[k] = i0 + k < len ? seq[i0 + k] : 'A';
+                cq[k] = i0 + k < len ? qual[i0 + k] : (uint8_t)P.q_offset;
+            }
+#pragma unroll
+            for (int k = 0; k < 16; ++k) {
+                if (i0 + k >= len) break;
+                const uint32_t c = cs[k] & 0xDFu;                  // upper case
+                const uint32_t code = c == 'A' ? 0u : c == 'C' ? 1u : c == 'T' ? 2u : c == 'G' ? 3u
+                                    : c == 'N' ? 4u : 255u;
+                const uint32_t qc = cq[k];
+                good &= code != 255u && qc >= P.q_offset && qc - P.q_offset <= 63u;
+                P.o_bases[o + i0 + k] = (uint8_t)code;
+                P.o_quals[o + i0 + k] = (uint8_t)(qc - P.q_offset);
+            }
         }
-        if (!__all_sync(FULL, good)) { err = ERR_PARSE; bad = min(bad, (unsigned long long)l); }
+        if (!good) { err = ERR_PARSE; bad = min(bad, (unsigned long long)l); }
     }
-    if (err && lane == 0) {
+    if (err) {
         atomicOr(P.err, err);
         atomicMin(P.bad_line, bad);
     }
