@@ -145,7 +145,7 @@ __device__ __forceinline__ uint64_t group_sum(uint64_t v) {
 }
 
 __global__ void __launch_bounds__(PNT) k_parse_meta(ParseArgs P) {
-    __shared__ __align__(16) uint8_t stage_s[PGROUPS][PSTAGE];
+    __shared__ __align__(16) uint8_t stage_s[PGROUPS][PSTAGE + 32];    // + the scan's overhang
     __shared__ uint64_t tab_s[PGROUPS][9];
     const int lane = threadIdx.x & 31, sub = lane & (PG - 1), g = threadIdx.x / PG;
     const int gbase = lane & ~(PG - 1);                       // first lane of this group
@@ -235,7 +235,8 @@ __global__ void __launch_bounds__(PNT) k_parse_meta(ParseArgs P) {
             if (eq)
                 for (uint32_t i = sub; i < P.chr_len; i += PG) eq &= at(ca + i) == P.chr[i];
         }
-        want = want && (__ballot_sync(FULL, !eq) & group_mask(lane)) == 0;
+        const uint32_t neq = __ballot_sync(FULL, !eq);          // every lane votes (no short circuit)
+        want = want && (neq & group_mask(lane)) == 0;
         // numeric fields n_hits (3), len (5), location (8): digits spread over the group
         uint64_t fa[3] = {tab[2] + 1, tab[4] + 1, tab[7] + 1};
         uint64_t fb[3] = {tab[3], tab[5], ntab >= 9 ? tab[8] : b};
