@@ -13,7 +13,8 @@
 //   k_sel_tiles / k_scan_partials / k_sel_apply   read index and base offset of every selected
 //                      line (exclusive scans of 1 and len over the lines of the wanted chr)
 //   k_parse_emit       one 8-lane group per selected line: pos/len/strand/hits, off[], and the
-//                      sequence / quality characters converted to codes (16 bytes per lane)
+//                      sequence / quality strings staged in shared memory and converted to codes
+//                      four characters per 32-bit store
 #pragma once
 
 namespace gsnp_dev {
@@ -201,15 +202,19 @@ __global__ void __launch_bounds__(PNT) k_parse_meta(ParseArgs P) {
                     const uint4 y = *reinterpret_cast<const uint4*>(buf + (q0 - A0) + 16);
                     const uint32_t w[8] = {x.x, x.y, x.z, x.w, y.x, y.y, y.z, y.w};
 #pragma unroll
-                    for (int k = 0; k < 32; ++k)
-                        m |= (((w[k >> 2] >> (8 * (k & 3))) & 255u) == 9u) ? 1u << k : 0u;
+                    for (int j = 0; j < 8; ++j) {          // byte == '\t' -> bit, 4 per word
+                        const uint32_t e = __vcmpeq4(w[j], 0x09090909u) & 0x01010101u;
+                        m |= ((e * 0x00204081u) >> 21 & 15u) << (4 * j);
+                    }
                 } else if (!fast) {
                     for (int k = 0; k < 32; ++k)
                         if (q0 + k < b && P.text[q0 + k] == '\t') m |= 1u << k;
                 }
                 // keep bytes inside [a, b)
-                for (int k = 0; k < 32; ++k)
-                    if (q0 + k < a || q0 + k >= b) m &= ~(1u << k);
+                const uint64_t lo = q0 < a ? a - q0 : 0, hi = b > q0 ? b - q0 : 0;
+                const uint32_t keep_hi = hi >= 32 ? ~0u : (1u << hi) - 1u;
+                const uint32_t keep_lo = lo >= 32 ? 0u : ~((1u << lo) - 1u);
+                m &= keep_hi & keep_lo;
             }
             uint32_t cnt = __popc(m), inc = cnt;
 #pragma unroll
@@ -328,51 +333,93 @@ __global__ void __launch_bounds__(PNT) k_sel_apply(ParseArgs P, const uint64_t* 
 }
 
 // one 8-lane group per selected line (four lines in flight per warp): the gsnp_reads arrays.
-// Lane `sub` converts bytes [16 sub + 128 k, +16) of the sequence and of the quality string.
+// The line's sequence and quality strings are staged in shared memory with 16-byte loads; each
+// lane then converts four characters at a time and writes them as one 32-bit store (the unaligned
+// head and tail bytes of each output run are stored singly).
+__device__ __forceinline__ uint32_t base_code(uint32_t c) {
+    c &= 0xDFu;                                                // upper case
+    return c == 'A' ? 0u : c == 'C' ? 1u : c == 'T' ? 2u : c == 'G' ? 3u : c == 'N' ? 4u : 255u;
+}
+
 __global__ void __launch_bounds__(PNT) k_parse_emit(ParseArgs P, uint64_t n_sel, uint64_t n_bases) {
-    const int lane = threadIdx.x & 31, sub = lane & (PG - 1);
+    __shared__ __align__(16) uint8_t stage_s[PGROUPS][2 * 256 + 48];
+    const int lane = threadIdx.x & 31, sub = lane & (PG - 1), g = threadIdx.x / PG;
+    uint8_t* buf = stage_s[g];
     const uint64_t ngroups = (uint64_t)gridDim.x * PGROUPS;
-    int err = 0;
+    bool good = true;
     unsigned long long bad = ~0ull;
-    for (uint64_t l = (uint64_t)blockIdx.x * PGROUPS + threadIdx.x / PG; l < P.n_lines; l += ngroups) {
-        const uint64_t m = P.meta[l];
-        if (!sel_of(m)) continue;
-        const uint64_t r = P.ridx[l], o = P.boff[l];
+    for (uint64_t l0 = (uint64_t)blockIdx.x * PGROUPS + (threadIdx.x / 32) * (32 / PG);
+         __any_sync(FULL, l0 + (lane / PG) < P.n_lines); l0 += ngroups) {
+        const uint64_t l = l0 + (lane / PG);
+        uint64_t m = 0, r = 0, o = 0, sp = 0;
+        if (l < P.n_lines) {
+            m = P.meta[l];
+            if (sel_of(m)) { r = P.ridx[l]; o = P.boff[l]; sp = P.ls[l] + (m >> 32); }
+        }
+        const bool act = sel_of(m) != 0;
         const uint32_t len = (uint32_t)len_of(m);
-        const uint8_t* seq = P.text + P.ls[l] + (m >> 32);
-        const uint8_t* qual = seq + len + 1;
-        if (sub == 0) {
-            P.o_pos[r] = P.pos[l];
-            P.o_len[r] = (uint16_t)len;
-            P.o_off[r] = o;
-            P.o_strand[r] = (uint8_t)((m >> 9) & 1u);
-            P.o_hits[r] = (uint16_t)((m >> 11) & 0xFFFFu);
-            if (r + 1 == n_sel) P.o_off[n_sel] = n_bases;
-        }
-        bool good = true;
-        for (uint32_t i0 = 16 * sub; i0 < len; i0 += 16 * PG) {
-            uint8_t cs[16], cq[16];
+        // stage seq '\t' qual: bytes [S0, sp + 2 len + 1) with S0 = sp rounded down to 16
+        const uint64_t S0 = sp & ~15ull, S1 = sp + 2 * (uint64_t)len + 1;
+        const uint32_t nchunk = act ? (uint32_t)((S1 - S0 + 15) / 16) : 0u;   // <= 33
 #pragma unroll
-            for (int k = 0; k < 16; ++k) {
-                cs[k] = i0 + k < len ? seq[i0 + k] : 'A';
-                cq[k] = i0 + k < len ? qual[i0 + k] : (uint8_t)P.q_offset;
-            }
-#pragma unroll
-            for (int k = 0; k < 16; ++k) {
-                if (i0 + k >= len) break;
-                const uint32_t c = cs[k] & 0xDFu;                  // upper case
-                const uint32_t code = c == 'A' ? 0u : c == 'C' ? 1u : c == 'T' ? 2u : c == 'G' ? 3u
-                                    : c == 'N' ? 4u : 255u;
-                const uint32_t qc = cq[k];
-                good &= code != 255u && qc >= P.q_offset && qc - P.q_offset <= 63u;
-                P.o_bases[o + i0 + k] = (uint8_t)code;
-                P.o_quals[o + i0 + k] = (uint8_t)(qc - P.q_offset);
+        for (int k = 0; k < 5; ++k) {
+            const uint32_t c = sub + PG * k;
+            if (c < nchunk) {
+                const uint64_t q = S0 + 16 * (uint64_t)c;
+                uint4 v;
+                if (q + 16 <= P.n_bytes) v = *reinterpret_cast<const uint4*>(P.text + q);
+                else {
+                    uint32_t w[4] = {0, 0, 0, 0};
+                    for (uint64_t i = q; i < P.n_bytes; ++i) w[(i - q) >> 2] |= (uint32_t)P.text[i] << (8 * ((i - q) & 3));
+                    v = make_uint4(w[0], w[1], w[2], w[3]);
+                }
+                *reinterpret_cast<uint4*>(buf + 16 * c) = v;
             }
         }
-        if (!good) { err = ERR_PARSE; bad = min(bad, (unsigned long long)l); }
+        __syncwarp();
+        if (act) {
+            if (sub == 0) {
+                P.o_pos[r] = P.pos[l];
+                P.o_len[r] = (uint16_t)len;
+                P.o_off[r] = o;
+                P.o_strand[r] = (uint8_t)((m >> 9) & 1u);
+                P.o_hits[r] = (uint16_t)((m >> 11) & 0xFFFFu);
+                if (r + 1 == n_sel) P.o_off[n_sel] = n_bases;
+            }
+            const uint32_t sb = (uint32_t)(sp - S0), qb = sb + len + 1;
+            // word stores need bases and quals equally aligned (else every byte singly)
+            const uintptr_t ab = reinterpret_cast<uintptr_t>(P.o_bases + o);
+            const bool words = ((ab ^ reinterpret_cast<uintptr_t>(P.o_quals + o)) & 3) == 0;
+            const uint32_t head = words ? min(len, (uint32_t)((4u - (uint32_t)(ab & 3)) & 3u)) : len;
+            const uint32_t nw = (len - head) / 4, tail0 = head + 4 * nw;
+            const uint32_t qo = P.q_offset;
+            // single bytes: head [0, head) and tail [tail0, len): at most 6, one per lane
+            for (uint32_t t = sub; t < head + (len - tail0); t += PG) {     // <= 6, or all if !words
+                const uint32_t i = t < head ? t : tail0 + (t - head);
+                const uint32_t bc = base_code(buf[sb + i]), qc = buf[qb + i];
+                good &= bc != 255u && qc >= qo && qc - qo <= 63u;
+                P.o_bases[o + i] = (uint8_t)bc;
+                P.o_quals[o + i] = (uint8_t)(qc - qo);
+            }
+            for (uint32_t wi = sub; wi < nw; wi += PG) {
+                const uint32_t i = head + 4 * wi;
+                uint32_t wb = 0, wq = 0;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const uint32_t bc = base_code(buf[sb + i + k]), qc = buf[qb + i + k];
+                    good &= bc != 255u && qc >= qo && qc - qo <= 63u;
+                    wb |= (bc & 255u) << (8 * k);
+                    wq |= ((qc - qo) & 255u) << (8 * k);
+                }
+                *reinterpret_cast<uint32_t*>(P.o_bases + o + i) = wb;
+                *reinterpret_cast<uint32_t*>(P.o_quals + o + i) = wq;
+            }
+            if (!good) bad = min(bad, (unsigned long long)l);
+        }
+        __syncwarp();
     }
-    if (err) {
-        atomicOr(P.err, err);
+    if (!good) {
+        atomicOr(P.err, ERR_PARSE);
         atomicMin(P.bad_line, bad);
     }
 }
