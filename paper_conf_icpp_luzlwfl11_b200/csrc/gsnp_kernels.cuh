@@ -782,19 +782,22 @@ __device__ __forceinline__ void sort_column(uint32_t* colp, uint32_t n) {
 // C6-C9 for one site held by one thread: priors, posterior, top-2, rank-sum pieces, record.
 // SORTED: the column holds the site's keys in canonical order (rank-sum by one merge).
 template <bool DBG, bool SORTED>
-__device__ __forceinline__ void thread_finish(const CallArgs& A, const uint32_t* colp,
+// lps: the novel log10 prior rows (R6) staged in shared memory; rt: the site's reference byte
+// (code | known << 3), loaded when the site's group was taken.
+__device__ __forceinline__ void thread_finish(const CallArgs& A, const double* lps, uint32_t rt,
+                                              const uint32_t* colp,
                                               uint64_t site, uint32_t n, const double* acc,
                                               uint64_t cu, uint64_t qs, uint32_t ca0,
                                               uint32_t ca1, uint32_t ca2, uint32_t ca3,
                                               uint32_t rep) {
     // C6/C7: priors, posterior, top-2
-    int refb;
-    const int64_t kidx = site_ref(A, site, refb);
-    const double* prow = kidx >= 0 ? A.known_lp + kidx * 10 : A.LP + refb * 10;
+    const int refb = (int)(rt & 7u);
+    const int64_t kidx = (rt & 8u) ? (int64_t)lower_bound_u64(A.known_pos, 0, A.n_known, site) : -1;
+    const double* prow = kidx >= 0 ? A.known_lp + kidx * 10 : lps + refb * 10;
     double lp[10], m = -INFINITY;
 #pragma unroll
     for (int j = 0; j < 10; ++j) {
-        lp[j] = acc[j] + __ldg(prow + j);
+        lp[j] = acc[j] + prow[j];
         m = lp[j] > m ? lp[j] : m;
     }
     int t1, t2;
@@ -872,7 +875,8 @@ __device__ __forceinline__ void thread_finish(const CallArgs& A, const uint32_t*
 }
 
 template <bool DBG>
-__device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* adj, uint32_t* colp,
+__device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* adj, const double* lps,
+                                            uint32_t rt, uint32_t* colp,
                                             uint64_t site, uint32_t n, bool slow_pcr, uint32_t ca0,
                                             uint32_t ca1, uint32_t ca2, uint32_t ca3, uint32_t rep) {
     if (DBG && A.dbg_keys_sorted) {
@@ -932,7 +936,7 @@ __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* ad
         add_row(T, (int)L, kk >> 17, key_cyc(kk), key_base(kk), acc);
     }
 #endif
-    thread_finish<DBG, true>(A, colp, site, n, acc, cu, qs, ca0, ca1, ca2, ca3, rep);
+    thread_finish<DBG, true>(A, lps, rt, colp, site, n, acc, cu, qs, ca0, ca1, ca2, ca3, rep);
 }
 
 // Deep thread path (32 < n <= 32*NCH, kernels built with 128 slots per site): each 32-key chunk
@@ -940,6 +944,7 @@ __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* ad
 // canonical order straight into Alg. 4 (q_adj and the Alg. 3 row per key).
 template <bool DBG, int NCH>
 __device__ __forceinline__ void thread_site_deep(const CallArgs& A, const uint8_t* adj,
+                                                 const double* lps, uint32_t rt,
                                                  uint32_t* colp, uint64_t site, uint32_t n,
                                                  uint32_t ca0, uint32_t ca1, uint32_t ca2,
                                                  uint32_t ca3, uint32_t rep) {
@@ -981,7 +986,7 @@ __device__ __forceinline__ void thread_site_deep(const CallArgs& A, const uint8_
         cu += 1ull << (16 * b);
         qs += (uint64_t)q << (16 * b);
     }
-    thread_finish<DBG, false>(A, colp, site, n, acc, cu, qs, ca0, ca1, ca2, ca3, rep);
+    thread_finish<DBG, false>(A, lps, rt, colp, site, n, acc, cu, qs, ca0, ca1, ca2, ca3, rep);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1448,6 +1453,8 @@ k_call_tile(CallArgs A, uint32_t* wlist, uint32_t* wlist_n, uint32_t* work, uint
     call_smem_bytes(A.L, adj_bytes, CC, &sm, smem);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     for (size_t i = tid; i < adj_bytes; i += NT) sm.adj[i] = A.adj[i];
+    __shared__ double lp_s[50];                             // novel log10 priors [ref][n] (R6)
+    for (int i = tid; i < 50; i += NT) lp_s[i] = A.LP[i];
     const uint8_t* adj = adj_smem ? sm.adj : A.adj;
     uint32_t* colp = sm.col + tid;                           // this lane's column
     __syncthreads();
@@ -1469,6 +1476,7 @@ k_call_tile(CallArgs A, uint32_t* wlist, uint32_t* wlist_n, uint32_t* work, uint
     const uint64_t g0 = A.w0 + grp * 32;                     // first site of the group
     const uint64_t site = g0 + lane;
     const bool active = site < A.w1;
+    const uint32_t rt = active ? A.ref[site - A.origin] : 4u;   // issued early, used at the end
 
     // ---- counting + base_word gather, one site per lane.  The warp
     // walks the reads covering its 32 sites: metadata of 32 reads is loaded coalesced and
@@ -1586,9 +1594,9 @@ k_call_tile(CallArgs A, uint32_t* wlist, uint32_t* wlist_n, uint32_t* work, uint
     if (small) {
         if (maxn <= 16) sort_column<16>(colp, n);
         else sort_column<32>(colp, n);
-        thread_site<DBG>(A, adj, colp, site, n, slow_pcr, ca0, ca1, ca2, ca3, rep);
+        thread_site<DBG>(A, adj, lp_s, rt, colp, site, n, slow_pcr, ca0, ca1, ca2, ca3, rep);
     } else if (mid) {
-        thread_site_deep<DBG, CC / 32>(A, adj, colp, site, n, ca0, ca1, ca2, ca3, rep);
+        thread_site_deep<DBG, CC / 32>(A, adj, lp_s, rt, colp, site, n, ca0, ca1, ca2, ca3, rep);
     }
     __syncwarp();
 
