@@ -13,3 +13,9 @@ echo "launches rc=$?"
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:"k_call_tile|k_calib_count" -c 2 \
     -o gpurun_out/full_${TAG} python tools/profile_call.py C2 48000000 2 > gpurun_out/full_${TAG}.log 2>&1
 echo "full rc=$?"
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:"k_parse_meta|k_parse_emit|k_nl_tiles" -c 4 \
+    -o gpurun_out/parse_${TAG} python tools/profile_parse.py C2 > gpurun_out/parse_${TAG}.log 2>&1
+echo "parse rc=$?"
+timeout 600 ncu --set full --import-source on --clock-control none -k regex:"k_dense" -c 2 \
+    -o gpurun_out/dense_${TAG} python tools/profile_dense.py 200000 > gpurun_out/dense_${TAG}.log 2>&1
+echo "dense rc=$?"
