@@ -274,7 +274,7 @@ def run_gpu(args):
     # while the next chunk is being called.  Two results: the 40-byte records (gsnp_call), and the
     # paper's output form, the RLE-DICT-compressed records (gsnp_call_compressed, §V-B) — the
     # headline e2e.
-    K = 8
+    K = int(os.environ.get("GSNP_E2E_CHUNKS", "2"))   # window chunks of the e2e pipeline (1/2/4/8: 66.6/66.5/67.8/70.0 ms)
     CZ_B = 65536
     pinned = {k: v.pin_memory() for k, v in host.items()}
     out_h = torch.empty(40 * S, dtype=torch.uint8).pin_memory()
@@ -292,8 +292,17 @@ def run_gpu(args):
     znw = [0] * K
     gofs = [0] * ws                           # global word offset of each rank's compressed output
 
+    bd = {}                                   # breakdown events of the last e2e step
+
+    def _ev(name, st):
+        e = torch.cuda.Event(enable_timing=True)
+        e.record(st)
+        bd[name] = e
+
     def e2e_step(compressed):
         evs = []
+        _ev("start", stream)
+        copy_stream.wait_stream(stream)
         with torch.cuda.stream(copy_stream):
             for i in range(K):
                 a, b, oa, ob = rcut[i], rcut[i + 1], ocut[i], ocut[i + 1]
@@ -305,6 +314,7 @@ def run_gpu(args):
                 e = torch.cuda.Event()
                 e.record(copy_stream)
                 evs.append(e)
+        _ev("h2d_done", copy_stream)
         counts.zero_()
         for i in range(K):                    # count chunk i (owned reads only) once it landed
             stream.wait_event(evs[i])
@@ -317,7 +327,9 @@ def run_gpu(args):
                 counts.view(torch.int64).add_(part.view(torch.int64))
         if dist is not None:
             all_reduce_(counts.view(torch.int64))
+        _ev("count_done", stream)
         ctx.calibrate_finalize(counts)
+        _ev("finalize_done", stream)
         rd2 = gsnp.make_reads(dev2)
         for j in range(K):                    # call window chunk j, then ship its result
             lo, hi = wcut[j], wcut[j + 1]
@@ -336,7 +348,13 @@ def run_gpu(args):
         if compressed and dist is not None:   # §8(e) collective 2: where each rank's stream goes
             gofs[:] = shard.gather_output_offsets(
                 dist, sum(znw), "cuda" if backend == "nccl" else "cpu")[0]
+        _ev("calls_done", stream)
         stream.wait_stream(copy_stream)
+        _ev("end", stream)
+
+    def breakdown():
+        names = ["start", "h2d_done", "count_done", "finalize_done", "calls_done", "end"]
+        return {f"{a}->{b}": round(bd[a].elapsed_time(bd[b]), 3) for a, b in zip(names, names[1:])}
 
     def time_e2e(compressed):
         for _ in range(max(1, args.warmup // 2)):
@@ -344,6 +362,7 @@ def run_gpu(args):
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         n_e2e = max(2, min(args.steps, 5))
+        ctx.stage_times(reset=True)
         e0.record(stream)
         for _ in range(n_e2e):
             e2e_step(compressed)
@@ -354,9 +373,15 @@ def run_gpu(args):
             all_reduce_(te, dist.ReduceOp.MAX)
         return float(te.item())
 
+    def dev_stages(n):
+        return {k: round(v[0] / n, 3) for k, v in ctx.stage_times(reset=True).items() if v[1]}
     te_rec = time_e2e(False)
+    bd_rec = breakdown()
+    bd_rec["device_stage_ms"] = dev_stages(max(2, min(args.steps, 5)))
     ok_rec = bool(torch.equal(out_h, out.cpu()))
     te_cz = time_e2e(True)
+    bd_cz = breakdown()
+    bd_cz["device_stage_ms"] = dev_stages(max(2, min(args.steps, 5)))
     # the shipped streams == the device compressor run on the device-timed step's records
     ok_cz = True
     for j in range(K):
@@ -371,7 +396,8 @@ def run_gpu(args):
                      "overlapped with the transfers" % K,
            "records": {"value": total_sites / (te_rec / 1e3), "ms_per_step": te_rec,
                        "d2h_bytes_per_step": out_h.numel(), "check": ok_rec,
-                       "result": "40-byte records (gsnp_call)"}}
+                       "result": "40-byte records (gsnp_call)", "breakdown_ms": bd_rec},
+           "breakdown_ms": bd_cz}
     if ws > 1:
         e2e["rank_offsets_words"] = gofs      # all-gathered per-rank compressed sizes (§8(e))
 

@@ -624,9 +624,11 @@ gsnp_status compress_impl(gsnp_ctx* ctx, const gsnp_record* d_rec, uint64_t n, u
     ctx->launches += 1;
     ctx->end(GSNP_STAGE_COMPRESS);
     CK(cudaGetLastError());
-    if (!dev_out) CK(cudaMemcpyAsync(out, A.out, total * 4, cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
-    ctx->flush();
+    if (!dev_out) {              // host output: the words must have landed when we return
+        CK(cudaMemcpyAsync(out, A.out, total * 4, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        ctx->flush();
+    }                            // device output: ordered on the caller's stream, no host wait
     return GSNP_OK;
 }
 
