@@ -158,7 +158,7 @@ __global__ void __launch_bounds__(DENSE_NT) k_dense_sites(DenseArgs D) {
                 m = lp[j] > m ? lp[j] : m;
             }
             int t1, t2;
-            top2(lp, t1, t2);
+            const double delta = top2(lp, t1, t2);
             double esum = 0.0;
 #pragma unroll
             for (int j = 0; j < 10; ++j)
@@ -178,7 +178,7 @@ __global__ void __launch_bounds__(DENSE_NT) k_dense_sites(DenseArgs D) {
                 }
             }
             const uint32_t* cn = D.cnt + s * 5;
-            site_record(A, site, refb, kidx >= 0, t1, lp[t1] - lp[t2], 1.0 / esum, cu[0], cu[1],
+            site_record(A, site, refb, kidx >= 0, t1, delta, 1.0 / esum, cu[0], cu[1],
                         cu[2], cu[3], qs[0], qs[1], qs[2], qs[3], cn[0], cn[1], cn[2], cn[3], cn[4],
                         wsum, tie);
         }

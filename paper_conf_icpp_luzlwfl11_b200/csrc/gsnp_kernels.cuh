@@ -617,14 +617,20 @@ __device__ __forceinline__ uint32_t pick4(uint32_t v0, uint32_t v1, uint32_t v2,
 }
 __device__ __forceinline__ uint32_t f16(uint64_t pack, int b) { return (uint32_t)(pack >> (16 * b)) & 0xFFFFu; }
 
-// Top-2 genotypes over lp (ties -> lowest n, R7).
-__device__ __forceinline__ void top2(const double* lp, int& t1, int& t2) {
+// Top-2 genotypes over lp (ties -> lowest n, R7); returns lp[t1] - lp[t2].  The best values
+// are carried in registers (no dynamic index into lp, which would put lp in local memory).
+__device__ __forceinline__ double top2(const double* lp, int& t1, int& t2) {
+    double v1 = lp[0];
     t1 = 0;
 #pragma unroll
-    for (int k = 1; k < 10; ++k) if (lp[k] > lp[t1]) t1 = k;
-    t2 = t1 == 0 ? 1 : 0;
+    for (int k = 1; k < 10; ++k)
+        if (lp[k] > v1) { v1 = lp[k]; t1 = k; }
+    double v2 = 0.0;
+    t2 = -1;
 #pragma unroll
-    for (int k = 0; k < 10; ++k) if (k != t1 && lp[k] > lp[t2]) t2 = k;
+    for (int k = 0; k < 10; ++k)
+        if (k != t1 && (t2 < 0 || lp[k] > v2)) { v2 = lp[k]; t2 = k; }
+    return v1 - v2;
 }
 
 // genotype n -> alleles, Alg. 4 lines 13-17 order (AA AC AT AG CC CT CG TT TG GG)
@@ -801,7 +807,7 @@ __device__ __forceinline__ void thread_finish(const CallArgs& A, const double* l
         m = lp[j] > m ? lp[j] : m;
     }
     int t1, t2;
-    top2(lp, t1, t2);
+    const double delta = top2(lp, t1, t2);
     // posterior denominator in genotype order; a term below 1e-18 of the maximum cannot change
     // the double sum (every term is <= 1 and the maximum's term is exactly 1), so it is skipped
     // unless the debug dump wants every posterior
@@ -869,7 +875,7 @@ __device__ __forceinline__ void thread_finish(const CallArgs& A, const double* l
             if (A.dbg_post10) A.dbg_post10[s * 10 + j] = exp10(lp[j] - m) / esum;
         }
     }
-    site_record(A, site, refb, kidx >= 0, t1, lp[t1] - lp[t2], 1.0 / esum, f16(cu, 0), f16(cu, 1),
+    site_record(A, site, refb, kidx >= 0, t1, delta, 1.0 / esum, f16(cu, 0), f16(cu, 1),
                 f16(cu, 2), f16(cu, 3), f16(qs, 0), f16(qs, 1), f16(qs, 2), f16(qs, 3), ca0, ca1,
                 ca2, ca3, rep, wsum, tie);
 }
@@ -1011,7 +1017,7 @@ __device__ __forceinline__ void group_epilogue(const CallArgs& A, uint64_t site,
         m = lp[n] > m ? lp[n] : m;
     }
     int t1, t2;
-    top2(lp, t1, t2);
+    const double delta = top2(lp, t1, t2);
     double x = -INFINITY;                         // genotype n handled by lane n
 #pragma unroll
     for (int n = 0; n < 10; ++n) if (lane == n) x = lp[n] - m;
@@ -1023,7 +1029,7 @@ __device__ __forceinline__ void group_epilogue(const CallArgs& A, uint64_t site,
     if (lane == 0) {
         if (A.dbg_L10)
             for (int k = 0; k < 10; ++k) A.dbg_L10[(site - A.w0) * 10 + k] = L10[k];
-        site_record(A, site, refb, kidx >= 0, t1, lp[t1] - lp[t2], 1.0 / esum, cu[0], cu[1],
+        site_record(A, site, refb, kidx >= 0, t1, delta, 1.0 / esum, cu[0], cu[1],
                     cu[2], cu[3], qs[0], qs[1], qs[2], qs[3], ca0, ca1, ca2, ca3, rep, wsum, tie);
     }
 }
