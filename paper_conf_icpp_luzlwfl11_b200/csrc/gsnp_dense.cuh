@@ -34,7 +34,7 @@ struct DenseArgs {
 };
 
 // counting: every base of every read that can touch [c0, c1)
-__global__ void __launch_bounds__(DENSE_NT) k_dense_count(DenseArgs D) {
+__global__ void __launch_bounds__(DENSE_NT) k_dense_count(const __grid_constant__ DenseArgs D) {
     const CallArgs& A = D.A;
     const uint64_t ga = (D.c0 - A.w0) / 32, gb = (D.c1 - 1 - A.w0) / 32;
     const uint64_t ra = A.tile_ra[ga], rb = A.tile_rb[gb];
@@ -69,7 +69,7 @@ __global__ void __launch_bounds__(DENSE_NT) k_dense_count(DenseArgs D) {
 }
 
 // likelihood (Alg. 1) + posterior + record, one warp per site
-__global__ void __launch_bounds__(DENSE_NT) k_dense_sites(DenseArgs D) {
+__global__ void __launch_bounds__(DENSE_NT) k_dense_sites(const __grid_constant__ DenseArgs D) {
     __shared__ uint16_t dep_s[DENSE_NT / 32][512];                 // dep_count[coord<<1|strand]
     __shared__ uint32_t hist_s[DENSE_NT / 32][4][64];              // unique keys per (base, q)
     const CallArgs& A = D.A;

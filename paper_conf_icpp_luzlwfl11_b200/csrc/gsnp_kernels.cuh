@@ -210,7 +210,7 @@ __device__ __forceinline__ void red_shared_inc_if(uint32_t saddr, uint32_t pred)
                  ::"r"(saddr), "r"(pred) : "memory");
 }
 
-__global__ void __launch_bounds__(CAL_NT, 1) k_calib_count(CalibArgs A) {
+__global__ void __launch_bounds__(CAL_NT, 1) k_calib_count(const __grid_constant__ CalibArgs A) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ uint64_t m_desc[2][CAL_MAXB];          // counted reads: rs | stage offset << 32
     __shared__ uint16_t m_ls[2][CAL_MAXB];            // len | strand << 9
@@ -1452,7 +1452,7 @@ struct BigSite {
 #endif
 template <bool DBG, int CC>
 __global__ void __launch_bounds__(NT, GSNP_CALL_MINB)
-k_call_tile(CallArgs A, uint32_t* wlist, uint32_t* wlist_n, uint32_t* work, uint32_t adj_smem) {
+k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist_n, uint32_t* work, uint32_t adj_smem) {
     extern __shared__ __align__(16) unsigned char smem[];
     TileSmem sm;
     const size_t adj_bytes = adj_smem ? (size_t)64 * A.adjP * A.adjG : 0;
@@ -1624,7 +1624,7 @@ k_call_tile(CallArgs A, uint32_t* wlist, uint32_t* wlist_n, uint32_t* work, uint
 // read range, re-gathers the unique keys into its slice of the col region and runs the warp
 // paths (n <= 32*CC) or hands the site to k_big_sites.
 template <int CC>
-__global__ void __launch_bounds__(NT) k_warp_sites(CallArgs A, const uint32_t* wlist,
+__global__ void __launch_bounds__(NT) k_warp_sites(const __grid_constant__ CallArgs A, const uint32_t* wlist,
                                                    const uint32_t* wlist_n, BigSite* big,
                                                    uint32_t* big_n, uint32_t big_cap) {
     extern __shared__ __align__(16) unsigned char smem[];
@@ -1676,7 +1676,7 @@ __global__ void __launch_bounds__(NT) k_warp_sites(CallArgs A, const uint32_t* w
 
 // Sites with more than 1024 unique keys: one CTA per site (persistent loop over the list),
 // keys gathered into a shared buffer of `cap` keys (GSNP_E_CAPACITY beyond it).
-__global__ void __launch_bounds__(NT) k_big_sites(CallArgs A, const BigSite* big,
+__global__ void __launch_bounds__(NT) k_big_sites(const __grid_constant__ CallArgs A, const BigSite* big,
                                                   const uint32_t* big_n, uint32_t cap) {
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ double red[NW * 18];
