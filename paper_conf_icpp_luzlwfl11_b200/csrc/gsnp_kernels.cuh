@@ -516,7 +516,7 @@ __global__ void k_tile_ranges(const uint64_t* pos, uint64_t n, uint64_t w0, uint
 constexpr int TS = NT;
 constexpr int COLS = 32;              // key slots per site, shallow kernel (thread path n <= 32)
 #ifndef GSNP_GB
-#define GSNP_GB 1
+#define GSNP_GB 2
 #endif
 constexpr int GB = GSNP_GB;           // reads whose bytes are in flight together in the gather
 constexpr int COLS_DEEP = 128;        // key slots per site, deep kernel (thread path n <= 128)
