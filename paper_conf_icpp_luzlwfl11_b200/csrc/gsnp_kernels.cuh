@@ -556,7 +556,7 @@ constexpr uint32_t KEY_BSLOT = (3u << 15) | 511u;                               
 #endif
 constexpr int kP2Unroll = GSNP_P2_UNROLL;      // rows in flight per thread in likelihood pass 2
 #ifndef GSNP_FUSED_PASS
-#define GSNP_FUSED_PASS 0
+#define GSNP_FUSED_PASS 1
 #endif
 // read-only 16-byte load that does not allocate in L1 (the table has little L1 reuse)
 __device__ __forceinline__ double2 ld_na(const double2* p) {
