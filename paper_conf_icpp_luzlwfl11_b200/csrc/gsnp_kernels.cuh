@@ -571,9 +571,20 @@ __device__ __forceinline__ double2 ld_na(const double2* p) {
 #define GSNP_T256 1
 #endif
 constexpr int TROW = GSNP_T256 ? 12 : 10;
+#ifndef GSNP_T_HINT
+#define GSNP_T_HINT 1
+#endif
 __device__ __forceinline__ void ld256(const double* p, double& a, double& b, double& c, double& d) {
+#if GSNP_T_HINT == 1      // rows do not allocate in L1 (little reuse; keeps the read bytes there)
+    asm volatile("ld.global.nc.L1::no_allocate.v4.f64 {%0, %1, %2, %3}, [%4];"
+                 : "=d"(a), "=d"(b), "=d"(c), "=d"(d) : "l"(p));
+#elif GSNP_T_HINT == 2    // rows marked evict-last in L2 (the table stays resident)
+    asm volatile("ld.global.nc.L2::evict_last.v4.f64 {%0, %1, %2, %3}, [%4];"
+                 : "=d"(a), "=d"(b), "=d"(c), "=d"(d) : "l"(p));
+#else
     asm volatile("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];"
                  : "=d"(a), "=d"(b), "=d"(c), "=d"(d) : "l"(p));
+#endif
 }
 __device__ __forceinline__ void add_row(const double* __restrict__ T, int L, uint32_t qa,
                                         uint32_t cyc, uint32_t b, double* acc) {
