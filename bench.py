@@ -428,7 +428,7 @@ def run_gpu(args):
     # Alg. 1 over per-site dense base_occ arrays (gsnp_call_dense) vs the sparse path, same
     # sub-window of this shard, same records.  CUDA events on the library's stream.
     dense = None
-    if not args.no_dense:
+    if not args.no_dense and ws == 1:         # side legs (outside the step) at N=1 only
         dlo = w0 + min(S // 4, 8_000_000)
         dhi = min(w1, dlo + (1 << 22))
         nd = dhi - dlo
@@ -466,7 +466,7 @@ def run_gpu(args):
     # ---- §8(f) NEXT #2, outside the step: input packing on the GPU — this shard's reads as SOAP
     # alignment text (resident in HBM), parsed into the gsnp_reads arrays (gsnp_parse_soap).
     parse = None
-    if not args.no_parse:
+    if not args.no_parse and ws == 1:
         import synth
         text = synth.soap_text(w, "chr21", 33)
         tdev = torch.frombuffer(bytearray(text), dtype=torch.uint8).cuda()
@@ -538,7 +538,7 @@ def run_gpu(args):
         except Exception:
             traffic = None
     cpu_v, cpu_desc = (None, None)
-    if not args.no_cpu:
+    if not args.no_cpu and ws == 1:            # the oracle baseline: rank 0 at N=1 only
         cpu_v, cpu_desc = cpu_oracle_rate(w, budget_s=args.ref_budget)
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
