@@ -11,6 +11,7 @@
 #include <chrono>
 #include <cmath>
 #include <cstdarg>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <string>
@@ -548,7 +549,9 @@ gsnp_status finalize_impl(gsnp_ctx* ctx, const uint64_t* counts_host) {
             build_T_q(L, p, T, q, c0, std::min(L, c0 + CCH));
         }
     };
-    const int nt = (int)std::max(1u, std::min(32u, std::thread::hardware_concurrency()));
+    static const int nt_env = [] { const char* e = getenv("GSNP_HOST_THREADS"); return e ? atoi(e) : 0; }();
+    const int nt = nt_env > 0 ? nt_env
+                              : (int)std::max(1u, std::min(32u, std::thread::hardware_concurrency()));
     std::vector<std::thread> th;
     for (int i = 1; i < nt; ++i) th.emplace_back(work);
     work();
