@@ -277,19 +277,25 @@ def run_gpu(args):
     # while the next chunk is being called.  Two results: the 40-byte records (gsnp_call), and the
     # paper's output form, the RLE-DICT-compressed records (gsnp_call_compressed, §V-B) — the
     # headline e2e.
-    K = int(os.environ.get("GSNP_E2E_CHUNKS", "2"))   # window chunks of the e2e pipeline (1/2/4/8: 66.6/66.5/67.8/70.0 ms)
+    # e2e pipeline: the reads go up in KR chunks (the calibration counts each chunk as it lands);
+    # the window is called in K chunks of geometrically shrinking size (8:4:2:1), so each chunk's
+    # result download hides under the next chunk's compute and the exposed tail is the smallest
+    KR = int(os.environ.get("GSNP_E2E_READ_CHUNKS", "8"))
+    K = int(os.environ.get("GSNP_E2E_CHUNKS", "4"))
     CZ_B = 65536
     pinned = {k: v.pin_memory() for k, v in host.items()}
     out_h = torch.empty(40 * S, dtype=torch.uint8).pin_memory()
     dev2 = {k: torch.empty_like(v, device="cuda") for k, v in host.items()}
     h2d = sum(v.numel() * v.element_size() for v in pinned.values())
     nr_all = int(len(w["pos"]))
-    rcut = [nr_all * i // K for i in range(K + 1)]
+    rcut = [nr_all * i // KR for i in range(KR + 1)]
     ocut = [int(w["off"][r]) for r in rcut]
-    wcut = [w0 + S * i // K for i in range(K + 1)]
+    wt = [2.0 ** (K - 1 - j) for j in range(K)]
+    wcut = [w0 + int(S * sum(wt[:j]) / sum(wt)) for j in range(K + 1)]
+    wcut[-1] = w1
     copy_stream = torch.cuda.Stream()
     part = torch.zeros_like(counts)
-    zcap = 11 * (S // K + 1) + 4096                 # words per chunk (> raw 10 words/record)
+    zcap = 11 * max(b - a for a, b in zip(wcut, wcut[1:])) + 4096   # words per chunk (> 10/record)
     zdev = torch.empty(K * zcap, dtype=torch.int32, device="cuda")
     zh = torch.empty(K * zcap, dtype=torch.int32).pin_memory()
     znw = [0] * K
@@ -307,7 +313,7 @@ def run_gpu(args):
         _ev("start", stream)
         copy_stream.wait_stream(stream)
         with torch.cuda.stream(copy_stream):
-            for i in range(K):
+            for i in range(KR):
                 a, b, oa, ob = rcut[i], rcut[i + 1], ocut[i], ocut[i + 1]
                 for k in ("pos", "len", "strand", "hits"):
                     dev2[k][a:b].copy_(pinned[k][a:b], non_blocking=True)
@@ -319,7 +325,7 @@ def run_gpu(args):
                 evs.append(e)
         _ev("h2d_done", copy_stream)
         counts.zero_()
-        for i in range(K):                    # count chunk i (owned reads only) once it landed
+        for i in range(KR):                   # count chunk i (owned reads only) once it landed
             stream.wait_event(evs[i])
             a, b = max(rcut[i], ora), min(rcut[i + 1], orb)
             if a < b:
@@ -336,6 +342,7 @@ def run_gpu(args):
         rd2 = gsnp.make_reads(dev2)
         for j in range(K):                    # call window chunk j, then ship its result
             lo, hi = wcut[j], wcut[j + 1]
+            _ev(f"call{j}_start", stream)
             if compressed:
                 znw[j] = ctx.call_compressed(rd2, lo, hi, zdev[j * zcap:(j + 1) * zcap], CZ_B)
                 src, dst = zdev[j * zcap:j * zcap + znw[j]], zh[j * zcap:j * zcap + znw[j]]
@@ -343,6 +350,7 @@ def run_gpu(args):
                 src = out[40 * (lo - w0):40 * (hi - w0)]
                 ctx.call_reads(rd2, lo, hi, src)
                 dst = out_h[40 * (lo - w0):40 * (hi - w0)]
+            _ev(f"call{j}_end", stream)
             e = torch.cuda.Event()
             e.record(stream)
             copy_stream.wait_event(e)
@@ -357,7 +365,10 @@ def run_gpu(args):
 
     def breakdown():
         names = ["start", "h2d_done", "count_done", "finalize_done", "calls_done", "end"]
-        return {f"{a}->{b}": round(bd[a].elapsed_time(bd[b]), 3) for a, b in zip(names, names[1:])}
+        out = {f"{a}->{b}": round(bd[a].elapsed_time(bd[b]), 3) for a, b in zip(names, names[1:])}
+        out["call_spans"] = [round(bd[f"call{j}_start"].elapsed_time(bd[f"call{j}_end"]), 3)
+                             for j in range(K)]
+        return out
 
     def time_e2e(compressed):
         for _ in range(max(1, args.warmup // 2)):
@@ -395,8 +406,8 @@ def run_gpu(args):
     d2h_cz = 4 * sum(znw)
     e2e = {"value": total_sites / (te_cz / 1e3), "unit": UNIT, "h2d_bytes_per_step": h2d,
            "d2h_bytes_per_step": d2h_cz, "ms_per_step": te_cz, "check": ok_cz,
-           "result": "RLE-DICT-compressed records (gsnp_call_compressed, §V-B), %d window chunks "
-                     "overlapped with the transfers" % K,
+           "result": "RLE-DICT-compressed records (gsnp_call_compressed, §V-B), %d read chunks "
+                     "and %d window chunks (8:4:2:1) overlapped with the transfers" % (KR, K),
            "records": {"value": total_sites / (te_rec / 1e3), "ms_per_step": te_rec,
                        "d2h_bytes_per_step": out_h.numel(), "check": ok_rec,
                        "result": "40-byte records (gsnp_call)", "breakdown_ms": bd_rec},

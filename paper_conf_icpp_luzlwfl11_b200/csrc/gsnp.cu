@@ -102,6 +102,11 @@ struct gsnp_ctx {
     DevBuf<uint64_t> cz_off;
     DevBuf<gsnp_record> cz_rec;
     uint64_t* h_cz_total = nullptr;     // pinned
+    // mapped pinned mailbox for the few scalars the host reads on the call path (status flag,
+    // window read range, compressed size): written by k_peek over PCIe with SM stores, so a
+    // caller's large device->host copy in flight on another stream (same DMA engine) cannot
+    // delay the read
+    uint64_t* mbox = nullptr;
     uint64_t launches = 0;
     // per-stage timing (GSNP_TIMING)
     struct Pending { int stage; cudaEvent_t a, b; };
@@ -336,6 +341,24 @@ gsnp_status map_err(gsnp_ctx* ctx, int e) {
     return fail(ctx, GSNP_E_CUDA, "device error flag %d", e);
 }
 
+__global__ void k_peek(uint8_t* dst, const uint8_t* src, uint32_t n) {
+    for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) dst[i] = src[i];
+}
+
+// copy n (<= 8) bytes at device address src into mailbox slot `slot` (read after a sync)
+gsnp_status peek(gsnp_ctx* ctx, int slot, const void* src, uint32_t n) {
+    if (!ctx->mbox) {
+        CK(cudaHostAlloc(&ctx->mbox, 16 * sizeof(uint64_t), cudaHostAllocMapped));
+        memset(ctx->mbox, 0, 16 * sizeof(uint64_t));
+    }
+    ctx->mbox[slot] = 0;
+    k_peek<<<1, 32, 0, ctx->stream>>>(reinterpret_cast<uint8_t*>(ctx->mbox + slot),
+                                      reinterpret_cast<const uint8_t*>(src), n);
+    ctx->launches++;
+    CK(cudaGetLastError());
+    return GSNP_OK;
+}
+
 gsnp_status launch_validate(gsnp_ctx* ctx, const DevReads& d) {
     if (d.n == 0) return GSNP_OK;
     unsigned blocks = (unsigned)((d.n + 255) / 256);
@@ -410,9 +433,12 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
     // deep windows (mean depth >= 48 by read count) keep up to 128 keys per thread
     uint64_t rr[2] = {0, 0};
     if (d.n) {
-        CK(cudaMemcpyAsync(&rr[0], ctx->tile_ra.p, 8, cudaMemcpyDeviceToHost, s));
-        CK(cudaMemcpyAsync(&rr[1], ctx->tile_rb.p + n_groups - 1, 8, cudaMemcpyDeviceToHost, s));
+        gsnp_status pst;
+        if ((pst = peek(ctx, 0, ctx->tile_ra.p, 8))) return pst;
+        if ((pst = peek(ctx, 1, ctx->tile_rb.p + n_groups - 1, 8))) return pst;
         CK(cudaStreamSynchronize(s));
+        rr[0] = ctx->mbox[0];
+        rr[1] = ctx->mbox[1];
     }
     const double depth_est = (double)(rr[1] - rr[0]) * A.L / (double)(w1 - w0);
     const bool deep = depth_est >= 48.0;
@@ -464,8 +490,10 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
 
 gsnp_status read_err(gsnp_ctx* ctx) {
     int h = 0;
-    CK(cudaMemcpyAsync(&h, ctx->d_err.p, sizeof(int), cudaMemcpyDeviceToHost, ctx->stream));
+    gsnp_status pst = peek(ctx, 2, ctx->d_err.p, sizeof(int));
+    if (pst) return pst;
     CK(cudaStreamSynchronize(ctx->stream));
+    memcpy(&h, ctx->mbox + 2, sizeof(int));
     ctx->flush();
     return map_err(ctx, h);
 }
@@ -607,9 +635,10 @@ gsnp_status compress_impl(gsnp_ctx* ctx, const gsnp_record* d_rec, uint64_t n, u
     k_cz_scan<<<1, 1024, 0, s>>>(ctx->cz_meta.p, nblk * NSEC, ctx->cz_off.p);
     ctx->launches += 3;
     CK(cudaGetLastError());
-    CK(cudaMemcpyAsync(ctx->h_cz_total, ctx->cz_off.p + nblk * NSEC, 8, cudaMemcpyDeviceToHost, s));
+    gsnp_status pst = peek(ctx, 3, ctx->cz_off.p + nblk * NSEC, 8);
+    if (pst) return pst;
     CK(cudaStreamSynchronize(s));
-    const uint64_t total = *ctx->h_cz_total;
+    const uint64_t total = ctx->mbox[3];
     if (n_words) *n_words = total;
     if (total > out_cap) {
         ctx->end(GSNP_STAGE_COMPRESS);
@@ -1212,6 +1241,7 @@ void gsnp_destroy(gsnp_ctx* ctx) {
     ctx->cz_cols.release(); ctx->cz_meta.release(); ctx->cz_dD.release(); ctx->cz_dict.release();
     ctx->cz_out.release(); ctx->cz_off.release(); ctx->cz_rec.release();
     if (ctx->h_cz_total) cudaFreeHost(ctx->h_cz_total);
+    if (ctx->mbox) cudaFreeHost(ctx->mbox);
     if (ctx->h_T) cudaFreeHost(ctx->h_T);
     if (ctx->h_cnt_pinned) cudaFreeHost(ctx->h_cnt_pinned);
     for (auto& p : ctx->pending) { cudaEventDestroy(p.a); cudaEventDestroy(p.b); }
