@@ -226,7 +226,10 @@ gsnp_status gsnp_get_tables(gsnp_ctx* ctx, uint64_t* counts, double* p_matrix, d
  *   rec: host or device memory (device: used in place).  out: host or device memory.
  *   out_cap: capacity in words.  *n_words: words of the stream (also on GSNP_E_CAPACITY, when
  *   out_cap is too small; nothing is written then).  out may be NULL with out_cap 0 to query.
- * Every step runs in the library's kernels (k_cz_*); the host only sums two sizes. */
+ * Every step runs in the library's kernels (k_cz_*); the host only reads the total size.
+ * Device output is written stream-ordered on params.stream (the call returns once the size is
+ * known; synchronise that stream, or order work after it, before reading the words); host
+ * output has landed when the call returns. */
 gsnp_status gsnp_compress(gsnp_ctx* ctx, const gsnp_record* rec, uint64_t n, uint32_t block_sites,
                           uint32_t* out, uint64_t out_cap, uint64_t* n_words);
 
