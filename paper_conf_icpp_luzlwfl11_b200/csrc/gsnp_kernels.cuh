@@ -17,7 +17,10 @@
 
 namespace gsnp_dev {
 
-constexpr int NT = 256;               // threads per CTA
+#ifndef GSNP_NT
+#define GSNP_NT 256
+#endif
+constexpr int NT = GSNP_NT;           // threads per CTA
 constexpr int NW = NT / 32;           // warps per CTA
 constexpr uint32_t FULL = 0xFFFFFFFFu;
 constexpr uint32_t KEY_INF = 0xFFFFFFFFu;
