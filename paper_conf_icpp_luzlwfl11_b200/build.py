@@ -7,7 +7,8 @@ import subprocess
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 SRC = os.path.join(HERE, "csrc", "gsnp.cu")
-DEPS = [SRC, os.path.join(HERE, "csrc", "gsnp_kernels.cuh"),
+SRC_DEEP = os.path.join(HERE, "csrc", "gsnp_deep.cu")   # deep-window kernel, 384-thread CTAs
+DEPS = [SRC, SRC_DEEP, os.path.join(HERE, "csrc", "gsnp_kernels.cuh"),
         os.path.join(HERE, "csrc", "gsnp_compress.cuh"), os.path.join(HERE, "csrc", "gsnp_dense.cuh"),
         os.path.join(HERE, "csrc", "gsnp_parse.cuh"),
         os.path.join(ROOT, "include", "gsnp.h")]
@@ -22,7 +23,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     stale = not os.path.exists(LIB) or any(os.path.getmtime(LIB) < os.path.getmtime(d) for d in DEPS)
     if force or stale:
         nvcc = os.environ.get("NVCC", "nvcc")
-        cmd = [nvcc] + NVCC_FLAGS + (["-Xptxas", "-v"] if verbose else []) + ["-o", LIB, SRC]
+        cmd = [nvcc] + NVCC_FLAGS + (["-Xptxas", "-v"] if verbose else []) + ["-o", LIB, SRC, SRC_DEEP]
         subprocess.check_call(cmd)
     return LIB
 

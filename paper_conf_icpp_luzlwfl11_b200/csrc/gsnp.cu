@@ -26,6 +26,12 @@
 
 using namespace gsnp_dev;
 
+namespace gsnp_deep {   // gsnp_deep.cu: the deep-window k_call_tile with 384-thread CTAs
+cudaError_t launch_call_tile_deep(const void* args, size_t args_size, bool dbg, int num_sms,
+                                  size_t adj_bytes, uint32_t adj_smem, uint32_t* wlist,
+                                  uint32_t* wlist_n, uint32_t* work, cudaStream_t s);
+}
+
 namespace {
 
 template <typename T>
@@ -450,18 +456,25 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
     CK(ctx->big_n.ensure(3));
     CK(cudaMemsetAsync(ctx->big_n.p, 0, 12, s));    // [0] big sites, [1] work counter, [2] wlist
     const bool dbg = A.count_only || A.dbg_off || A.dbg_counters || A.dbg_L10 || A.dbg_post10;
-    auto kern = dbg ? (deep ? k_call_tile<true, COLS_DEEP> : k_call_tile<true, COLS>)
-                    : (deep ? k_call_tile<false, COLS_DEEP> : k_call_tile<false, COLS>);
-    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    int per_sm = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NT, smem));
-    const uint64_t want = (uint64_t)g_num_sms * std::max(per_sm, 1);
-    const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, n_tiles));
-    ctx->begin();
-    kern<<<grid, NT, smem, s>>>(A, ctx->wlist.p, ctx->big_n.p + 2, ctx->big_n.p + 1, adj_smem);
-    ctx->end(GSNP_STAGE_CALL);
-    ctx->launches++;
-    CK(cudaGetLastError());
+    if (deep) {
+        ctx->begin();
+        CK(gsnp_deep::launch_call_tile_deep(&A, sizeof A, dbg, g_num_sms, adj_bytes, adj_smem,
+                                            ctx->wlist.p, ctx->big_n.p + 2, ctx->big_n.p + 1, s));
+        ctx->end(GSNP_STAGE_CALL);
+        ctx->launches++;
+    } else {
+        auto kern = dbg ? k_call_tile<true, COLS> : k_call_tile<false, COLS>;
+        CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        int per_sm = 0;
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NT, smem));
+        const uint64_t want = (uint64_t)g_num_sms * std::max(per_sm, 1);
+        const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, n_tiles));
+        ctx->begin();
+        kern<<<grid, NT, smem, s>>>(A, ctx->wlist.p, ctx->big_n.p + 2, ctx->big_n.p + 1, adj_smem);
+        ctx->end(GSNP_STAGE_CALL);
+        ctx->launches++;
+        CK(cudaGetLastError());
+    }
     if (!A.count_only) {
         // listed sites (n > 32 keys, or beyond the deep kernel's thread path): warp per site
         auto wk = deep ? k_warp_sites<COLS_DEEP> : k_warp_sites<COLS>;
