@@ -518,6 +518,9 @@ __global__ void k_tile_ranges(const uint64_t* pos, uint64_t n, uint64_t w0, uint
 // parallelisation).  Shared-memory layout (host: call_smem_bytes()).
 constexpr int TS = NT;
 constexpr int COLS = 32;              // key slots per site, shallow kernel (thread path n <= 32)
+#ifndef GSNP_CLAIM
+#define GSNP_CLAIM 4
+#endif
 #ifndef GSNP_GB
 #define GSNP_GB 2
 #endif
@@ -1481,17 +1484,24 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
     const uint64_t n_groups = (A.w1 - A.w0 + 31) / 32;
     // persistent warps: each takes the next group of 32 consecutive sites from a counter; the
     // next group's index and read range are fetched while the current one is processed
-    uint64_t nxt = 0, nra = 0, nrb = 0;
-    if (lane == 0) nxt = atomicAdd(work, 1u);
+    // groups are claimed GSNP_CLAIM at a time (fewer atomics on the one counter)
+    uint64_t nxt = 0, nra = 0, nrb = 0, claim_end = 0;
+    if (lane == 0) nxt = atomicAdd(work, (uint32_t)GSNP_CLAIM);
     nxt = __shfl_sync(FULL, nxt, 0);
+    claim_end = nxt + GSNP_CLAIM;
     if (nxt < n_groups) { nra = A.tile_ra[nxt]; nrb = A.tile_rb[nxt]; }
     for (;;) {
     const uint64_t grp = nxt;
     if (grp >= n_groups) break;
     const uint64_t wra = nra;
     uint64_t wrb = nrb;
-    if (lane == 0) nxt = atomicAdd(work, 1u);
-    nxt = __shfl_sync(FULL, nxt, 0);
+    if (grp + 1 < claim_end) {
+        nxt = grp + 1;
+    } else {
+        if (lane == 0) nxt = atomicAdd(work, (uint32_t)GSNP_CLAIM);
+        nxt = __shfl_sync(FULL, nxt, 0);
+        claim_end = nxt + GSNP_CLAIM;
+    }
     if (nxt < n_groups) { nra = A.tile_ra[nxt]; nrb = A.tile_rb[nxt]; }
     const uint64_t g0 = A.w0 + grp * 32;                     // first site of the group
     const uint64_t site = g0 + lane;
