@@ -1193,7 +1193,7 @@ __device__ void warp_site(const CallArgs& A, const uint32_t* col, int warp, uint
     double wsum = 0.0, tie = 0.0;
     if ((A.flags & GSNP_RANK_SUM) && a1 != a2 && pick4(cu[0], cu[1], cu[2], cu[3], a1) &&
         pick4(cu[0], cu[1], cu[2], cu[3], a2)) {
-#pragma unroll 1
+#pragma unroll                            // constant indices: key[] stays in registers
         for (int k = 0; k < K; ++k) {
             const uint32_t x = key[k];
             const uint32_t xb = key_base(x), xq = key_q(x);
