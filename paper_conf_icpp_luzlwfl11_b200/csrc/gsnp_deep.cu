@@ -7,7 +7,10 @@
 // the shallow kernel keeps 256-thread CTAs (three per SM).
 #include <cstring>
 
-#define GSNP_NT 384
+#ifndef GSNP_DEEP_NT
+#define GSNP_DEEP_NT 384
+#endif
+#define GSNP_NT GSNP_DEEP_NT
 #define GSNP_CALL_MINB 1
 #define gsnp_dev gsnp_dev384
 #include "gsnp_kernels.cuh"
@@ -25,7 +28,11 @@ cudaError_t launch_call_tile_deep(const void* args, size_t args_size, bool dbg, 
     if (args_size != sizeof(CallArgs)) return cudaErrorInvalidValue;
     CallArgs A;
     memcpy(&A, args, sizeof A);
-    const size_t smem = call_smem_bytes(A.L, adj_smem ? adj_bytes : 0, COLS_DEEP, nullptr, nullptr);
+    size_t smem = call_smem_bytes(A.L, adj_smem ? adj_bytes : 0, COLS_DEEP, nullptr, nullptr);
+    if (adj_smem && smem > 227 * 1024) {     // no room for the adjust table: read it from global
+        adj_smem = 0;
+        smem = call_smem_bytes(A.L, 0, COLS_DEEP, nullptr, nullptr);
+    }
     auto kern = dbg ? k_call_tile<true, COLS_DEEP> : k_call_tile<false, COLS_DEEP>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
