@@ -73,10 +73,12 @@ class Params:
     rank_sum: bool = True
     monoploid: bool = False      # R18: heterozygous genotypes get prior 0
     titv: bool = False           # R18: novel transition:transversion 2:1
+    rank_exact: bool = False     # R20: exact small-sample rank-sum when nothing ties
 
     def c(self) -> _Params:
         return _Params(self.max_read_len, self.q_max, self.het_novel, self.althom_novel,
-                       self.global_dep, self.pcr_dep, self.calib_min_count, int(self.rank_sum),
+                       self.global_dep, self.pcr_dep, self.calib_min_count,
+                       int(self.rank_sum) * (2 if self.rank_exact else 1),
                        int(self.monoploid) | 2 * int(self.titv))
 
 
@@ -104,6 +106,8 @@ def lib():
         L.or_dense_likelihood.argtypes = [PP, P, ctypes.c_uint64, P, P, P, P, P]
         L.or_rank_sum.restype = ctypes.c_double
         L.or_rank_sum.argtypes = [ctypes.c_uint64, P, ctypes.c_uint64, P]
+        L.or_rank_sum_exact.restype = ctypes.c_double
+        L.or_rank_sum_exact.argtypes = [ctypes.c_uint64, P, ctypes.c_uint64, P]
         L.or_call_window.restype = ctypes.c_int
         L.or_call_window.argtypes = [PP, P, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64, P, P,
                                      P, ctypes.POINTER(_Reads), ctypes.c_uint64, ctypes.c_uint64,
@@ -202,6 +206,13 @@ def rank_sum(X, Y) -> float:
     X = np.ascontiguousarray(X, np.uint8)
     Y = np.ascontiguousarray(Y, np.uint8)
     return lib().or_rank_sum(len(X), _p(X), len(Y), _p(Y))
+
+
+def rank_sum_exact(X, Y) -> float:
+    """R20: exact two-sided p when len(X), len(Y) <= 32 and nothing ties, else rank_sum."""
+    X = np.ascontiguousarray(X, np.uint8)
+    Y = np.ascontiguousarray(Y, np.uint8)
+    return lib().or_rank_sum_exact(len(X), _p(X), len(Y), _p(Y))
 
 
 def call_window(P: Params, w: dict, p: np.ndarray, w0: int, w1: int, debug: bool = False):

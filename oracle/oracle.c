@@ -10,7 +10,8 @@
  * or the DESIGN.md reading (R<n>) where the paper is silent.
  *
  * Pins (tests/test_oracle_pins.py): Fig. 3 keys; dense Alg. 1 == sparse Alg. 4; brute-force
- * products vs log-sums; closed forms; scipy's Mann-Whitney asymptotic p; calibration invariants.
+ * products vs log-sums; closed forms; scipy's Mann-Whitney asymptotic and exact p (R20);
+ * calibration invariants.
  * Functions without an external pin say "parity unpinned" in their comment.
  */
 #include <math.h>
@@ -26,7 +27,7 @@ typedef struct {
     double global_dep;       /* R3 global dependency coefficient (linear) */
     double pcr_dep;          /* R3 PCR dependency coefficient (linear) */
     uint32_t calib_min_count;/* R1 tau */
-    uint32_t rank_sum;       /* R8: 1 = apply the rank-sum test to het calls */
+    uint32_t rank_sum;       /* R8: 1 = apply the rank-sum test to het calls; 2 = R20 exact */
     uint32_t prior_mode;     /* R18: bit 0 monoploid, bit 1 ti/tv 2:1 */
 } or_params;
 
@@ -346,6 +347,47 @@ double or_rank_sum(uint64_t n1, const uint8_t* X, uint64_t n2, const uint8_t* Y)
     return erfc(fabs(z) / sqrt(2.0));
 }
 
+/* C8 exact variant (PAPER SILENT, reading R20; SURVEY §8(f) NEXT #4 "exact small-N rank-sum").
+ * When n1, n2 <= 32 and no two pooled qualities tie, W = sum of the integer ranks of X and the
+ * p-value is the definition of the exact two-sided test: under H0 every n1-subset of the ranks
+ * {1..N} is equally likely, so P(W <= w) = #{subsets with rank sum <= w} / C(N, n1).  The subset
+ * counts come from the plain 0/1-knapsack over ranks 1..N (cnt[k][s]: k ranks summing to s).
+ * p = min(1, 2 min(P(W <= w), P(W >= w))).  Otherwise the normal approximation (or_rank_sum). */
+double or_rank_sum_exact(uint64_t n1, const uint8_t* X, uint64_t n2, const uint8_t* Y) {
+    if (n1 == 0 || n2 == 0) return 0.0;
+    if (n1 > 32 || n2 > 32) return or_rank_sum(n1, X, n2, Y);
+    uint64_t N = n1 + n2;
+    for (uint64_t i = 0; i < N; ++i)
+        for (uint64_t j = i + 1; j < N; ++j) {
+            uint8_t a = i < n1 ? X[i] : Y[i - n1], b = j < n1 ? X[j] : Y[j - n1];
+            if (a == b) return or_rank_sum(n1, X, n2, Y);
+        }
+    uint64_t W = 0;
+    for (uint64_t i = 0; i < n1; ++i) {
+        uint64_t less = 0;
+        for (uint64_t j = 0; j < n1; ++j) less += X[j] < X[i];
+        for (uint64_t j = 0; j < n2; ++j) less += Y[j] < X[i];
+        W += less + 1;
+    }
+    uint64_t smax = N * (N + 1) / 2;
+    double* cnt = (double*)calloc((n1 + 1) * (smax + 1), sizeof(double));
+    cnt[0] = 1.0;
+    for (uint64_t r = 1; r <= N; ++r)                   /* add rank r to every subset */
+        for (uint64_t k = (r < n1 ? r : n1); k >= 1; --k)
+            for (uint64_t s = smax; s >= r; --s)
+                cnt[k * (smax + 1) + s] += cnt[(k - 1) * (smax + 1) + s - r];
+    double tot = 0.0, le = 0.0, ge = 0.0;
+    for (uint64_t s = 0; s <= smax; ++s) {
+        double c = cnt[n1 * (smax + 1) + s];
+        tot += c;
+        if (s <= W) le += c;
+        if (s >= W) ge += c;
+    }
+    free(cnt);
+    double p = 2.0 * (le < ge ? le : ge) / tot;
+    return p < 1.0 ? p : 1.0;
+}
+
 /* ------------------------------------------------------------------------------------------
  * One window [w0, w1): C0 gathering, then per site C2..C9.  Optional debug outputs (may be NULL):
  *   off[S+1] (u32 CSR offsets of keys), keys_sorted, counters[S][15] =
@@ -450,7 +492,8 @@ int or_call_window(const or_params* P, const uint8_t* ref, uint64_t n_sites, uin
                 if (bb[k] == a1) X[nx++] = qq[k];
                 else if (bb[k] == a2) Y[ny++] = qq[k];
             }
-            rank_p = or_rank_sum(nx, X, ny, Y);
+            rank_p = P->rank_sum == 2 ? or_rank_sum_exact(nx, X, ny, Y)
+                                      : or_rank_sum(nx, X, ny, Y);
             free(X); free(Y);
         }
         /* C9 — best and second base: rank by q_sum (unique bases) or, with no unique base, by

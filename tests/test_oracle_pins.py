@@ -235,6 +235,43 @@ def test_rank_sum_special_cases():
     assert abs(oracle.rank_sum(X, Y) - math.erfc(abs(z) / math.sqrt(2))) < 1e-15
 
 
+# R20: exact small-sample rank-sum
+def test_rank_sum_exact_matches_scipy_exact():
+    from scipy.stats import mannwhitneyu
+    rng = np.random.default_rng(5)
+    for _ in range(60):
+        n1, n2 = int(rng.integers(1, 33)), int(rng.integers(1, 33))
+        v = rng.permutation(np.arange(2, 2 + n1 + n2 + int(rng.integers(0, 20))))  # no ties
+        X, Y = v[:n1], v[n1:n1 + n2]
+        want = mannwhitneyu(X, Y, alternative="two-sided", method="exact").pvalue
+        assert abs(oracle.rank_sum_exact(X, Y) - want) <= 1e-12 * want + 1e-300
+
+
+def test_rank_sum_exact_closed_forms_and_fallbacks():
+    # n1 = 1: U is uniform on 0..n2, so P(U <= u) = (u+1)/(n2+1)
+    for n2 in (1, 5, 32):
+        for rank in range(1, n2 + 2):                       # rank of the single X among N
+            Y = [q for q in range(10, 10 + n2 + 1) if q != 9 + rank]
+            u = rank - 1
+            want = min(1.0, 2 * min(u + 1, n2 + 1 - u) / (n2 + 1))
+            assert abs(oracle.rank_sum_exact([9 + rank], Y) - want) < 1e-15
+    # complete separation of n1 = n2 = 10: one of C(20,10) rank sets at each extreme
+    assert abs(oracle.rank_sum_exact(range(10, 20), range(30, 40)) - 2 / math.comb(20, 10)) < 1e-20
+    # brute force over all n1-subsets for small N
+    import itertools
+    X, Y = [3, 17, 8, 25], [11, 2, 30, 14, 6]
+    ranks = {q: r + 1 for r, q in enumerate(sorted(X + Y))}
+    W = sum(ranks[q] for q in X)
+    sums = [sum(c) for c in itertools.combinations(range(1, 10), 4)]
+    le, ge = sum(s <= W for s in sums), sum(s >= W for s in sums)
+    assert abs(oracle.rank_sum_exact(X, Y) - min(1, 2 * min(le, ge) / len(sums))) < 1e-15
+    # ties or a group above 32 -> the normal approximation of R8; empty group -> 0
+    assert oracle.rank_sum_exact([30, 31, 32], [30, 33]) == oracle.rank_sum([30, 31, 32], [30, 33])
+    big = list(range(2, 35))
+    assert oracle.rank_sum_exact(big, [40]) == oracle.rank_sum(big, [40])
+    assert oracle.rank_sum_exact([], [30]) == 0.0
+
+
 # ---------------------------------------------------------------- C0 / C1: counting
 def test_site_counters_match_bruteforce_recount():
     w = synth.generate("C1")
