@@ -48,6 +48,14 @@ typedef int32_t gsnp_status;
 #define GSNP_MONOPLOID 0x4u   /* heterozygous genotypes get prior 0 at every site (known rows too) */
 #define GSNP_TITV 0x8u        /* novel priors weighted for transition:transversion 2:1: the
                                  transition allele of ref (A<->G, C<->T) x2, transversions x1/2 */
+/* Exact small-sample rank-sum (reading R20, SURVEY §8(f) NEXT #4 "exact small-N rank-sum table";
+ * the paper never names the test).  With GSNP_RANK_SUM also set: when both
+ * allele groups hold <= GSNP_RANK_EXACT_MAX unique reads and the pooled qualities have no ties,
+ * rank_p is the exact two-sided p-value min(1, 2 min(P(U <= u), P(U >= u))) of the Mann-Whitney
+ * U = W - n1(n1+1)/2 under H0 (all C(n1+n2, n1) rank sets equally likely), read from a table the
+ * library builds at gsnp_create; otherwise the normal approximation of R8 stays. */
+#define GSNP_RANK_EXACT 0x10u
+#define GSNP_RANK_EXACT_MAX 32
 
 /* stages reported by gsnp_stage_times */
 #define GSNP_STAGE_VALIDATE 0     /* k_validate_reads */

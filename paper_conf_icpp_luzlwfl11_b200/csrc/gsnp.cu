@@ -74,6 +74,7 @@ struct gsnp_ctx {
     int adjP = 1, adjG = 1;
     DevBuf<uint8_t> adj;
     DevBuf<double> LP;
+    DevBuf<double> rank_cdf;       // R20 exact rank-sum table (GSNP_RANK_EXACT only)
     std::vector<uint64_t> h_counts;
     std::vector<double> h_p;   // [64][256][4][4]
     double* h_T = nullptr;     // [64][L][4][10], pinned host copy of the score table
@@ -200,6 +201,32 @@ int adjust_expr(double lpd, double lgd, int q, int pcr, int g) {
     double e = lq + (double)(pcr - 1) * lpd + (double)g * lgd;
     int qa = (int)(pow(10.0, e) + 0.5);
     return qa < 1 ? 1 : qa;
+}
+
+// R20 table F[(m*33+n)*1025 + u] = P(U <= u) of the Mann-Whitney U for sample sizes m, n <= 32
+// under H0.  Frequencies by the recursion on the largest pooled observation:
+// c(m,n,u) = c(m-1,n,u-n) + c(m,n-1,u), c(0,n,u) = c(m,0,u) = [u == 0]; doubles are exact up to
+// 2^53 and relative 1e-16 beyond (C(64,32) ~ 1.8e18).
+void build_rank_cdf(std::vector<double>& F) {
+    const int M = GSNP_RANK_EXACT_MAX, S = (M + 1) * (M + 1) * 1025;
+    std::vector<double> c(S, 0.0);
+    auto at = [&](int m, int n) { return c.data() + (size_t)(m * 33 + n) * 1025; };
+    for (int m = 0; m <= M; ++m)
+        for (int n = 0; n <= M; ++n) {
+            double* cm = at(m, n);
+            if (m == 0 || n == 0) { cm[0] = 1.0; continue; }
+            const double *a = at(m - 1, n), *b = at(m, n - 1);
+            for (int u = 0; u <= m * n; ++u) cm[u] = (u >= n ? a[u - n] : 0.0) + b[u];
+        }
+    F.assign(S, 1.0);
+    for (int m = 0; m <= M; ++m)
+        for (int n = 0; n <= M; ++n) {
+            const double* cm = at(m, n);
+            double tot = 0.0, run = 0.0;
+            for (int u = 0; u <= m * n; ++u) tot += cm[u];
+            double* f = F.data() + (size_t)(m * 33 + n) * 1025;
+            for (int u = 0; u <= m * n; ++u) { run += cm[u]; f[u] = run / tot; }
+        }
 }
 
 // Build adj[64][P][G].  The expression is non-increasing in pcr and g (coefficients <= 1), so
@@ -406,6 +433,7 @@ gsnp_status prep_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t 
     A.n_known = ctx->n_known;
     A.LP = ctx->LP.p;
     A.T = ctx->T.p;
+    A.rank_cdf = (ctx->prm.flags & GSNP_RANK_EXACT) ? ctx->rank_cdf.p : nullptr;
     A.adj = ctx->adj.p;
     A.adjP = ctx->adjP;
     A.adjG = ctx->adjG;
@@ -796,6 +824,12 @@ gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
     CKC(cudaMemcpy(ctx->LP.p, LP, sizeof LP, cudaMemcpyHostToDevice));
     CKC(ctx->adj.ensure(ctx->h_adj.size()));
     CKC(cudaMemcpy(ctx->adj.p, ctx->h_adj.data(), ctx->h_adj.size(), cudaMemcpyHostToDevice));
+    if (params->flags & GSNP_RANK_EXACT) {
+        std::vector<double> F;
+        build_rank_cdf(F);
+        CKC(ctx->rank_cdf.ensure(F.size()));
+        CKC(cudaMemcpy(ctx->rank_cdf.p, F.data(), F.size() * 8, cudaMemcpyHostToDevice));
+    }
     CKC(ctx->d_err.ensure(1));
 #undef CKC
     *out = ctx;
@@ -1240,7 +1274,7 @@ void gsnp_destroy(gsnp_ctx* ctx) {
     if (!ctx) return;
     cudaSetDevice(ctx->prm.device);
     ctx->ref.release(); ctx->known_pos.release(); ctx->known_lp.release();
-    ctx->adj.release(); ctx->LP.release(); ctx->T.release(); ctx->d_err.release();
+    ctx->adj.release(); ctx->LP.release(); ctx->rank_cdf.release(); ctx->T.release(); ctx->d_err.release();
     ctx->d_counts.release(); ctx->tile_ra.release(); ctx->tile_rb.release(); ctx->rec.release();
     ctx->big.release(); ctx->big_n.release(); ctx->wlist.release();
     ctx->dense_occ.release(); ctx->dense_cnt.release();

@@ -48,6 +48,7 @@ struct CallArgs {
     uint64_t n_known;
     const double* LP;                 // [5][10] log10 novel priors per reference code (R6)
     const double* T;                  // [64][L][4][TROW] score table (Alg. 3), rows padded
+    const double* rank_cdf;           // R20: [(n1*33+n2)*1025 + u] = P(U <= u); null if unused
     const uint8_t* adj;               // [64][adjP][adjG] adjust table (R3)
     int adjP, adjG;
     int L, q_max;
@@ -686,7 +687,13 @@ __device__ __noinline__ void site_record(const CallArgs& A, uint64_t site, int r
             double n1d = (double)n1, n2d = (double)n2, Nd = (double)(n1 + n2);
             double mu = n1d * (Nd + 1.0) / 2.0;
             double var = n1d * n2d / 12.0 * ((Nd + 1.0) - tie / (Nd * (Nd - 1.0)));
-            if (!(var > 0.0)) rank_p = 1.0;
+            if (A.rank_cdf && tie == 0.0 && n1 <= GSNP_RANK_EXACT_MAX &&
+                n2 <= GSNP_RANK_EXACT_MAX) {
+                // R20 exact: U = W - n1(n1+1)/2 is an integer when nothing ties
+                const int u = (int)llrint(wsum - n1d * (n1d + 1.0) / 2.0);
+                const double* F = A.rank_cdf + (size_t)(n1 * 33 + n2) * 1025;
+                rank_p = fmin(1.0, 2.0 * fmin(F[u], F[(int)(n1 * n2) - u]));
+            } else if (!(var > 0.0)) rank_p = 1.0;
             else {
                 double z = (wsum - mu) / sqrt(var);
                 rank_p = erfc(fabs(z) / sqrt(2.0));

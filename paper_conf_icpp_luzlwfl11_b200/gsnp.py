@@ -18,6 +18,7 @@ GSNP_RANK_SUM = 0x1
 GSNP_TIMING = 0x2
 GSNP_MONOPLOID = 0x4
 GSNP_TITV = 0x8
+GSNP_RANK_EXACT = 0x10      # R20 exact small-sample rank-sum (include/gsnp.h)
 STAGES = ("validate", "calib_count", "tile_ranges", "call_tile", "finalize", "big_sites",
           "compress", "warp_sites", "dense_count", "dense_lik", "dense_recycle", "parse")
 STATUS = {0: "GSNP_OK", -1: "GSNP_E_INVAL", -2: "GSNP_E_RANGE", -3: "GSNP_E_UNSORTED",

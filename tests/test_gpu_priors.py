@@ -68,3 +68,22 @@ def test_priors_from_freq_library_equals_oracle_and_calls():
         ctx.calibrate(w)
         rec_g = ctx.call(w, 0, 6_000)
     compare(w, rec_g, rec_o, dbg["L10"])
+
+
+@pytest.mark.parametrize("depth", [6.0, 12.0])
+def test_rank_exact_parity(depth):
+    """R20: exact small-sample rank-sum table in every call path vs the
+    oracle's subset-count definition; het-rich input so the exact branch decides many sites."""
+    w = synth.generate("C1", n_sites=8_000, depth=depth, seed=47, het_rate=0.05)
+    P = oracle.Params(rank_exact=True)
+    p = oracle.p_matrix(P, oracle.calib_counts(P, w))
+    rec_o, dbg = oracle.call_window(P, w, p, 0, 8_000, debug=True)
+    rec_n = oracle.call_window(oracle.Params(), w, p, 0, 8_000)
+    assert (rec_o["rank_p"] != rec_n["rank_p"]).sum() >= 20       # the exact branch is exercised
+    with gsnp.Context.from_workload(w, flags=gsnp.GSNP_RANK_SUM | gsnp.GSNP_RANK_EXACT) as ctx:
+        ctx.calibrate(w)
+        rec_g = ctx.call(w, 0, 8_000)
+        dg = ctx.debug_window(w, 0, 8_000)
+        rec_d = ctx.call_dense(w, 0, 8_000, chunk_sites=2048)
+    assert rec_g.tobytes() == dg["records"].tobytes() == rec_d.tobytes()
+    compare(w, rec_g, rec_o, dbg["L10"])
