@@ -87,3 +87,16 @@ def test_rank_exact_parity(depth):
         rec_d = ctx.call_dense(w, 0, 8_000, chunk_sites=2048)
     assert rec_g.tobytes() == dg["records"].tobytes() == rec_d.tobytes()
     compare(w, rec_g, rec_o, dbg["L10"])
+
+
+def test_rank_exact_needs_rank_sum():
+    """R20 refines R8's p-value only: GSNP_RANK_EXACT without GSNP_RANK_SUM applies no test."""
+    w = synth.generate("C1", n_sites=4_000, depth=6.0, seed=48, het_rate=0.05)
+    P = oracle.Params(rank_sum=False, rank_exact=True)
+    p = oracle.p_matrix(P, oracle.calib_counts(P, w))
+    rec_o, dbg = oracle.call_window(P, w, p, 0, 4_000, debug=True)
+    with gsnp.Context.from_workload(w, flags=gsnp.GSNP_RANK_EXACT) as ctx:
+        ctx.calibrate(w)
+        rec_g = ctx.call(w, 0, 4_000)
+    assert np.all(rec_g["rank_p"] == 1.0)
+    compare(w, rec_g, rec_o, dbg["L10"])
