@@ -561,9 +561,20 @@ gsnp_status count_impl(gsnp_ctx* ctx, const gsnp_reads* reads) {
         A.tma_ok = ((reinterpret_cast<uintptr_t>(d.bases) | reinterpret_cast<uintptr_t>(d.quals)) & 15) == 0;
         // shared memory: u32 diagonal histogram [q][t][cycle] + two stages of (bases, quals,
         // reference window).  Cycles beyond Lh (only for long reads at high q_max) use global REDs.
-        const size_t budget = 200 * 1024;
+        // budget: the opt-in maximum per CTA less the kernel's static shared memory (larger
+        // batches amortise the per-batch barriers and metadata over more words per thread)
+        static size_t budget = 0;
+        if (!budget) {
+            int optin = 0;
+            cudaFuncAttributes fa{};
+            cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, ctx->prm.device);
+            CK(cudaFuncGetAttributes(&fa, k_calib_count));
+            budget = optin > (int)fa.sharedSizeBytes + 64 * 1024 ? (size_t)optin - fa.sharedSizeBytes - 256
+                                                                 : 200 * 1024;
+            if (const char* e = getenv("GSNP_CAL_BUDGET_KB")) budget = (size_t)atoi(e) * 1024;
+        }
         A.RB = 8 * 1024;                               // reference window per stage
-        A.SB = 24 * 1024;                              // bases (and quals) per stage
+        A.SB = 32 * 1024;                              // bases (and quals) per stage
         const size_t per_cyc = (size_t)(A.q_max + 1) * 4 * 4;
         A.Lh = std::min<int>(A.L, (int)((budget - 2 * (2 * 4096 + A.RB) - 16) / per_cyc) & ~3);
         const size_t hist = align16(per_cyc * ((A.Lh + 3) / 4 * 4));
