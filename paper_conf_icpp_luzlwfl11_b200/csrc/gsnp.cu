@@ -115,6 +115,10 @@ struct gsnp_ctx {
     // delay the read
     uint64_t* mbox = nullptr;
     uint64_t launches = 0;
+    // per-device facts, read at gsnp_create on prm.device (a process may hold contexts on
+    // several devices)
+    int num_sms = 148;
+    size_t cal_budget = 0;            // k_calib_count shared-memory budget (0 = not yet sized)
     // per-stage timing (GSNP_TIMING)
     struct Pending { int stage; cudaEvent_t a, b; };
     std::vector<cudaEvent_t> ev_pool;
@@ -404,8 +408,6 @@ gsnp_status launch_validate(gsnp_ctx* ctx, const DevReads& d) {
     return GSNP_OK;
 }
 
-int g_num_sms = 0;
-
 // a3: per-32-site-group read ranges of [w0, w1) (k_tile_ranges) and the kernels' arguments
 gsnp_status prep_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w1,
                         gsnp_record* d_out, CallArgs& A) {
@@ -486,7 +488,7 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
     const bool dbg = A.count_only || A.dbg_off || A.dbg_counters || A.dbg_L10 || A.dbg_post10;
     if (deep) {
         ctx->begin();
-        CK(gsnp_deep::launch_call_tile_deep(&A, sizeof A, dbg, g_num_sms, adj_bytes, adj_smem,
+        CK(gsnp_deep::launch_call_tile_deep(&A, sizeof A, dbg, ctx->num_sms, adj_bytes, adj_smem,
                                             ctx->wlist.p, ctx->big_n.p + 2, ctx->big_n.p + 1, s));
         ctx->end(GSNP_STAGE_CALL);
         ctx->launches++;
@@ -495,7 +497,7 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
         CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         int per_sm = 0;
         CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NT, smem));
-        const uint64_t want = (uint64_t)g_num_sms * std::max(per_sm, 1);
+        const uint64_t want = (uint64_t)ctx->num_sms * std::max(per_sm, 1);
         const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, n_tiles));
         ctx->begin();
         kern<<<grid, NT, smem, s>>>(A, ctx->wlist.p, ctx->big_n.p + 2, ctx->big_n.p + 1, adj_smem);
@@ -511,7 +513,7 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
         int wper = 0;
         CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&wper, wk, NT, wsm));
         ctx->begin();
-        wk<<<(unsigned)(g_num_sms * std::max(wper, 1)), NT, wsm, s>>>(A, ctx->wlist.p, ctx->big_n.p + 2,
+        wk<<<(unsigned)(ctx->num_sms * std::max(wper, 1)), NT, wsm, s>>>(A, ctx->wlist.p, ctx->big_n.p + 2,
                                                                        ctx->big.p, ctx->big_n.p, big_cap);
         ctx->end(GSNP_STAGE_WARP);
         ctx->launches++;
@@ -521,7 +523,7 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
         const size_t bsm = 4 * (size_t)cap + (size_t)8 * A.L;
         CK(cudaFuncSetAttribute(k_big_sites, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bsm));
         ctx->begin();
-        k_big_sites<<<(unsigned)g_num_sms, NT, bsm, s>>>(A, ctx->big.p, ctx->big_n.p, cap);
+        k_big_sites<<<(unsigned)ctx->num_sms, NT, bsm, s>>>(A, ctx->big.p, ctx->big_n.p, cap);
         ctx->end(GSNP_STAGE_BIG);
         ctx->launches++;
         CK(cudaGetLastError());
@@ -563,7 +565,7 @@ gsnp_status count_impl(gsnp_ctx* ctx, const gsnp_reads* reads) {
         // reference window).  Cycles beyond Lh (only for long reads at high q_max) use global REDs.
         // budget: the opt-in maximum per CTA less the kernel's static shared memory (larger
         // batches amortise the per-batch barriers and metadata over more words per thread)
-        static size_t budget = 0;
+        size_t& budget = ctx->cal_budget;
         if (!budget) {
             int optin = 0;
             cudaFuncAttributes fa{};
@@ -581,7 +583,7 @@ gsnp_status count_impl(gsnp_ctx* ctx, const gsnp_reads* reads) {
         while (A.SB > 4096 && hist + 2 * (2 * (size_t)A.SB + A.RB) + 16 > budget) A.SB -= 4096;
         A.CB = std::max(1, std::min<int>(CAL_MAXB, (int)(A.SB - 32) / A.L));
         const size_t smem = hist + 2 * (2 * (size_t)A.SB + A.RB) + 16;
-        unsigned grid = (unsigned)std::min<uint64_t>((uint64_t)g_num_sms, (d.n + A.CB - 1) / A.CB);
+        unsigned grid = (unsigned)std::min<uint64_t>((uint64_t)ctx->num_sms, (d.n + A.CB - 1) / A.CB);
         grid = std::max(grid, 1u);
         CK(cudaFuncSetAttribute(k_calib_count, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         ctx->begin();
@@ -681,7 +683,7 @@ gsnp_status compress_impl(gsnp_ctx* ctx, const gsnp_record* d_rec, uint64_t n, u
     CK(cudaFuncSetAttribute(k_cz_sections<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_size));
     CK(cudaFuncSetAttribute(k_cz_sections<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_write));
     ctx->begin();
-    const unsigned g0 = (unsigned)std::min<uint64_t>((n + 255) / 256, (uint64_t)g_num_sms * 8);
+    const unsigned g0 = (unsigned)std::min<uint64_t>((n + 255) / 256, (uint64_t)ctx->num_sms * 8);
     k_cz_columns<<<g0, 256, 0, s>>>(d_rec, n, A.col);
     k_cz_sections<false><<<(unsigned)(nblk * NSEC), gsnp_cz::NT, sm_size, s>>>(A);
     k_cz_scan<<<1, 1024, 0, s>>>(ctx->cz_meta.p, nblk * NSEC, ctx->cz_off.p);
@@ -772,9 +774,10 @@ gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
     ctx->stream = (cudaStream_t)params->stream;
     auto bail = [&](gsnp_status s) { gsnp_destroy(ctx); return s; };
     if (cudaSetDevice(params->device) != cudaSuccess) { cudaGetLastError(); return bail(GSNP_E_CUDA); }
-    if (!g_num_sms) {
-        cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, params->device);
-        if (g_num_sms <= 0) g_num_sms = 148;
+    {
+        int sms = 0;
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, params->device);
+        ctx->num_sms = sms > 0 ? sms : 148;
     }
     ctx->n_sites = ref->n_sites;
     ctx->origin = ref->origin;
@@ -965,13 +968,13 @@ gsnp_status gsnp_call_dense(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0,
         CK(cudaMemsetAsync(D.cnt, 0, n * 5 * 4, s));
         if (d.n) {
             ctx->begin();
-            k_dense_count<<<(unsigned)(g_num_sms * 8), DENSE_NT, 0, s>>>(D);
+            k_dense_count<<<(unsigned)(ctx->num_sms * 8), DENSE_NT, 0, s>>>(D);
             ctx->end(GSNP_STAGE_DENSE_COUNT);
             ctx->launches++;
             CK(cudaGetLastError());
         }
         ctx->begin();
-        k_dense_sites<<<(unsigned)std::min<uint64_t>((n + 7) / 8, (uint64_t)g_num_sms * 8), DENSE_NT, 0, s>>>(D);
+        k_dense_sites<<<(unsigned)std::min<uint64_t>((n + 7) / 8, (uint64_t)ctx->num_sms * 8), DENSE_NT, 0, s>>>(D);
         ctx->end(GSNP_STAGE_DENSE_LIK);
         ctx->launches++;
         CK(cudaGetLastError());
@@ -1060,7 +1063,7 @@ gsnp_status gsnp_parse_soap(gsnp_ctx* ctx, const char* text, uint64_t n_bytes, c
         CK(ctx->p_part.ensure(2 * (n_sel_tiles + 1)));
         P.meta = ctx->p_meta.p; P.pos = ctx->p_pos.p; P.ridx = ctx->p_ridx.p; P.boff = ctx->p_boff.p;
         const unsigned wgrid = (unsigned)std::min<uint64_t>((n_lines + PGROUPS - 1) / PGROUPS,
-                                                            (uint64_t)g_num_sms * 8);
+                                                            (uint64_t)ctx->num_sms * 8);
         uint64_t* part_n = ctx->p_part.p;
         uint64_t* part_b = ctx->p_part.p + n_sel_tiles + 1;
         ctx->begin();
@@ -1112,7 +1115,7 @@ gsnp_status gsnp_parse_soap(gsnp_ctx* ctx, const char* text, uint64_t n_bytes, c
         const uint64_t* part_b = ctx->p_part.p + n_sel_tiles + 1;
         ctx->begin();
         k_sel_apply<<<(unsigned)n_sel_tiles, PNT, 0, s>>>(P, part_n, part_b);
-        k_parse_emit<<<(unsigned)std::min<uint64_t>((n_lines + PGROUPS - 1) / PGROUPS, (uint64_t)g_num_sms * 8), PNT, 0, s>>>(
+        k_parse_emit<<<(unsigned)std::min<uint64_t>((n_lines + PGROUPS - 1) / PGROUPS, (uint64_t)ctx->num_sms * 8), PNT, 0, s>>>(
             P, tot[0], tot[1]);
         ctx->end(GSNP_STAGE_PARSE);
         ctx->launches += 2;

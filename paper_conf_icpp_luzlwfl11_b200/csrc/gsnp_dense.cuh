@@ -36,6 +36,7 @@ struct DenseArgs {
 // counting: every base of every read that can touch [c0, c1)
 __global__ void __launch_bounds__(DENSE_NT) k_dense_count(const __grid_constant__ DenseArgs D) {
     const CallArgs& A = D.A;
+    if (reads_invalid(A.err)) return;
     const uint64_t ga = (D.c0 - A.w0) / 32, gb = (D.c1 - 1 - A.w0) / 32;
     const uint64_t ra = A.tile_ra[ga], rb = A.tile_rb[gb];
     const int lane = threadIdx.x & 31;

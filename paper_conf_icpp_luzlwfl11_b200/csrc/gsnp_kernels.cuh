@@ -25,7 +25,16 @@ constexpr int NW = NT / 32;           // warps per CTA
 constexpr uint32_t FULL = 0xFFFFFFFFu;
 constexpr uint32_t KEY_INF = 0xFFFFFFFFu;
 
-enum : int { ERR_RANGE = 1, ERR_UNSORTED = 2, ERR_DEEP = 4, ERR_QUAL = 8 };
+enum : int { ERR_RANGE = 1, ERR_UNSORTED = 2, ERR_DEEP = 4, ERR_QUAL = 8, ERR_VALID = 64 };
+
+// k_validate_reads sets ERR_VALID (with the specific bits) when the read arrays break the ABI
+// contract (unsorted positions, offsets, lengths or positions out of range).  Every kernel that
+// dereferences pos/off/len runs after it on the same stream and returns at once when the flag is
+// up, so out-of-contract input yields a status, never an out-of-bounds access.  Only the
+// validator writes this bit, so every thread of a launch reads the same value.
+__device__ __forceinline__ bool reads_invalid(const int* err) {
+    return (*reinterpret_cast<const volatile int*>(err) & ERR_VALID) != 0;
+}
 
 struct DevReads {
     const uint64_t* pos;
@@ -98,7 +107,7 @@ __global__ void k_validate_reads(DevReads R, uint64_t origin, uint64_t n_sites, 
     if (p < origin || p + l > origin + n_sites) e |= ERR_RANGE;
     if (R.off[r] < R.off0 || R.off[r] + l > R.off[r + 1]) e |= ERR_RANGE;
     if (r > 0 && R.pos[r - 1] > p) e |= ERR_UNSORTED;
-    if (e) atomicOr(err, e);
+    if (e) atomicOr(err, e | ERR_VALID);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -228,6 +237,7 @@ __global__ void __launch_bounds__(CAL_NT, 1) k_calib_count(const __grid_constant
     // or ~0 for a read that is not counted
     __shared__ uint32_t m_flat[2][CAL_MAXB];
     __shared__ uint32_t m_fl[2][3];                   // uniform flag, reads in batch, length Lb
+    if (reads_invalid(A.err)) return;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int L = A.L, Lh = A.Lh;
     const uint32_t qmax = (uint32_t)A.q_max;
@@ -306,7 +316,9 @@ __global__ void __launch_bounds__(CAL_NT, 1) k_calib_count(const __grid_constant
         const uint64_t r0 = m.p0 >= A.origin ? ((m.p0 - A.origin) & ~15ull) : 0;   // = st_rs
         if (m.in)
             m_flat[sidx][tid] = keep ? (uint32_t)(m.p - A.origin - r0) | m.st << 31 : 0xFFFFFFFFu;
-        const bool uni = !m.in || (m.l == m.l0 && m.o - m.ob0 == (uint64_t)tid * m.l0);
+        // (flat mode needs Lb >= 2: its read index is a multiply-high by ceil(2^32 / Lb), which
+        // wraps to 0 at Lb == 1 — batches of 1-bp reads take the staged path)
+        const bool uni = m.l0 >= 2 && (!m.in || (m.l == m.l0 && m.o - m.ob0 == (uint64_t)tid * m.l0));
         const int all_uni = __syncthreads_and(uni);
         if (tid == 0) { m_fl[sidx][0] = all_uni; m_fl[sidx][1] = m.nall; m_fl[sidx][2] = m.l0; }
     };
@@ -1477,6 +1489,7 @@ struct BigSite {
 template <bool DBG, int CC>
 __global__ void __launch_bounds__(NT, GSNP_CALL_MINB)
 k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist_n, uint32_t* work, uint32_t adj_smem) {
+    if (reads_invalid(A.err)) return;
     extern __shared__ __align__(16) unsigned char smem[];
     TileSmem sm;
     const size_t adj_bytes = adj_smem ? (size_t)64 * A.adjP * A.adjG : 0;
@@ -1658,6 +1671,7 @@ template <int CC>
 __global__ void __launch_bounds__(NT) k_warp_sites(const __grid_constant__ CallArgs A, const uint32_t* wlist,
                                                    const uint32_t* wlist_n, BigSite* big,
                                                    uint32_t* big_n, uint32_t big_cap) {
+    if (reads_invalid(A.err)) return;
     extern __shared__ __align__(16) unsigned char smem[];
     TileSmem sm;
     call_smem_bytes(A.L, 0, CC, &sm, smem);
@@ -1709,6 +1723,7 @@ __global__ void __launch_bounds__(NT) k_warp_sites(const __grid_constant__ CallA
 // keys gathered into a shared buffer of `cap` keys (GSNP_E_CAPACITY beyond it).
 __global__ void __launch_bounds__(NT) k_big_sites(const __grid_constant__ CallArgs A, const BigSite* big,
                                                   const uint32_t* big_n, uint32_t cap) {
+    if (reads_invalid(A.err)) return;
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ double red[NW * 18];
     __shared__ uint32_t cnt;
