@@ -215,13 +215,17 @@ def rank_sum_exact(X, Y) -> float:
     return lib().or_rank_sum_exact(len(X), _p(X), len(Y), _p(Y))
 
 
-def call_window(P: Params, w: dict, p: np.ndarray, w0: int, w1: int, debug: bool = False):
+def call_window(P: Params, w: dict, p: np.ndarray, w0: int, w1: int, debug: bool = False,
+                want=("off", "keys", "counters", "L10", "post10"), out=None):
     """C0-C9 over sites [w0, w1).  Returns records (RECORD_DTYPE) and, with debug=True, a dict
-    with off (u32[S+1]), keys (sorted, CSR), counters (u32[S,15]), L10, post10 (f64[S,10])."""
+    with off (u32[S+1]), keys (sorted, CSR), counters (u32[S,15]), L10, post10 (f64[S,10]) —
+    only the parts named in `want`.  `out` may supply the destination arrays (dict with "rec" and
+    any of the debug names), e.g. views of shared memory."""
     c = P.c()
     r, keep = _reads(w)
     S = w1 - w0
-    rec = np.zeros(S, RECORD_DTYPE)
+    out = out or {}
+    rec = out["rec"] if "rec" in out else np.zeros(S, RECORD_DTYPE)
     ref = np.ascontiguousarray(w["ref"], np.uint8)
     kp = np.ascontiguousarray(w["known_pos"], np.uint64)
     kpr = np.ascontiguousarray(w["known_prior10"], np.float64)
@@ -229,17 +233,21 @@ def call_window(P: Params, w: dict, p: np.ndarray, w0: int, w1: int, debug: bool
     dbg = None
     if debug:
         nb = int(w["off"][-1]) if len(w["off"]) else 0
-        dbg = dict(off=np.zeros(S + 1, np.uint32), keys=np.zeros(max(nb, 1), np.uint32),
-                   counters=np.zeros((S, 15), np.uint32), L10=np.zeros((S, 10)),
-                   post10=np.zeros((S, 10)))
-    g = (lambda k: _p(dbg[k]) if dbg else None)
+        make = dict(off=lambda: np.zeros(S + 1, np.uint32), keys=lambda: np.zeros(max(nb, 1), np.uint32),
+                    counters=lambda: np.zeros((S, 15), np.uint32), L10=lambda: np.zeros((S, 10)),
+                    post10=lambda: np.zeros((S, 10)))
+        dbg = {k: (out[k] if k in out else make[k]()) for k in want}
+        if "keys" in dbg and "off" not in dbg:
+            dbg["off"] = make["off"]()
+    g = (lambda k: _p(dbg[k]) if dbg and k in dbg else None)
     rc = lib().or_call_window(ctypes.byref(c), _p(ref), len(ref), int(w["origin"]), len(kp),
                               _p(kp), _p(kpr), _p(pp), ctypes.byref(r), w0, w1, _p(rec),
                               g("off"), g("keys"), g("counters"), g("L10"), g("post10"))
     if rc != 0:
         raise ValueError(f"or_call_window: {rc}")
     if dbg:
-        dbg["keys"] = dbg["keys"][: dbg["off"][-1]]
+        if "keys" in dbg:
+            dbg["keys"] = dbg["keys"][: dbg["off"][-1]]
         return rec, dbg
     return rec
 

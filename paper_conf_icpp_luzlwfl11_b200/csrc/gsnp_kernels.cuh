@@ -1070,10 +1070,11 @@ __device__ __forceinline__ void group_epilogue(const CallArgs& A, uint64_t site,
     }
 }
 
-// Warp gather of one site's unique non-N keys from the reads [ra, rb) into the warp slice;
-// returns the count.
+// Warp gather of one site's unique non-N keys from the reads [ra, rb) into the warp slice (at
+// most cap keys are stored: a deeper site goes to k_big_sites, which gathers again); returns the
+// count.
 __device__ __forceinline__ uint32_t warp_gather(const CallArgs& A, uint32_t* col, int warp,
-                                                uint64_t s, uint64_t ra, uint64_t rb) {
+                                                uint64_t s, uint64_t ra, uint64_t rb, uint32_t cap) {
     const int lane = threadIdx.x & 31;
     uint32_t m = 0;
     for (uint64_t r0 = ra; r0 < rb; r0 += 32) {
@@ -1093,7 +1094,8 @@ __device__ __forceinline__ uint32_t warp_gather(const CallArgs& A, uint32_t* col
             }
         }
         const uint32_t v = __ballot_sync(FULL, key != KEY_INF);
-        if (key != KEY_INF) col[wslot(warp, m + __popc(v & lanemask_lt()))] = key;
+        const uint32_t e = m + __popc(v & lanemask_lt());
+        if (key != KEY_INF && e < cap) col[wslot(warp, e)] = key;
         m += __popc(v);
     }
     __syncwarp();
@@ -1702,7 +1704,7 @@ __global__ void __launch_bounds__(NT) k_warp_sites(const __grid_constant__ CallA
             for (int x = 0; x < 4; ++x) c[x] += __shfl_xor_sync(FULL, c[x], d);
             rp += __shfl_xor_sync(FULL, rp, d);
         }
-        const uint32_t m = warp_gather(A, sm.col, warp, s, ra, rb);
+        const uint32_t m = warp_gather(A, sm.col, warp, s, ra, rb, 32u * CC);
         if (m > 32u * CC) {
             if (lane == 0) {
                 const uint32_t k = atomicAdd(big_n, 1u);

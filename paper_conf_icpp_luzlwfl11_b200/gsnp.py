@@ -330,22 +330,30 @@ class Context:
                                           cap, ctypes.byref(nw)), self.h)
         return int(nw.value)
 
-    def debug_window(self, reads: dict, w0: int, w1: int):
+    def debug_window(self, reads: dict, w0: int, w1: int,
+                     want=("off", "keys_built", "keys_sorted", "counters", "L10", "post10",
+                           "records")):
+        """gsnp_debug_window into host arrays; only the parts named in `want` are returned."""
         S = w1 - w0
-        nb = int(np.asarray(reads["off"][-1]) - np.asarray(reads["off"][0])) \
-            if len(reads["off"]) else 0
-        out = dict(off=np.zeros(S + 1, np.uint32), keys_built=np.zeros(max(nb, 1), np.uint32),
-                   keys_sorted=np.zeros(max(nb, 1), np.uint32),
-                   counters=np.zeros((S, 15), np.uint32), L10=np.zeros((S, 10)),
-                   post10=np.zeros((S, 10)), records=np.zeros(S, RECORD_DTYPE))
+        nb = int(reads["off"][-1]) - int(reads["off"][0]) if len(reads["off"]) else 0
+        make = dict(off=lambda: np.zeros(S + 1, np.uint32),
+                    keys_built=lambda: np.zeros(max(nb, 1), np.uint32),
+                    keys_sorted=lambda: np.zeros(max(nb, 1), np.uint32),
+                    counters=lambda: np.zeros((S, 15), np.uint32), L10=lambda: np.zeros((S, 10)),
+                    post10=lambda: np.zeros((S, 10)), records=lambda: np.zeros(S, RECORD_DTYPE))
+        out = {k: make[k]() for k in want}
+        if ("keys_built" in out or "keys_sorted" in out) and "off" not in out:
+            out["off"] = make["off"]()
         r = make_reads(reads)
-        _check(lib().gsnp_debug_window(self.h, ctypes.byref(r), w0, w1, _ptr(out["off"]),
-                                       _ptr(out["keys_built"]), _ptr(out["keys_sorted"]),
-                                       _ptr(out["counters"]), _ptr(out["L10"]),
-                                       _ptr(out["post10"]), _ptr(out["records"])), self.h)
-        K = int(out["off"][-1])
-        out["keys_built"] = out["keys_built"][:K]
-        out["keys_sorted"] = out["keys_sorted"][:K]
+        g = (lambda k: _ptr(out[k]) if k in out else None)
+        _check(lib().gsnp_debug_window(self.h, ctypes.byref(r), w0, w1, g("off"), g("keys_built"),
+                                       g("keys_sorted"), g("counters"), g("L10"), g("post10"),
+                                       g("records")), self.h)
+        if "off" in out:
+            K = int(out["off"][-1])
+            for k in ("keys_built", "keys_sorted"):
+                if k in out:
+                    out[k] = out[k][:K]
         return out
 
     def get_tables(self, calibrated: bool = True):

@@ -134,3 +134,35 @@ def test_contract_violations_are_statuses_in_calibrate_and_call(device_arrays):
     C = oracle.calib_counts(P, w)
     rec_o, dbg = oracle.call_window(P, w, oracle.p_matrix(P, C), 0, S, debug=True)
     compare(w, rec, rec_o, dbg["L10"])
+
+
+def test_pile_inside_shallow_window():
+    """A 1500-read pile inside a long low-depth window: the window is called by the shallow kernel,
+    whose warp path must hand the >1024-key sites to the CTA path without overrunning its
+    shared-memory key buffer."""
+    w0 = synth.generate("C1", n_sites=60_000, depth=5.0, seed=57)
+    rng = np.random.default_rng(57)
+    ref = w0["ref"]
+    reads = []
+    for k in range(len(w0["pos"])):
+        o = int(w0["off"][k])
+        ln = int(w0["len"][k])
+        reads.append(dict(pos=int(w0["pos"][k]), strand=int(w0["strand"][k]), hits=int(w0["hits"][k]),
+                          bases=w0["bases"][o:o + ln], quals=w0["quals"][o:o + ln]))
+    for k in range(1500):
+        p = 30_000 + int(rng.integers(0, 4))
+        b = ref[p:p + 100].copy()
+        b[b == 4] = 0
+        reads.append(dict(pos=p, strand=int(rng.integers(2)), bases=b, quals=list(rng.integers(2, 41, 100))))
+    w = workload(ref, reads)
+    S = len(ref)
+    P = OP
+    C = oracle.calib_counts(P, w)
+    p = oracle.p_matrix(P, C)
+    lo, hi = 29_000, 31_500
+    rec_o, dbg = oracle.call_window(P, w, p, lo, hi, debug=True)
+    with gsnp.Context.from_workload(w) as ctx:
+        ctx.calibrate(w)
+        rec_all = ctx.call(w, 0, S)
+    assert int(rec_all["depth"][30_050]) > 1024
+    compare(w, rec_all[lo:hi], rec_o, dbg["L10"])

@@ -417,3 +417,119 @@ def test_quality_cases_hand_computed():
     rec = oracle.call_window(P1, w, p, 50, 51)
     assert oracle.GENOTYPES[rec["genotype"][0]] == "AG" and rec["known"][0] == 1
     assert rec["quality"][0] == 0 and rec["rank_p"][0] == 0.0
+
+
+# ---------------------------------------------------------------- hand-computed pins (round 2)
+def _theory_p(q, a, o):
+    """Rule 4 of the estimator (R1) — what calibrating on no reads yields: e = min(.75, 10^-q/10)."""
+    e = min(0.75, 10 ** (-q / 10))
+    return 1 - e if a == o else e / 3
+
+
+def _hand_L10(obs):
+    """Alg. 2 per observation, summed in the given order: obs = [(q_adj, base)]."""
+    out = []
+    for n in range(10):
+        a1, a2 = oracle.GA1[n], oracle.GA2[n]
+        s = 0.0
+        for qa, b in obs:
+            s += math.log10(0.5 * _theory_p(qa, a1, b) + 0.5 * _theory_p(qa, a2, b))
+        out.append(s)
+    return np.array(out)
+
+
+def _site_reads(site, specs, L=100):
+    """Reads of length L covering `site`: specs = [(pos, strand, base_at_site, q_at_site)]; every
+    other base matches the all-A reference."""
+    reads = []
+    for pos, st, b, q in specs:
+        bases = ["A"] * L
+        bases[site - pos] = b
+        quals = [30] * L
+        quals[site - pos] = q
+        reads.append(dict(pos=pos, strand=st, bases="".join(bases), quals=quals))
+    return reads
+
+
+def test_dependency_counters_hand_computed_default_coefficients():
+    """pcr and g of Alg. 4 l.8-12 under reading R3 at the default 0.5 / 0.9, written
+    out by hand.  Site 50, reference A.  Six A keys at q30 on '+': reads at 43, 42, 41 give cycles
+    7, 8, 9 (distinct (strand, coord) slots) and three reads at 40 share cycle 10 (PCR duplicates).
+    Canonical order is cycle 7, 8, 9, 10, 10, 10, so (pcr, g) = (1,0) (1,1) (1,2) (1,3) (2,3) (3,3)
+    and q_adj = round(30 * .5^(pcr-1) * .9^g) = 30, 27, 24 (24.3), 22 (21.87), 11 (10.935),
+    5 (5.4675).  Two G keys at q20 on '-' (reads at 45 and 46: cycles 99-5 = 94 and 95) restart the
+    counters for the new base (l.8-11): g = 0, 1 -> 20, 18."""
+    site = 50
+    specs = [(40, 0, "A", 30)] * 3 + [(41, 0, "A", 30), (42, 0, "A", 30), (43, 0, "A", 30),
+                                      (45, 1, "G", 20), (46, 1, "G", 20)]
+    w = workload("A" * 200, _site_reads(site, specs))
+    P = oracle.Params()
+    p = oracle.p_matrix(P, np.zeros((64, 256, 4, 4), np.uint64))
+    rec, dbg = oracle.call_window(P, w, p, site, site + 1, debug=True)
+    q_adj_A = [30, 27, 24, 22, 11, 5]
+    q_adj_G = [20, 18]
+    want = _hand_L10([(q, 0) for q in q_adj_A] + [(q, 3) for q in q_adj_G])
+    assert np.all(np.abs(dbg["L10"][0] - want) <= 1e-12 * np.abs(want))
+    # the pin separates the plausible misreadings: g counted before the increment, g not reset per
+    # base, pcr ignored, and adjust without the 0.5 rounding
+    wrong = {
+        "g_before_increment": [30, 30, 27, 24, 11, 5],
+        "no_pcr": [30, 27, 24, 22, 22, 22],
+        "truncate": [30, 27, 24, 21, 10, 5],
+    }
+    for name, seq in wrong.items():
+        alt = _hand_L10([(q, 0) for q in seq] + [(q, 3) for q in q_adj_G])
+        assert np.max(np.abs(alt - dbg["L10"][0]) / np.abs(want)) > 1e-6, name
+    alt = _hand_L10([(q, 0) for q in q_adj_A] + [(q, 3) for q in (16, 15)])   # g carried over
+    assert np.max(np.abs(alt - dbg["L10"][0]) / np.abs(want)) > 1e-6
+    # the same counters drive the dense Alg. 1 walk (C5)
+    L_dense = oracle.dense_likelihood(P, p, [0] * 6 + [3] * 2, [30] * 6 + [20] * 2,
+                                      [10, 10, 10, 9, 8, 7, 94, 95], [0] * 6 + [1] * 2)
+    assert np.all(np.abs(L_dense - want) <= 1e-12 * np.abs(want))
+
+
+def _hand_quality(obs_raw, ref, rank_sum_p=1.0):
+    """Raw consensus quality (C9 step 2) with identity adjust: int(10 (lp1 - lp2) + 10 log10 p)."""
+    L = _hand_L10(obs_raw)
+    pri = []
+    for n in range(10):
+        a1, a2 = oracle.GA1[n], oracle.GA2[n]
+        v = 1.0 if (a1 == ref and a2 == ref) else 1e-3 if (a1 == ref or a2 == ref) else \
+            5e-4 if a1 == a2 else 5e-7
+        pri.append(math.log10(v))
+    lp = L + np.array(pri)
+    o = np.argsort(-lp, kind="stable")
+    return int(o[0]), int(10 * (lp[o[0]] - lp[o[1]]) + 10 * math.log10(rank_sum_p))
+
+
+def test_quality_caps_bind_below_99():
+    """C9 steps 3-4 where the caps decide the quality (the earlier cases never bind below 99).
+    Identity adjust (coefficients 1, R3) and theoretical p, so each raw quality is a hand sum.
+    Hom: 3 A at q12 + 1 C at q2 on distinct cycles, ref A -> AA, raw 37 > cap
+    q_sum[A] - q_sum[C] = 36 - 2 = 34.  Het (rank-sum off): 8 A at q8 + 3 G at q40, ref A -> AG,
+    raw 68 > cap min(q_sum[A], q_sum[G]) = min(64, 120) = 64."""
+    site = 50
+    P1 = oracle.Params(global_dep=1.0, pcr_dep=1.0)
+    p = oracle.p_matrix(P1, np.zeros((64, 256, 4, 4), np.uint64))
+    specs = [(40 + k, 0, "A", 12) for k in range(3)] + [(44, 0, "C", 2)]
+    w = workload("A" * 200, _site_reads(site, specs))
+    t1, raw = _hand_quality([(12, 0)] * 3 + [(2, 1)], 0)
+    assert (t1, raw) == (0, 37)
+    r = oracle.call_window(P1, w, p, site, site + 1)[0]
+    assert (r["genotype"], r["base1"], r["base2"]) == (0, 0, 1)
+    assert r["quality"] == 34
+    P2 = oracle.Params(global_dep=1.0, pcr_dep=1.0, rank_sum=False)
+    specs = [(30 + k, 0, "A", 8) for k in range(8)] + [(40 + k, 0, "G", 40) for k in range(3)]
+    w = workload("A" * 200, _site_reads(site, specs))
+    t1, raw = _hand_quality([(8, 0)] * 8 + [(40, 3)] * 3, 0)
+    assert (oracle.GENOTYPES[t1], raw) == ("AG", 68)
+    r = oracle.call_window(P2, w, p, site, site + 1)[0]
+    assert oracle.GENOTYPES[r["genotype"]] == "AG" and r["rank_p"] == 1.0
+    assert r["quality"] == 64
+    # with the rank-sum on, the same site pays 10 log10(p) of the disjoint quality groups
+    # (N = 11, W = 36, mu = 48, sigma^2 = 2 (12 - 528/110) = 14.4, z = -12/3.795): raw
+    # int(68.x - 28.05) = 40 < cap
+    r = oracle.call_window(P1, w, p, site, site + 1)[0]
+    pz = math.erfc(12 / math.sqrt(14.4) / math.sqrt(2))
+    assert abs(r["rank_p"] - pz) <= 1e-6 * pz
+    assert r["quality"] == _hand_quality([(8, 0)] * 8 + [(40, 3)] * 3, 0, pz)[1] == 40
