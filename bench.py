@@ -107,18 +107,57 @@ def _dist():
     return ws, rank, local
 
 
-def make_shard(cfg_name: str, rank: int, ws: int):
-    """Weak scaling: rank r holds sites [r*n, (r+1)*n) of one genome of ws*n sites (the config's
-    recipe with its N blocks spread over the genome), generated region by region — the reads
-    covering the shard and the reference under them (shard.py)."""
+STRONG = ("C3", "C4")          # BASELINE configs quoted as one genome sharded over the GPUs
+
+
+def shard_plan(cfg_name: str, ws: int):
+    """Contiguous shards of the config's genome, one per rank.  C3/C4 (strong scaling, BASELINE
+    configs[2..3]): the whole genome split by expected aligned bases — shard.plan_by_bases over a
+    thin sample of read starts drawn with the generator's placement density (no full generation).
+    Other configs (weak scaling): rank r holds a config-sized piece of a ws-times longer genome."""
     import synth
+    from paper_conf_icpp_luzlwfl11_b200 import shard
     base = synth.CONFIGS[cfg_name]
-    if ws == 1:
-        return synth.generate(base)
+    if cfg_name in STRONG:
+        starts = synth.sample_read_starts(base, 2_000_000, seed=base.seed)
+        ln = np.full(len(starts), base.read_len, np.int64)
+        return base, shard.plan_by_bases(starts, ln, base.n_sites, base.origin, ws)
     n = base.n_sites
-    cfg = base.scaled(n_sites=n * ws, n_lead_frac=base.n_lead_frac / ws,
-                      n_blocks=base.n_blocks * ws, region_lo=rank * n, region_hi=(rank + 1) * n)
-    return synth.generate(cfg)
+    if ws == 1:
+        return base, [(base.origin, base.origin + n)]
+    genome = base.scaled(n_sites=n * ws, n_lead_frac=base.n_lead_frac / ws,
+                         n_blocks=base.n_blocks * ws)
+    return genome, [(r * n, (r + 1) * n) for r in range(ws)]
+
+
+def make_shard(cfg_name: str, rank: int, ws: int):
+    """This rank's shard: the reads covering its sites (read-length halo included) and the
+    reference under them, generated region by region (shard.py)."""
+    import synth
+    genome, plan = shard_plan(cfg_name, ws)
+    lo, hi = plan[rank]
+    if lo == genome.origin and hi == genome.origin + genome.n_sites:
+        return synth.generate(genome)
+    return synth.generate(genome.scaled(region_lo=lo - genome.origin, region_hi=hi - genome.origin))
+
+
+def count_keys(w, w0: int, w1: int, chunk: int = 1 << 20) -> int:
+    """Unique non-N aligned bases at sites [w0, w1) (one score-table row each), counted read chunk
+    by read chunk (bounded memory at C3/C4 sizes)."""
+    pos = np.asarray(w["pos"], np.int64)
+    ln = np.asarray(w["len"], np.int64)
+    off = np.asarray(w["off"], np.int64)
+    keys = 0
+    for a in range(0, len(pos), chunk):
+        b = min(len(pos), a + chunk)
+        uni = np.repeat(np.asarray(w["hits"][a:b]) == 1, ln[a:b])
+        ok = uni & (np.asarray(w["bases"][off[a]:off[b]]) < 4)
+        if pos[a] < w0 or pos[b - 1] + ln[a:b].max() > w1:          # reads crossing the edges
+            site = np.repeat(pos[a:b], ln[a:b]) + (np.arange(off[a], off[b]) -
+                                                  np.repeat(off[a:b], ln[a:b]))
+            ok &= (site >= w0) & (site < w1)
+        keys += int(np.count_nonzero(ok))
+    return keys
 
 
 def input_bytes(w) -> int:
@@ -126,60 +165,71 @@ def input_bytes(w) -> int:
                                                       "strand", "hits"))
 
 
-def cpu_oracle_rate(w, budget_s: float = 15.0, max_sites: int | None = None):
-    """Oracle (as it stands) on a bounded sample of the shard: calibration + call over the
-    first S non-trivial sites; returns (sites/s, description)."""
+def _oracle_step(w, lo, hi, procs=None):
+    """One oracle step over sites [lo, hi) of w: calibration counts over the reads that touch the
+    sites, p matrix, and every record — P independent single-threaded oracle processes over
+    windows (SURVEY.md §8(d) timing protocol, tests/_mp.py).  Returns (records, stats)."""
     import oracle
     import synth
+    from tests._mp import calib_parallel, call_parallel
     P = oracle.Params()
-    origin = int(w["origin"])
-    ref = w["ref"]
-    nz = np.nonzero(ref != 4)[0]
-    s0 = origin + int(nz[0]) if len(nz) else origin
-    S = 50_000
-    rate = None
-    desc = ""
-    spent = 0.0
-    while True:
-        s1 = min(s0 + S, origin + len(ref))
-        ra, rb = synth.read_range(w, s0, s1)
-        sub = synth.slice_reads(w, ra, rb)
-        t = time.perf_counter()
-        C = oracle.calib_counts(P, sub)
-        p = oracle.p_matrix(P, C)
-        oracle.call_window(P, sub, p, s0, s1)
-        dt = time.perf_counter() - t
-        spent += dt
-        rate = (s1 - s0) / dt
-        desc = (f"oracle calibrate+call over {s1 - s0} sites [{s0},{s1}) of the shard "
-                f"({rb - ra} reads), single thread, {dt:.2f} s")
-        if spent > budget_s * 0.4 or s1 - s0 >= (max_sites or 1 << 62) or s1 >= origin + len(ref):
-            break
-        S = int(min(max(S * 2, budget_s * 0.6 * rate), 5_000_000))
-    return rate, desc
+    t0 = time.perf_counter()
+    ra, rb = synth.read_range(w, lo, hi)
+    sub = w if (ra == 0 and rb == len(w["pos"])) else synth.slice_reads(w, ra, rb)
+    C, cst = calib_parallel(P, sub, procs)
+    tp = time.perf_counter()
+    p = oracle.p_matrix(P, C)
+    tp = time.perf_counter() - tp
+    rec, _, _, st = call_parallel(P, sub, p, lo, hi, procs=procs)
+    wall = time.perf_counter() - t0
+    return rec, {"wall_s": wall, "cpu_s": cst["cpu_s"] + tp + st["cpu_s"], "procs": st["procs"],
+                 "sites": hi - lo, "reads": rb - ra}
+
+
+def cpu_baseline_full(w, rec_gpu=None):
+    """cpu_baseline: the oracle as it stands over the WHOLE shard (calibration + every site) on all
+    host cores.  Also compares its records with the GPU's (full-config parity counters)."""
+    lo, hi = w["region"]
+    rec, st = _oracle_step(w, lo, hi)
+    out = {"value": st["sites"] / st["wall_s"], "unit": UNIT, "cores": st["procs"], "kind": "oracle",
+           "sample": f"the whole shard: calibration over all {st['reads']} reads + all {st['sites']} "
+                     f"sites, {st['procs']} single-threaded oracle processes over windows",
+           "wall_s": round(st["wall_s"], 2), "core_seconds": round(st["cpu_s"], 1),
+           "per_core_value": st["sites"] / st["cpu_s"]}
+    if rec_gpu is not None and len(rec_gpu) == len(rec):
+        out["parity"] = {f: int(np.count_nonzero(rec_gpu[f] != rec[f]))
+                         for f in ("genotype", "quality", "base1", "base2", "depth", "cnt_uni1")}
+        out["parity"]["note"] = ("mismatching records per field, GPU vs oracle over the whole shard "
+                                 "(tests/test_gpu_fullsize.py applies the near-tie / near-integer rules)")
+    return out
 
 
 def run_reference(args):
+    """--impl reference: the oracle (this tier's reference arm) on the host cores, each step a
+    bounded contiguous sample (1/8) of the shard, timed step by step (measured ms_per_step)."""
     ws, rank, _ = _dist()
     if rank != 0:
         return 0
     w = make_shard(args.config, 0, 1)
-    for _ in range(args.warmup):
-        cpu_oracle_rate(w, budget_s=1.0, max_sites=20_000)
-    vals = []
-    desc = ""
-    for _ in range(args.steps):
-        v, desc = cpu_oracle_rate(w, budget_s=args.ref_budget)
-        vals.append(v)
-    v = float(np.median(vals))
     lo, hi = w["region"]
+    S = hi - lo
+    n = max(1, S // args.ref_frac)
+    s0 = lo + (S - n) // 2                       # mid-shard (C2 starts with its leading N block)
+    for _ in range(args.warmup):
+        _oracle_step(w, s0, s0 + max(1, n // 16))
+    times, st = [], None
+    for _ in range(args.steps):
+        _, st = _oracle_step(w, s0, s0 + n)
+        times.append(st["wall_s"])
+    ms = 1e3 * float(np.mean(times))
+    v = n / (ms / 1e3)
+    desc = (f"oracle calibrate+call over sites [{s0},{s0 + n}) (1/{args.ref_frac} of the {S}-site "
+            f"shard, {st['reads']} reads) per step, {st['procs']} single-threaded processes")
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
-            "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": 1e3 * (hi - lo) / v,        # the whole shard at the sampled rate
-            "ms_per_step_note": "projected: shard sites / sampled oracle rate",
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic", "config": {"workload": args.config, "sample": desc},
-            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": st["procs"], "kind": "oracle",
                              "sample": desc},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -267,8 +317,16 @@ def run_gpu(args):
         all_reduce_(t, dist.ReduceOp.MAX)
     ms_max = float(t.item())
     ms_step = ms_max / args.steps
-    total_sites = S * ws
+    # per-rank shard sizes (all-gathered; the max-over-ranks time above covers every rank)
+    mine = [S, int(len(w["pos"])), int(w["off"][-1] - w["off"][0]), float(ms_total / args.steps)]
+    if dist is not None:
+        allv = [None] * ws
+        dist.all_gather_object(allv, mine)
+    else:
+        allv = [mine]
+    total_sites = sum(int(v[0]) for v in allv)
     value = total_sites / (ms_step / 1e3)
+    strong = args.config in STRONG
 
     # ---- e2e: the same step through the public API with pinned host inputs and outputs, the
     # host->device copy of the reads and the device->host copy of the result inside the timed
@@ -442,7 +500,8 @@ def run_gpu(args):
     # Alg. 1 over per-site dense base_occ arrays (gsnp_call_dense) vs the sparse path, same
     # sub-window of this shard, same records.  CUDA events on the library's stream.
     dense = None
-    if not args.no_dense and ws == 1:         # side legs (outside the step) at N=1 only
+    side = ws == 1 and args.config not in STRONG      # side legs (outside the step): N=1, C1/C2/C5
+    if not args.no_dense and side:
         dlo = w0 + min(S // 4, 8_000_000)
         dhi = min(w1, dlo + (1 << 22))
         nd = dhi - dlo
@@ -480,7 +539,7 @@ def run_gpu(args):
     # ---- §8(f) NEXT #2, outside the step: input packing on the GPU — this shard's reads as SOAP
     # alignment text (resident in HBM), parsed into the gsnp_reads arrays (gsnp_parse_soap).
     parse = None
-    if not args.no_parse and ws == 1:
+    if not args.no_parse and side:
         import synth
         text = synth.soap_text(w, "chr21", 33)
         tdev = torch.frombuffer(bytearray(text), dtype=torch.uint8).cuda()
@@ -518,26 +577,31 @@ def run_gpu(args):
         if dist is not None:
             dist.destroy_process_group()
         return 0
-    # ---- roofline of the dominant kernel (k_call_tile).  Its dominant traffic is the score-table
-    # gather: one 80-byte row of T (Alg. 3) per unique aligned base, from L2 (the table is 2 MB).
-    # The ceiling for that access pattern is measured live by tools/l2_gather_peak (random 80-byte
-    # rows from an L2-resident table); the HBM view (algorithmic HBM bytes vs MEASURED_PEAKS) is
-    # reported beside it.  DESIGN.md §6.
+    # ---- roofline.  The metric is SURVEY.md §8(d)'s: METHOD bytes — what the
+    # method must move through HBM: 18.2 B per aligned base (2 B read input, 0.16 B read metadata,
+    # 4 B key write, 8 B sort read+write, 4 B key read) + 53 B per site (1 B reference, 12 B
+    # offsets and counters, 40 B record) — per launch of the dominant kernel, k_call_tile (a3-a8
+    # fused: it moves only the compulsory part of these bytes; keys stay on chip), over its average
+    # launch time (CUDA events on the library's stream), against MEASURED_PEAKS.json's HBM copy
+    # bandwidth.  Beside it: the whole step (+ the calibration's second read of the input,
+    # 2.16 B/base), k_calib_count's own stream, and the L2 view of the score-table gather (80 B per
+    # unique base vs the live gather ceiling of tools/l2_gather_peak).
     peak, peak_kind = _peaks()
     call_ms, call_n = st["call_tile"]
     call_avg_ms = call_ms / max(call_n, 1)
+    cal_ms, cal_n = st["calib_count"]
+    cal_avg_ms = cal_ms / max(cal_n, 1)
     nreads = int(len(w["pos"]))
     nbases = int(w["off"][-1] - w["off"][0])
-    hits_b = np.repeat(w["hits"], w["len"].astype(np.int64))
-    keys = int(np.count_nonzero((hits_b == 1) & (w["bases"] < 4)))
-    if nreads and (int(w["pos"][0]) < w0 or int(w["pos"][-1]) + 256 > w1):   # halo reads
-        site_b = np.repeat(w["pos"].astype(np.int64), w["len"].astype(np.int64)) + (
-            np.arange(nbases) - np.repeat(w["off"][:-1].astype(np.int64), w["len"].astype(np.int64)))
-        keys = int(np.count_nonzero((hits_b == 1) & (w["bases"] < 4) & (site_b >= w0) & (site_b < w1)))
-    # algorithmic HBM bytes of one k_call_tile launch: bases+quals (2 B/base), read metadata
-    # (pos 8 + len 2 + off 8 + strand 1 + hits 2 = 21 B/read), reference (1 B/site), records (40 B/site)
-    alg_bytes = 2 * nbases + 21 * nreads + 1 * S + 40 * S
-    hbm_achieved = alg_bytes / (call_avg_ms / 1e3) / 1e9
+    keys = count_keys(w, w0, w1)
+    method_call = 18.2 * nbases + 53.0 * S
+    call_gbs = method_call / (call_avg_ms / 1e3) / 1e9
+    own_reads = orb - ora
+    own_bases = int(w["off"][orb] - w["off"][ora]) if own_reads else 0
+    method_cal = 2.16 * own_bases                       # bases + quals + read metadata
+    cal_gbs = method_cal / (cal_avg_ms / 1e3) / 1e9 if cal_n else 0.0
+    step_gbs = (method_call + method_cal) / (ms_step / 1e3) / 1e9
+    compulsory = 2 * nbases + 21 * nreads + 1 * S + 40 * S    # fused kernel's HBM floor
     t_bytes = 80 * keys                              # score-table rows gathered per launch
     l2_achieved = t_bytes / (call_avg_ms / 1e3) / 1e9
     l2_peak, l2_kind = _l2_gather_peak(live=not args.no_cpu)
@@ -551,27 +615,44 @@ def run_gpu(args):
                 traffic = tr.get("bytes_per_launch")
         except Exception:
             traffic = None
-    cpu_v, cpu_desc = (None, None)
+    roofline = {
+        "bound": "hbm", "achieved": call_gbs, "peak": peak, "unit": "GB/s", "frac": call_gbs / peak,
+        "traffic": traffic, "peak_kind": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})",
+        "kernel": "k_call_tile", "launch_ms": call_avg_ms, "alg_bytes_per_launch": method_call,
+        "alg_bytes": "SURVEY §8(d) method bytes: 18.2 B per aligned base + 53 B per site",
+        "units_per_launch": {"bases": nbases, "sites": S, "unique_keys": keys},
+        "step_view": {"achieved": step_gbs, "frac": step_gbs / peak,
+                      "alg_bytes_per_step": method_call + method_cal,
+                      "alg_bytes": "k_call_tile's method bytes + the calibration read (2.16 B/base)"},
+        "calib_view": {"kernel": "k_calib_count", "launch_ms": cal_avg_ms, "achieved": cal_gbs,
+                       "frac": cal_gbs / peak, "alg_bytes_per_launch": method_cal},
+        "compulsory_view": {"alg_bytes_per_launch": compulsory,
+                            "achieved": compulsory / (call_avg_ms / 1e3) / 1e9,
+                            "note": "inputs 2 B/base + 21 B/read + ref 1 B/site + record 40 B/site"},
+        "l2_view": {"achieved": l2_achieved, "peak": l2_peak, "frac": l2_achieved / l2_peak,
+                    "peak_kind": l2_kind, "alg_bytes_per_launch": t_bytes,
+                    "alg_bytes": "80 B score-table row per unique base, gathered from L2"}}
+    cpu = None
     if not args.no_cpu and ws == 1:            # the oracle baseline: rank 0 at N=1 only
-        cpu_v, cpu_desc = cpu_oracle_rate(w, budget_s=args.ref_budget)
+        rec_gpu = out.cpu().numpy().view(gsnp.RECORD_DTYPE)
+        cpu = cpu_baseline_full(w, rec_gpu)
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "scaling": "strong" if strong else "weak", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic",
         "config": {"workload": args.config, "sites_per_gpu": S, "reads_per_gpu": nreads,
+                   "total_sites": total_sites,
+                   "per_rank": [{"sites": int(v[0]), "reads": int(v[1]), "bases": int(v[2]),
+                                 "ms_per_step": round(v[3], 3)} for v in allv],
                    "bases_per_gpu": nbases, "depth": synth_depth(args.config),
                    "read_len": 100, "l2": "inputs (%.2f GB/GPU) > L2 126 MB; no flush" %
-                   (input_bytes(w) / 1e9), "parallelism": f"shard{ws}",
+                   (input_bytes(w) / 1e9),
+                   "parallelism": f"shard{ws}" + (" (plan_by_bases)" if strong else ""),
                    "stage_ms_per_step": {k: round(v[0] / args.steps, 4) for k, v in st.items()},
                    "stage_share": stage_share},
-        "roofline": {"bound": "l2", "achieved": l2_achieved, "peak": l2_peak, "unit": "GB/s",
-                     "frac": l2_achieved / l2_peak, "traffic": traffic, "peak_kind": l2_kind,
-                     "kernel": "k_call_tile", "launch_ms": call_avg_ms,
-                     "alg_bytes_per_launch": t_bytes, "alg_bytes": "80 B score-table row per unique base",
-                     "hbm_view": {"achieved": hbm_achieved, "peak": peak, "peak_kind": peak_kind,
-                                  "frac": hbm_achieved / peak, "alg_bytes_per_launch": alg_bytes}},
-        "cpu_baseline": ({"value": cpu_v, "unit": UNIT, "cores": 1, "kind": "oracle",
-                          "sample": cpu_desc} if cpu_v else None),
+        "roofline": roofline,
+        "cpu_baseline": cpu,
         "e2e": e2e,
         "gpu_launches": launches,
         "clocks": clk.summary(),
@@ -600,7 +681,8 @@ def main():
     ap.add_argument("--impl", default="gsnp", choices=["gsnp", "reference"])
     ap.add_argument("--no-cpu", action="store_true",
                     help="skip the cpu_baseline leg and the live L2-gather microbenchmark")
-    ap.add_argument("--ref-budget", type=float, default=15.0)
+    ap.add_argument("--ref-frac", type=int, default=8,
+                    help="--impl reference: each step is this fraction (1/k) of the shard")
     ap.add_argument("--no-dense", action="store_true", help="skip the dense-ablation leg")
     ap.add_argument("--no-parse", action="store_true", help="skip the SOAP-text parsing leg")
     args = ap.parse_args()

@@ -97,6 +97,8 @@ def _lib():
     lib.syn_soap_text.restype = ctypes.c_uint64
     lib.syn_soap_text.argtypes = [ctypes.c_uint64] + [P] * 7 + [ctypes.c_char_p, ctypes.c_uint32,
                                                                ctypes.c_uint64, P]
+    lib.syn_n_intervals.restype = ctypes.c_uint64
+    lib.syn_n_intervals.argtypes = [ctypes.POINTER(_Cfg), P]
     lib.syn_known.restype = ctypes.c_uint64
     lib.syn_known.argtypes = [ctypes.POINTER(_Cfg), P, P, P, P, P]
     return lib
@@ -104,6 +106,44 @@ def _lib():
 
 def _p(a: np.ndarray):
     return a.ctypes.data_as(ctypes.c_void_p)
+
+
+def _cfg(cfg: SynthConfig) -> _Cfg:
+    return _Cfg(cfg.seed, cfg.n_sites, cfg.origin, cfg.depth, cfg.read_len, cfg.q_hi, cfg.n_frac,
+                cfg.n_lead_frac, cfg.n_blocks, cfg.het_rate, cfg.hom_rate, cfg.multi_hit_rate,
+                cfg.dup_rate, cfg.base_n_rate, cfg.known_frac, cfg.n_threads, 0, cfg.region_lo,
+                cfg.region_hi)
+
+
+def n_intervals(cfg: SynthConfig | str) -> np.ndarray:
+    """The genome's N blocks as an (k, 2) array of [begin, end) genome indices (no generation)."""
+    if isinstance(cfg, str):
+        cfg = CONFIGS[cfg]
+    lib = _lib()
+    c = _cfg(cfg)
+    k = lib.syn_n_intervals(ctypes.byref(c), None)
+    out = np.zeros(2 * max(k, 1), np.uint64)
+    lib.syn_n_intervals(ctypes.byref(c), _p(out))
+    return out[:2 * k].reshape(-1, 2).astype(np.int64)
+
+
+def sample_read_starts(cfg: SynthConfig | str, n: int = 1_000_000, seed: int = 0) -> np.ndarray:
+    """n read starts drawn uniformly over the genome's non-N sites (sorted): a thin sample with the
+    placement density of the generated reads, for planning shards (shard.plan_by_bases)."""
+    if isinstance(cfg, str):
+        cfg = CONFIGS[cfg]
+    iv = n_intervals(cfg)
+    cuts = [0]
+    for a, b in iv:
+        cuts += [int(a), int(b)]
+    cuts.append(cfg.n_sites)
+    seg = np.array(cuts, np.int64).reshape(-1, 2)          # non-N segments [a, b)
+    seg = seg[seg[:, 1] > seg[:, 0]]
+    w = (seg[:, 1] - seg[:, 0]).astype(np.float64)
+    rng = np.random.default_rng(seed)
+    k = rng.choice(len(seg), n, p=w / w.sum())
+    pos = seg[k, 0] + (rng.random(n) * (seg[k, 1] - seg[k, 0])).astype(np.int64)
+    return np.sort(pos).astype(np.uint64) + np.uint64(cfg.origin)
 
 
 def generate(cfg: SynthConfig | str, **overrides) -> dict:

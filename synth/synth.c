@@ -274,6 +274,28 @@ static uint64_t run_jobs(const syn_config* c, const uint8_t* ref, const uint8_t*
     return total;
 }
 
+/* The N blocks of the whole genome as [begin, end) genome indices (the leading block first, then
+ * the interior blocks in order; empty blocks omitted), the same placement make_reference uses.
+ * out holds 2 * (n_blocks + 1) entries (NULL: count only); returns the number of intervals.
+ * Lets a multi-GPU run plan shards by expected aligned bases without generating the genome. */
+uint64_t syn_n_intervals(const syn_config* c, uint64_t* out) {
+    uint64_t n = c->n_sites, k = 0;
+    uint64_t lead = (uint64_t)(c->n_lead_frac * (double)n);
+    if (lead > n) lead = n;
+    if (lead) { if (out) { out[0] = 0; out[1] = lead; } ++k; }
+    double rest = c->n_frac - c->n_lead_frac;
+    if (rest > 0 && c->n_blocks > 0 && n > lead) {
+        uint64_t blk = (uint64_t)(rest * (double)n / c->n_blocks);
+        uint64_t span = (n - lead) / c->n_blocks;
+        for (uint32_t j = 0; j < c->n_blocks; ++j) {
+            uint64_t jit = span > blk ? h4(c->seed, T_NBLK, j, 0) % (span - blk) : 0;
+            uint64_t st = lead + (uint64_t)j * span + jit, en = st + blk < n ? st + blk : n;
+            if (en > st) { if (out) { out[2 * k] = st; out[2 * k + 1] = en; } ++k; }
+        }
+    }
+    return k;
+}
+
 /* Phase 1: reference window, SNPs, eligibility (arrays of g1 - g0); returns the read count. */
 uint64_t syn_plan(const syn_config* c, uint8_t* ref, uint8_t* snp, uint8_t* alt, uint8_t* elig) {
     if (c->read_len == 0 || c->read_len > 256 || c->n_sites == 0) return (uint64_t)-1;
