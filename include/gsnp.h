@@ -70,7 +70,8 @@ typedef int32_t gsnp_status;
 #define GSNP_STAGE_DENSE_LIK 9      /* k_dense_sites (dense Alg. 1 + posterior + record) */
 #define GSNP_STAGE_DENSE_RECYCLE 10 /* re-zeroing base_occ after each chunk (memset) */
 #define GSNP_STAGE_PARSE 11         /* k_nl_tiles, k_parse_meta, k_sel_*, k_parse_emit (gsnp_parse_soap) */
-#define GSNP_N_STAGES 12
+#define GSNP_STAGE_UNPACK 12        /* k_unpack (gsnp_unpack_reads, packed reads R21) */
+#define GSNP_N_STAGES 13
 
 typedef struct gsnp_ctx gsnp_ctx;  /* opaque; owned by the library until gsnp_destroy */
 
@@ -180,6 +181,34 @@ gsnp_status gsnp_parse_soap(gsnp_ctx* ctx, const char* text, uint64_t n_bytes, c
                             uint64_t* off, uint8_t* bases, uint8_t* quals, uint8_t* strand,
                             uint16_t* hits, uint64_t reads_cap, uint64_t bases_cap,
                             uint64_t* n_reads, uint64_t* n_bases);
+
+/* SURVEY.md §8(f) NEXT #2, second half — the compressed copy of the input (PAPER.md P:L708-727,
+ * §V-A: GSNP's first pass writes it, about a third of the input's size, for the second pass).  Here
+ * it is what crosses PCIe: reading R21 of DESIGN.md (oracle/pack.py), a stream of 2-bit bases
+ * with an N exception list, qualities as maximal runs of equal value inside each read
+ * (P:L761-764), and 6 bytes of metadata per read (position relative to its block of block_reads
+ * reads, length, strand | hits, run count; hits >= 128 as exceptions) — ~47 bytes per 100-bp read
+ * against 221 unpacked.
+ *
+ * gsnp_pack_reads: encode host reads (on_device 0; bases contiguous per read at off[r]) on the
+ *   host's cores.  block_reads 1..4096.  out: host buffer of cap bytes; *n_bytes receives the
+ *   stream size (also on GSNP_E_CAPACITY, when out is NULL or cap too small — a size query).
+ *   A length outside 1..256, base > 4, quality > 63, strand > 1, hits 0, or a position before its
+ *   block's first read or >= 2^32 past it -> GSNP_E_RANGE.  No context needed.
+ * gsnp_packed_sizes: n_reads / n_bases of a stream (host memory; the header is checked).
+ * gsnp_unpack_reads: decode a stream (host — copied H2D in chunks on the library's copy stream,
+ *   overlapped with the decode — or device memory) into DEVICE arrays sized by gsnp_packed_sizes
+ *   (off: n_reads + 1 entries, rebuilt contiguous from 0).  Work is stream-ordered on
+ *   params.stream; the call returns once a host stream has been copied (it may be reused).  The
+ *   decoded reads are then passed to gsnp_calibrate / gsnp_call like any device reads (they are
+ *   validated there).  A bad header -> GSNP_E_INVAL. */
+gsnp_status gsnp_pack_reads(const gsnp_reads* reads, uint32_t block_reads, void* out, uint64_t cap,
+                            uint64_t* n_bytes);
+gsnp_status gsnp_packed_sizes(const void* packed, uint64_t n_bytes, uint64_t* n_reads,
+                              uint64_t* n_bases);
+gsnp_status gsnp_unpack_reads(gsnp_ctx* ctx, const void* packed, uint64_t n_bytes, uint64_t* pos,
+                              uint16_t* len, uint64_t* off, uint8_t* bases, uint8_t* quals,
+                              uint8_t* strand, uint16_t* hits);
 
 /* Call sites [w0, w1) (global coordinates inside the reference): one gsnp_record per site,
  * written to out[0 .. w1-w0).  reads must include every read overlapping the window (the

@@ -11,6 +11,7 @@ SRC_DEEP = os.path.join(HERE, "csrc", "gsnp_deep.cu")   # deep-window kernel, 38
 DEPS = [SRC, SRC_DEEP, os.path.join(HERE, "csrc", "gsnp_kernels.cuh"),
         os.path.join(HERE, "csrc", "gsnp_compress.cuh"), os.path.join(HERE, "csrc", "gsnp_dense.cuh"),
         os.path.join(HERE, "csrc", "gsnp_parse.cuh"),
+        os.path.join(HERE, "csrc", "gsnp_pack.cuh"),
         os.path.join(ROOT, "include", "gsnp.h")]
 LIB = os.path.join(HERE, "libgsnp.so")
 

@@ -23,6 +23,7 @@
 #include "gsnp_compress.cuh"
 #include "gsnp_dense.cuh"
 #include "gsnp_parse.cuh"
+#include "gsnp_pack.cuh"
 
 using namespace gsnp_dev;
 
@@ -115,6 +116,10 @@ struct gsnp_ctx {
     // delay the read
     uint64_t* mbox = nullptr;
     uint64_t launches = 0;
+    // packed reads (R21): device copy of a host stream, the copy stream and its chunk events
+    DevBuf<uint8_t> pk_buf;
+    cudaStream_t copy_stream = nullptr;
+    std::vector<cudaEvent_t> pk_ev;
     // per-device facts, read at gsnp_create on prm.device (a process may hold contexts on
     // several devices)
     int num_sms = 148;
@@ -1140,6 +1145,187 @@ gsnp_status gsnp_parse_soap(gsnp_ctx* ctx, const char* text, uint64_t n_bytes, c
     return GSNP_OK;
 }
 
+gsnp_status gsnp_pack_reads(const gsnp_reads* reads, uint32_t block_reads, void* out, uint64_t cap,
+                            uint64_t* n_bytes) {
+    using namespace gsnp_pk;
+    if (n_bytes) *n_bytes = 0;
+    if (!reads || reads->on_device) return GSNP_E_INVAL;
+    if (block_reads < 1 || block_reads > MAX_BLOCK) return GSNP_E_INVAL;
+    const uint64_t n = reads->n_reads;
+    if (n && (!reads->pos || !reads->len || !reads->off || !reads->bases || !reads->quals ||
+              !reads->strand || !reads->hits)) return GSNP_E_INVAL;
+    HostReads R{n, reads->pos, reads->len, reads->off, reads->bases, reads->quals, reads->strand,
+                reads->hits};
+    const uint64_t nblk = (n + block_reads - 1) / block_reads;
+    std::vector<BlockSize> bs(nblk);
+    const int nt = (int)std::max(1u, std::min(32u, std::thread::hardware_concurrency()));
+    auto par = [&](auto&& fn) {                  // fn(block) over all blocks on nt threads
+        std::atomic<uint64_t> next{0};
+        auto work = [&] { for (uint64_t b; (b = next.fetch_add(1)) < nblk;) fn(b); };
+        std::vector<std::thread> th;
+        for (int i = 1; i < nt && (uint64_t)i < nblk; ++i) th.emplace_back(work);
+        work();
+        for (auto& t : th) t.join();
+    };
+    par([&](uint64_t b) {
+        bs[b] = size_block(R, b * block_reads, std::min(n, (b + 1) * block_reads));
+    });
+    std::vector<uint64_t> table(5 * nblk);
+    Header h{};
+    for (uint64_t b = 0; b < nblk; ++b) {
+        if (bs[b].bad) return GSNP_E_RANGE;
+        uint64_t* t = table.data() + 5 * b;
+        t[0] = R.pos[b * block_reads];
+        t[1] = h.n_bases; t[2] = h.n_runs; t[3] = h.n_nexc; t[4] = h.n_hexc;
+        h.n_bases += bs[b].bases; h.n_runs += bs[b].runs; h.n_nexc += bs[b].nexc; h.n_hexc += bs[b].hexc;
+    }
+    h.n_reads = n;
+    h.n_blocks = (uint32_t)nblk;
+    h.block_reads = block_reads;
+    h.sec[0] = HDR;
+    h.sec[1] = a16(h.sec[0] + 40 * nblk);
+    meta_offsets(h);
+    h.sec[2] = a16(h.m_nrun + n);
+    h.sec[3] = a16(h.sec[2] + (h.n_bases + 3) / 4);
+    h.sec[4] = a16(h.sec[3] + 2 * h.n_runs);
+    h.sec[5] = a16(h.sec[4] + 4 * h.n_nexc);
+    const uint64_t total = a16(h.sec[5] + 8 * h.n_hexc);
+    if (n_bytes) *n_bytes = total;
+    if (!out || cap < total) return GSNP_E_CAPACITY;
+    uint8_t* o = static_cast<uint8_t*>(out);
+    memset(o, 0, HDR);
+    const uint32_t magic = MAGIC, ver = 1;
+    memcpy(o, &magic, 4); memcpy(o + 4, &ver, 4);
+    memcpy(o + 8, &h.n_reads, 8); memcpy(o + 16, &h.n_bases, 8); memcpy(o + 24, &h.n_runs, 8);
+    memcpy(o + 32, &h.n_nexc, 8); memcpy(o + 40, &h.n_hexc, 8); memcpy(o + 48, &h.n_blocks, 4);
+    memcpy(o + 52, &h.block_reads, 4); memcpy(o + 56, h.sec, 48);
+    // zero every padding gap and the 2-bit plane (edge bytes are OR-ed by neighbouring blocks)
+    auto zero = [&](uint64_t a, uint64_t b) { if (b > a) memset(o + a, 0, b - a); };
+    zero(h.sec[0] + 40 * nblk, h.sec[1]);
+    zero(h.m_pos + 4 * n, h.m_len); zero(h.m_len + n, h.m_sh); zero(h.m_sh + n, h.m_nrun);
+    zero(h.m_nrun + n, h.sec[2]);
+    zero(h.sec[2], h.sec[3]);
+    zero(h.sec[3] + 2 * h.n_runs, h.sec[4]); zero(h.sec[4] + 4 * h.n_nexc, h.sec[5]);
+    zero(h.sec[5] + 8 * h.n_hexc, total);
+    if (nblk) memcpy(o + h.sec[0], table.data(), 40 * nblk);
+    par([&](uint64_t b) {
+        write_block(R, b * block_reads, std::min(n, (b + 1) * block_reads), h, table.data() + 5 * b, o);
+    });
+    return GSNP_OK;
+}
+
+gsnp_status gsnp_packed_sizes(const void* packed, uint64_t n_bytes, uint64_t* n_reads,
+                              uint64_t* n_bases) {
+    gsnp_pk::Header h;
+    if (!packed || !gsnp_pk::parse_header(static_cast<const uint8_t*>(packed), n_bytes, h))
+        return GSNP_E_INVAL;
+    if (n_reads) *n_reads = h.n_reads;
+    if (n_bases) *n_bases = h.n_bases;
+    return GSNP_OK;
+}
+
+gsnp_status gsnp_unpack_reads(gsnp_ctx* ctx, const void* packed, uint64_t n_bytes, uint64_t* pos,
+                              uint16_t* len, uint64_t* off, uint8_t* bases, uint8_t* quals,
+                              uint8_t* strand, uint16_t* hits) {
+    using namespace gsnp_pk;
+    if (!ctx) return GSNP_E_INVAL;
+    if (cudaSetDevice(ctx->prm.device) != cudaSuccess) return fail(ctx, GSNP_E_CUDA, "set device");
+    if (!packed) return fail(ctx, GSNP_E_INVAL, "packed == NULL");
+    cudaStream_t s = ctx->stream;
+    const uint8_t* pk = static_cast<const uint8_t*>(packed);
+    const bool dev_in = is_device_ptr(packed);
+    Header h;
+    uint8_t hb[HDR];
+    if (n_bytes < HDR) return fail(ctx, GSNP_E_INVAL, "packed stream shorter than its header");
+    if (dev_in) {
+        CK(cudaMemcpyAsync(hb, pk, HDR, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+    } else {
+        memcpy(hb, pk, HDR);
+    }
+    if (!parse_header(hb, n_bytes, h)) return fail(ctx, GSNP_E_INVAL, "not a GSR1 packed-read stream");
+    if (!off || (h.n_reads && (!pos || !len || !strand || !hits)) || (h.n_bases && (!bases || !quals)))
+        return fail(ctx, GSNP_E_INVAL, "NULL output array");
+    if (!is_device_ptr(off) || (h.n_reads && !is_device_ptr(pos)) || (h.n_bases && !is_device_ptr(bases)))
+        return fail(ctx, GSNP_E_INVAL, "outputs must be device arrays");
+    UnpackArgs U;
+    memset(&U, 0, sizeof U);
+    U.h = h;
+    U.pos = pos; U.len = len; U.off = off; U.bases = bases; U.quals = quals; U.strand = strand;
+    U.hits = hits;
+    if (h.n_reads == 0) {
+        CK(cudaMemsetAsync(off, 0, 8, s));
+        CK(cudaStreamSynchronize(s));
+        return GSNP_OK;
+    }
+    if (dev_in && (reinterpret_cast<uintptr_t>(pk) & 15) == 0) {
+        U.buf = pk;                                  // in place: one launch over every block
+        ctx->begin();
+        k_unpack<<<h.n_blocks, UNT, 0, s>>>(U);
+        ctx->end(GSNP_STAGE_UNPACK);
+        ctx->launches++;
+        CK(cudaGetLastError());
+        return GSNP_OK;
+    }
+    CK(ctx->pk_buf.ensure(n_bytes));
+    U.buf = ctx->pk_buf.p;
+    if (dev_in) {                                    // unaligned device stream: one D2D copy
+        CK(cudaMemcpyAsync(ctx->pk_buf.p, pk, n_bytes, cudaMemcpyDeviceToDevice, s));
+        ctx->begin();
+        k_unpack<<<h.n_blocks, UNT, 0, s>>>(U);
+        ctx->end(GSNP_STAGE_UNPACK);
+        ctx->launches++;
+        CK(cudaGetLastError());
+        return GSNP_OK;
+    }
+    // host stream: the header and block table first, then chunks of blocks — each chunk's slices
+    // of every section on the copy stream, its decode on the library stream once they landed
+    if (!ctx->copy_stream) CK(cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking));
+    cudaStream_t cs = ctx->copy_stream;
+    const uint64_t* bt = reinterpret_cast<const uint64_t*>(pk + h.sec[0]);
+    const uint32_t K = (uint32_t)std::min<uint64_t>(h.n_blocks, 8);
+    while (ctx->pk_ev.size() < K + 1) {
+        cudaEvent_t e;
+        CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        ctx->pk_ev.push_back(e);
+    }
+    CK(cudaEventRecord(ctx->pk_ev[K], s));           // the buffer is free once earlier work is done
+    CK(cudaStreamWaitEvent(cs, ctx->pk_ev[K], 0));
+    CK(cudaMemcpyAsync(ctx->pk_buf.p, pk, h.sec[1], cudaMemcpyHostToDevice, cs));
+    auto cp = [&](uint64_t a, uint64_t b) -> cudaError_t {
+        return b > a ? cudaMemcpyAsync(ctx->pk_buf.p + a, pk + a, b - a, cudaMemcpyHostToDevice, cs)
+                     : cudaSuccess;
+    };
+    auto brow = [&](uint32_t b, int f) -> uint64_t {  // block b's counter f (b == n_blocks: totals)
+        if (b < h.n_blocks) return bt[5ull * b + f];
+        const uint64_t tot[5] = {0, h.n_bases, h.n_runs, h.n_nexc, h.n_hexc};
+        return tot[f];
+    };
+    for (uint32_t k = 0; k < K; ++k) {
+        const uint32_t b0 = (uint32_t)((uint64_t)h.n_blocks * k / K);
+        const uint32_t b1 = (uint32_t)((uint64_t)h.n_blocks * (k + 1) / K);
+        const uint64_t r0 = (uint64_t)b0 * h.block_reads, r1 = std::min(h.n_reads, (uint64_t)b1 * h.block_reads);
+        CK(cp(h.m_pos + 4 * r0, h.m_pos + 4 * r1));
+        CK(cp(h.m_len + r0, h.m_len + r1));
+        CK(cp(h.m_sh + r0, h.m_sh + r1));
+        CK(cp(h.m_nrun + r0, h.m_nrun + r1));
+        CK(cp(h.sec[2] + brow(b0, 1) / 4, h.sec[2] + (brow(b1, 1) + 3) / 4));
+        CK(cp(h.sec[3] + 2 * brow(b0, 2), h.sec[3] + 2 * brow(b1, 2)));
+        CK(cp(h.sec[4] + 4 * brow(b0, 3), h.sec[4] + 4 * brow(b1, 3)));
+        CK(cp(h.sec[5] + 8 * brow(b0, 4), h.sec[5] + 8 * brow(b1, 4)));
+        CK(cudaEventRecord(ctx->pk_ev[k], cs));
+        CK(cudaStreamWaitEvent(s, ctx->pk_ev[k], 0));
+        U.blk0 = b0;
+        ctx->begin();
+        k_unpack<<<b1 - b0, UNT, 0, s>>>(U);
+        ctx->end(GSNP_STAGE_UNPACK);
+        ctx->launches++;
+        CK(cudaGetLastError());
+    }
+    CK(cudaStreamSynchronize(cs));                   // the host stream may be reused on return
+    return GSNP_OK;
+}
+
 gsnp_status gsnp_compress(gsnp_ctx* ctx, const gsnp_record* rec, uint64_t n, uint32_t block_sites,
                           uint32_t* out, uint64_t out_cap, uint64_t* n_words) {
     if (!ctx) return GSNP_E_INVAL;
@@ -1305,6 +1491,9 @@ void gsnp_destroy(gsnp_ctx* ctx) {
     if (ctx->mbox) cudaFreeHost(ctx->mbox);
     if (ctx->h_T) cudaFreeHost(ctx->h_T);
     if (ctx->h_cnt_pinned) cudaFreeHost(ctx->h_cnt_pinned);
+    ctx->pk_buf.release();
+    for (auto e : ctx->pk_ev) cudaEventDestroy(e);
+    if (ctx->copy_stream) cudaStreamDestroy(ctx->copy_stream);
     for (auto& p : ctx->pending) { cudaEventDestroy(p.a); cudaEventDestroy(p.b); }
     for (auto e : ctx->ev_pool) cudaEventDestroy(e);
     delete ctx;

@@ -20,7 +20,7 @@ GSNP_MONOPLOID = 0x4
 GSNP_TITV = 0x8
 GSNP_RANK_EXACT = 0x10      # R20 exact small-sample rank-sum (include/gsnp.h)
 STAGES = ("validate", "calib_count", "tile_ranges", "call_tile", "finalize", "big_sites",
-          "compress", "warp_sites", "dense_count", "dense_lik", "dense_recycle", "parse")
+          "compress", "warp_sites", "dense_count", "dense_lik", "dense_recycle", "parse", "unpack")
 STATUS = {0: "GSNP_OK", -1: "GSNP_E_INVAL", -2: "GSNP_E_RANGE", -3: "GSNP_E_UNSORTED",
           -4: "GSNP_E_STATE", -5: "GSNP_E_NOMEM", -6: "GSNP_E_CUDA", -7: "GSNP_E_CAPACITY"}
 
@@ -28,6 +28,7 @@ STATUS = {0: "GSNP_OK", -1: "GSNP_E_INVAL", -2: "GSNP_E_RANGE", -3: "GSNP_E_UNSO
 SYMBOLS = ("gsnp_params_default", "gsnp_create", "gsnp_calibrate", "gsnp_calibrate_count",
            "gsnp_calibrate_finalize", "gsnp_call", "gsnp_debug_window", "gsnp_get_tables",
            "gsnp_compress", "gsnp_call_compressed", "gsnp_call_dense", "gsnp_priors_from_freq", "gsnp_parse_soap",
+           "gsnp_pack_reads", "gsnp_packed_sizes", "gsnp_unpack_reads",
            "gsnp_launch_count", "gsnp_stage_times", "gsnp_strerror", "gsnp_last_error",
            "gsnp_destroy")
 
@@ -113,6 +114,13 @@ def lib():
         L.gsnp_parse_soap.restype = S
         L.gsnp_parse_soap.argtypes = [P, P, u64, ctypes.c_char_p, ctypes.c_uint32, u64] + [P] * 7 + \
             [u64, u64, ctypes.POINTER(u64), ctypes.POINTER(u64)]
+        L.gsnp_pack_reads.restype = S
+        L.gsnp_pack_reads.argtypes = [ctypes.POINTER(gsnp_reads), ctypes.c_uint32, P, u64,
+                                      ctypes.POINTER(u64)]
+        L.gsnp_packed_sizes.restype = S
+        L.gsnp_packed_sizes.argtypes = [P, u64, ctypes.POINTER(u64), ctypes.POINTER(u64)]
+        L.gsnp_unpack_reads.restype = S
+        L.gsnp_unpack_reads.argtypes = [P, P, u64] + [P] * 7
         L.gsnp_launch_count.restype = u64
         L.gsnp_launch_count.argtypes = [P]
         L.gsnp_stage_times.restype = S
@@ -356,6 +364,26 @@ class Context:
                     out[k] = out[k][:K]
         return out
 
+    def unpack_reads(self, packed, out=None):
+        """gsnp_unpack_reads: a packed stream (numpy / pinned or CUDA tensor) -> device read
+        arrays (dict of CUDA tensors; allocated when out is None)."""
+        import torch
+        n_reads, n_bases = packed_sizes(packed)
+        if out is None:
+            dev = "cuda"
+            out = dict(pos=torch.empty(n_reads, dtype=torch.uint64, device=dev),
+                       len=torch.empty(n_reads, dtype=torch.uint16, device=dev),
+                       off=torch.empty(n_reads + 1, dtype=torch.uint64, device=dev),
+                       bases=torch.empty(max(n_bases, 1), dtype=torch.uint8, device=dev),
+                       quals=torch.empty(max(n_bases, 1), dtype=torch.uint8, device=dev),
+                       strand=torch.empty(n_reads, dtype=torch.uint8, device=dev),
+                       hits=torch.empty(n_reads, dtype=torch.uint16, device=dev))
+        nb = _nbytes(packed)
+        _check(lib().gsnp_unpack_reads(self.h, _ptr(packed), nb, *[_ptr(out[k]) for k in
+                                       ("pos", "len", "off", "bases", "quals", "strand", "hits")]),
+               self.h)
+        return out
+
     def get_tables(self, calibrated: bool = True):
         dims = np.zeros(3, np.uint32)
         _check(lib().gsnp_get_tables(self.h, None, None, None, None, _ptr(dims)), self.h)
@@ -387,6 +415,36 @@ class Context:
 
 
 # ABI-named free functions (thin aliases)
+def _nbytes(a) -> int:
+    if hasattr(a, "element_size"):
+        return a.numel() * a.element_size()
+    return np.asarray(a).nbytes
+
+
+def pack_reads(reads: dict, block_reads: int = 1024) -> np.ndarray:
+    """gsnp_pack_reads: host read arrays -> the packed stream R21 (numpy uint8)."""
+    r = make_reads(reads)
+    n = ctypes.c_uint64(0)
+    st = lib().gsnp_pack_reads(ctypes.byref(r), block_reads, None, 0, ctypes.byref(n))
+    if st not in (0, -7):
+        _check(st, None)
+    out = np.zeros(max(int(n.value), 1), np.uint8)
+    _check(lib().gsnp_pack_reads(ctypes.byref(r), block_reads, _ptr(out), out.nbytes,
+                                 ctypes.byref(n)), None)
+    return out[:int(n.value)]
+
+
+def packed_sizes(packed) -> tuple:
+    """(n_reads, n_bases) of a packed stream (its header is read from host memory)."""
+    hdr = packed[:128]
+    if hasattr(hdr, "cpu"):
+        hdr = hdr.cpu().numpy()
+    hdr = np.ascontiguousarray(hdr, np.uint8)
+    a, b = ctypes.c_uint64(0), ctypes.c_uint64(0)
+    _check(lib().gsnp_packed_sizes(_ptr(hdr), _nbytes(packed), ctypes.byref(a), ctypes.byref(b)), None)
+    return int(a.value), int(b.value)
+
+
 def gsnp_create(ref, origin=0, known_pos=None, known_prior10=None, **params) -> Context:
     return Context(ref, origin, known_pos, known_prior10, **params)
 
