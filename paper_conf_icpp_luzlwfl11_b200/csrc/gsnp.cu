@@ -123,6 +123,9 @@ struct gsnp_ctx {
     // per-device facts, read at gsnp_create on prm.device (a process may hold contexts on
     // several devices)
     int num_sms = 148;
+    // window depth thresholds of the 64- / 128-slot k_call_tile instantiations (pick_variant)
+    float mid_at = 24.0f, deep_at = 48.0f;
+    bool mid_adj_smem = false;        // the 64-slot kernel reads adj from L1/L2: 3 CTAs per SM
     size_t cal_budget = 0;            // k_calib_count shared-memory budget (0 = not yet sized)
     // per-stage timing (GSNP_TIMING)
     struct Pending { int stage; cudaEvent_t a, b; };
@@ -471,49 +474,44 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
 #define GSNP_ADJ_SMEM_MAX (48 * 1024)
 #endif
     const uint32_t adj_smem = adj_bytes <= GSNP_ADJ_SMEM_MAX ? 1u : 0u;
-    // deep windows (mean depth >= 48 by read count) keep up to 128 keys per thread
-    uint64_t rr[2] = {0, 0};
-    if (d.n) {
-        gsnp_status pst;
-        if ((pst = peek(ctx, 0, ctx->tile_ra.p, 8))) return pst;
-        if ((pst = peek(ctx, 1, ctx->tile_rb.p + n_groups - 1, 8))) return pst;
-        CK(cudaStreamSynchronize(s));
-        rr[0] = ctx->mbox[0];
-        rr[1] = ctx->mbox[1];
-    }
-    const double depth_est = (double)(rr[1] - rr[0]) * A.L / (double)(w1 - w0);
-    const bool deep = depth_est >= 48.0;
-    const int cols = deep ? COLS_DEEP : COLS;
-    const size_t smem = call_smem_bytes(A.L, adj_smem ? adj_bytes : 0, cols, nullptr, nullptr);
+    // the three k_call_tile instantiations (32 / 64 / 128 key slots per thread) are all launched;
+    // each reads the window's depth from the read ranges on the device and only the one that fits
+    // the window does the work (pick_variant) — no host round trip
+    A.mid_at = ctx->mid_at;
+    A.deep_at = ctx->deep_at;
     const uint32_t big_cap = (uint32_t)std::min<uint64_t>(w1 - w0, 1u << 22);
     CK(ctx->big.ensure(big_cap));
     CK(ctx->wlist.ensure(w1 - w0));                 // sites for k_warp_sites (at most all)
     CK(ctx->big_n.ensure(3));
     CK(cudaMemsetAsync(ctx->big_n.p, 0, 12, s));    // [0] big sites, [1] work counter, [2] wlist
     const bool dbg = A.count_only || A.dbg_off || A.dbg_counters || A.dbg_L10 || A.dbg_post10;
-    if (deep) {
-        ctx->begin();
-        CK(gsnp_deep::launch_call_tile_deep(&A, sizeof A, dbg, ctx->num_sms, adj_bytes, adj_smem,
-                                            ctx->wlist.p, ctx->big_n.p + 2, ctx->big_n.p + 1, s));
-        ctx->end(GSNP_STAGE_CALL);
-        ctx->launches++;
-    } else {
-        auto kern = dbg ? k_call_tile<true, COLS> : k_call_tile<false, COLS>;
+    auto launch_tile = [&](auto kern, int cols, uint32_t adj_on) -> gsnp_status {
+        const size_t smem = call_smem_bytes(A.L, adj_on ? adj_bytes : 0, cols, nullptr, nullptr, false);
         CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         int per_sm = 0;
         CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NT, smem));
         const uint64_t want = (uint64_t)ctx->num_sms * std::max(per_sm, 1);
         const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, n_tiles));
         ctx->begin();
-        kern<<<grid, NT, smem, s>>>(A, ctx->wlist.p, ctx->big_n.p + 2, ctx->big_n.p + 1, adj_smem);
+        kern<<<grid, NT, smem, s>>>(A, ctx->wlist.p, ctx->big_n.p + 2, ctx->big_n.p + 1, adj_on);
         ctx->end(GSNP_STAGE_CALL);
         ctx->launches++;
         CK(cudaGetLastError());
-    }
+        return GSNP_OK;
+    };
+    gsnp_status lst;
+    if ((lst = launch_tile(dbg ? k_call_tile<true, COLS> : k_call_tile<false, COLS>, COLS, adj_smem))) return lst;
+    if ((lst = launch_tile(dbg ? k_call_tile<true, COLS_MID> : k_call_tile<false, COLS_MID>, COLS_MID,
+                           adj_smem && ctx->mid_adj_smem))) return lst;
+    ctx->begin();
+    CK(gsnp_deep::launch_call_tile_deep(&A, sizeof A, dbg, ctx->num_sms, adj_bytes, adj_smem,
+                                        ctx->wlist.p, ctx->big_n.p + 2, ctx->big_n.p + 1, s));
+    ctx->end(GSNP_STAGE_CALL);
+    ctx->launches++;
     if (!A.count_only) {
         // listed sites (n > 32 keys, or beyond the deep kernel's thread path): warp per site
-        auto wk = deep ? k_warp_sites<COLS_DEEP> : k_warp_sites<COLS>;
-        const size_t wsm = call_smem_bytes(A.L, 0, cols, nullptr, nullptr);
+        auto wk = k_warp_sites<COLS>;
+        const size_t wsm = call_smem_bytes(A.L, 0, COLS, nullptr, nullptr);
         CK(cudaFuncSetAttribute(wk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)wsm));
         int wper = 0;
         CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&wper, wk, NT, wsm));
@@ -783,6 +781,9 @@ gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
         int sms = 0;
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, params->device);
         ctx->num_sms = sms > 0 ? sms : 148;
+        if (const char* e = getenv("GSNP_MID_AT")) ctx->mid_at = (float)atof(e);
+        if (const char* e = getenv("GSNP_DEEP_AT")) ctx->deep_at = (float)atof(e);
+        if (const char* e = getenv("GSNP_MID_ADJ_SMEM")) ctx->mid_adj_smem = atoi(e) != 0;
     }
     ctx->n_sites = ref->n_sites;
     ctx->origin = ref->origin;

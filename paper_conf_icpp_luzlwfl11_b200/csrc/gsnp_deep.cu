@@ -28,10 +28,10 @@ cudaError_t launch_call_tile_deep(const void* args, size_t args_size, bool dbg, 
     if (args_size != sizeof(CallArgs)) return cudaErrorInvalidValue;
     CallArgs A;
     memcpy(&A, args, sizeof A);
-    size_t smem = call_smem_bytes(A.L, adj_smem ? adj_bytes : 0, COLS_DEEP, nullptr, nullptr);
+    size_t smem = call_smem_bytes(A.L, adj_smem ? adj_bytes : 0, COLS_DEEP, nullptr, nullptr, false);
     if (adj_smem && smem > 227 * 1024) {     // no room for the adjust table: read it from global
         adj_smem = 0;
-        smem = call_smem_bytes(A.L, 0, COLS_DEEP, nullptr, nullptr);
+        smem = call_smem_bytes(A.L, 0, COLS_DEEP, nullptr, nullptr, false);
     }
     auto kern = dbg ? k_call_tile<true, COLS_DEEP> : k_call_tile<false, COLS_DEEP>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);

@@ -67,6 +67,7 @@ struct CallArgs {
     const uint64_t* tile_rb;
     gsnp_record* out;                 // out[site - w0]
     int* err;
+    float mid_at, deep_at;            // window depth thresholds of the 64- and 128-slot kernels
     // debug (all may be null)
     uint32_t* dbg_nuni;               // count-only pass: unique keys per site
     const uint32_t* dbg_off;          // CSR offsets for the key dumps
@@ -538,6 +539,7 @@ constexpr int COLS = 32;              // key slots per site, shallow kernel (thr
 #define GSNP_GB 2
 #endif
 constexpr int GB = GSNP_GB;           // reads whose bytes are in flight together in the gather
+constexpr int COLS_MID = 64;          // key slots per site, mid-depth kernel (thread path n <= 64)
 constexpr int COLS_DEEP = 128;        // key slots per site, deep kernel (thread path n <= 128)
 
 struct TileSmem {
@@ -547,11 +549,13 @@ struct TileSmem {
     uint8_t* adj;        // copy of the adjust table (adj_bytes, 0 = use global)
 };
 
+// slot: reserve the per-warp dependency counters of the warp paths (k_warp_sites); k_call_tile
+// leaves them out
 __host__ __device__ inline size_t call_smem_bytes(int L, size_t adj_bytes, int cols, TileSmem* s,
-                                                   unsigned char* base) {
+                                                   unsigned char* base, bool slot = true) {
     size_t o_col = 0;
     size_t o_slot = align16(4 * (size_t)cols * TS);
-    size_t o_adj = align16(o_slot + (size_t)NW * 8 * L);
+    size_t o_adj = align16(o_slot + (slot ? (size_t)NW * 8 * L : 0));
     size_t total = align16(o_adj + adj_bytes);
     if (s) {
         s->col = reinterpret_cast<uint32_t*>(base + o_col);
@@ -1488,14 +1492,28 @@ struct BigSite {
 #ifndef GSNP_CALL_MINB
 #define GSNP_CALL_MINB 3
 #endif
+// Which k_call_tile instantiation calls this window (decided on the device, so gsnp_call needs no
+// host round trip): by the window's mean depth = reads overlapping it x L / sites (a3's read
+// ranges), the 32-slot kernel below mid_at, the 64-slot kernel below deep_at, the 128-slot kernel
+// (gsnp_deep.cu) above.  Every instantiation is launched; all but the chosen one return at once.
+// All of them give the same records: each sums a site's thread-path keys in canonical order, and
+// sites beyond their capacity go to the warp / CTA paths.
+__device__ __forceinline__ int pick_variant(const CallArgs& A) {
+    const uint64_t ng = (A.w1 - A.w0 + 31) / 32;
+    const uint64_t nr = A.tile_rb[ng - 1] - A.tile_ra[0];
+    const float depth = (float)((double)nr * A.L / (double)(A.w1 - A.w0));
+    return depth >= A.deep_at ? 2 : depth >= A.mid_at ? 1 : 0;
+}
+template <int CC> __host__ __device__ constexpr int variant_of() { return CC >= 128 ? 2 : CC >= 64 ? 1 : 0; }
+
 template <bool DBG, int CC>
 __global__ void __launch_bounds__(NT, GSNP_CALL_MINB)
 k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist_n, uint32_t* work, uint32_t adj_smem) {
-    if (reads_invalid(A.err)) return;
+    if (reads_invalid(A.err) || pick_variant(A) != variant_of<CC>()) return;
     extern __shared__ __align__(16) unsigned char smem[];
     TileSmem sm;
     const size_t adj_bytes = adj_smem ? (size_t)64 * A.adjP * A.adjG : 0;
-    call_smem_bytes(A.L, adj_bytes, CC, &sm, smem);
+    call_smem_bytes(A.L, adj_bytes, CC, &sm, smem, false);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     for (size_t i = tid; i < adj_bytes; i += NT) sm.adj[i] = A.adj[i];
     __shared__ double lp_s[50];                             // novel log10 priors [ref][n] (R6)
