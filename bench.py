@@ -533,6 +533,44 @@ def run_gpu(args):
                 "note": "device records -> device stream, whole shard; not part of the step "
                         "(SURVEY §8(f) #1)"}
 
+    # ---- windowed calling, outside the step: the paper calls a chromosome in windows of >= 256 K
+    # sites (Fig. 11).  The same shard in 2^18-site windows through
+    # gsnp_call_async (device reads, each window's read range with its halo; no host round trip
+    # per window) after one calibration; CUDA events on the library's stream.
+    windowed = None
+    if ws == 1 and args.config not in STRONG:
+        import synth
+        windowed = []
+        for WIN in (1 << 18, 1 << 22):
+          wins = [(a, min(w1, a + WIN)) for a in range(w0, w1, WIN)]
+          wrd = []
+          for a, b in wins:
+            ra, rb = synth.read_range(w, a, b)
+            wrd.append(gsnp.make_reads(dict(dev, pos=dev["pos"][ra:rb], len=dev["len"][ra:rb],
+                                            off=dev["off"][ra:rb + 1], strand=dev["strand"][ra:rb],
+                                            hits=dev["hits"][ra:rb])))
+
+          def win_step():
+            ctx.calibrate_count(owned(dev), counts)
+            ctx.calibrate_finalize(counts)
+            for (a, b), r in zip(wins, wrd):
+                ctx.call_async(r, a, b, out[40 * (a - w0):40 * (b - w0)])
+            ctx.wait()
+          win_step()
+          torch.cuda.synchronize()
+          ctx.stage_times(reset=True)
+          v0, v1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+          n_w = 3
+          v0.record(stream)
+          for _ in range(n_w):
+              win_step()
+          v1.record(stream)
+          torch.cuda.synchronize()
+          wms = v0.elapsed_time(v1) / n_w
+          windowed.append({"window_sites": WIN, "windows": len(wins), "ms_per_step": wms,
+                           "value": S / (wms / 1e3), "vs_one_window": ms_step / wms,
+                           "note": "calibration + every window through gsnp_call_async, one gsnp_wait"})
+
     # ---- §8(f) NEXT #3, outside the step: the dense ablation (Fig. 5) — SOAPsnp's
     # Alg. 1 over per-site dense base_occ arrays (gsnp_call_dense) vs the sparse path, same
     # sub-window of this shard, same records.  CUDA events on the library's stream.
@@ -624,10 +662,12 @@ def run_gpu(args):
     # 2.16 B/base), k_calib_count's own stream, and the L2 view of the score-table gather (80 B per
     # unique base vs the live gather ceiling of tools/l2_gather_peak).
     peak, peak_kind = _peaks()
+    # per call: gsnp_call launches the three k_call_tile instantiations (32/64/128 slots; the two
+    # the window's depth does not pick return at once) — their events sum to the call's kernel time
     call_ms, call_n = st["call_tile"]
-    call_avg_ms = call_ms / max(call_n, 1)
+    call_avg_ms = call_ms / args.steps
     cal_ms, cal_n = st["calib_count"]
-    cal_avg_ms = cal_ms / max(cal_n, 1)
+    cal_avg_ms = cal_ms / args.steps
     nreads = int(len(w["pos"]))
     nbases = int(w["off"][-1] - w["off"][0])
     keys = count_keys(w, w0, w1)
@@ -694,6 +734,7 @@ def run_gpu(args):
         "gpu_launches": launches,
         "clocks": clk.summary(),
         "compress": compress,
+        "windowed": windowed,
         "dense_ablation": dense,
         "parse": parse,
     }

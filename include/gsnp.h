@@ -58,10 +58,10 @@ typedef int32_t gsnp_status;
 #define GSNP_RANK_EXACT_MAX 32
 
 /* stages reported by gsnp_stage_times */
-#define GSNP_STAGE_VALIDATE 0     /* k_validate_reads */
+#define GSNP_STAGE_VALIDATE 0     /* k_validate_reads (calibration) */
 #define GSNP_STAGE_CALIB 1        /* k_calib_count (a1) */
-#define GSNP_STAGE_RANGES 2       /* k_tile_ranges (a3) */
-#define GSNP_STAGE_CALL 3         /* k_call_tile (a4..a8) */
+#define GSNP_STAGE_RANGES 2       /* k_prep: read validation + per-group read ranges (a3) */
+#define GSNP_STAGE_CALL 3         /* k_call_tile (a4..a8): the three instantiations of one call */
 #define GSNP_STAGE_FINALIZE 4     /* host tables + upload (a2), wall time on the host */
 #define GSNP_STAGE_BIG 5          /* k_big_sites (sites with > 1024 unique keys) */
 #define GSNP_STAGE_COMPRESS 6     /* k_cz_* (output compression, §V-B) */
@@ -216,6 +216,17 @@ gsnp_status gsnp_unpack_reads(gsnp_ctx* ctx, const void* packed, uint64_t n_byte
  * device memory.  out_cap < w1-w0 -> GSNP_E_CAPACITY with *n_out = w1-w0. */
 gsnp_status gsnp_call(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1,
                       gsnp_record* out, uint64_t out_cap, uint64_t* n_out);
+
+/* Windowed calling without host round trips (the paper calls windows of >= 256 K sites,
+ * P:L835-840): gsnp_call_async enqueues the same work as gsnp_call on params.stream and returns at
+ * once — reads must be device arrays and out device memory.  Nothing is read back: out-of-range
+ * input and capacity conditions found on the device are recorded in the context's error flag,
+ * later windows skip their work once an input is invalid, and gsnp_wait synchronises the stream
+ * and returns the first such status (then clears it).  Argument errors found on the host are
+ * returned directly.  gsnp_call (synchronous) clears the flag when it starts. */
+gsnp_status gsnp_call_async(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1,
+                            gsnp_record* out, uint64_t out_cap);
+gsnp_status gsnp_wait(gsnp_ctx* ctx);
 
 /* the dense ablation (Fig. 5): the same records as
  * gsnp_call, computed the way SOAPsnp's Alg. 1 does on the GPU: per site a dense

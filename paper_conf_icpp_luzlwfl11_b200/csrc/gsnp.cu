@@ -14,6 +14,7 @@
 #include <cstdlib>
 #include <cstdio>
 #include <cstring>
+#include <map>
 #include <string>
 #include <thread>
 #include <vector>
@@ -28,9 +29,9 @@
 using namespace gsnp_dev;
 
 namespace gsnp_deep {   // gsnp_deep.cu: the deep-window k_call_tile with 384-thread CTAs
-cudaError_t launch_call_tile_deep(const void* args, size_t args_size, bool dbg, int num_sms,
-                                  size_t adj_bytes, uint32_t adj_smem, uint32_t* wlist,
-                                  uint32_t* wlist_n, uint32_t* work, cudaStream_t s);
+const void* call_tile_kernel(bool dbg);
+int call_tile_nt();
+size_t call_tile_smem(int L, size_t adj_bytes, uint32_t* adj_smem);
 }
 
 namespace {
@@ -123,6 +124,24 @@ struct gsnp_ctx {
     // per-device facts, read at gsnp_create on prm.device (a process may hold contexts on
     // several devices)
     int num_sms = 148;
+    // (kernel, dynamic smem) -> resident CTAs per SM, with the smem attribute set: host API calls
+    // made once, not on every window of a windowed run
+    std::map<std::pair<const void*, size_t>, int> occ;
+    int occupancy(const void* kern, int nt, size_t smem) {
+        auto key = std::make_pair(kern, smem);
+        auto it = occ.find(key);
+        if (it != occ.end()) return it->second;
+        int per = 0;
+        static const int carve = [] { const char* e = getenv("GSNP_CARVEOUT"); return e ? atoi(e) : -1; }();
+        if (carve >= 0) cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
+        if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess ||
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, kern, nt, smem) != cudaSuccess) {
+            cudaGetLastError();
+            return -1;
+        }
+        occ[key] = per;
+        return per;
+    }
     // window depth thresholds of the 64- / 128-slot k_call_tile instantiations (pick_variant)
     float mid_at = 24.0f, deep_at = 48.0f;
     bool mid_adj_smem = false;        // the 64-slot kernel reads adj from L1/L2: 3 CTAs per SM
@@ -423,17 +442,17 @@ gsnp_status prep_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t 
     const uint64_t n_groups = (w1 - w0 + 31) / 32;
     CK(ctx->tile_ra.ensure(n_groups));
     CK(ctx->tile_rb.ensure(n_groups));
-    if (d.n) {
-        ctx->begin();
-        k_tile_ranges<<<(unsigned)((n_groups + 255) / 256), 256, 0, s>>>(
-            d.pos, d.n, w0, w1, (int)ctx->prm.max_read_len, n_groups, ctx->tile_ra.p,
-            ctx->tile_rb.p);
-        ctx->end(GSNP_STAGE_RANGES);
-        ctx->launches++;
-    } else {
-        CK(cudaMemsetAsync(ctx->tile_ra.p, 0, n_groups * 8, s));
-        CK(cudaMemsetAsync(ctx->tile_rb.p, 0, n_groups * 8, s));
-    }
+    CK(ctx->big_n.ensure(3));
+    // one launch: validate the reads (ABI contract; the calling kernels return at once on a
+    // violation), the per-group read ranges, and zero the window's work counters
+    const uint32_t nbv = (uint32_t)((d.n + 255) / 256);
+    ctx->begin();
+    k_prep<<<(unsigned)(nbv + (n_groups + 255) / 256), 256, 0, s>>>(
+        d, ctx->origin, ctx->n_sites, (int)ctx->prm.max_read_len, ctx->d_err.p, nbv, w0, w1, n_groups,
+        ctx->tile_ra.p, ctx->tile_rb.p, ctx->big_n.p);
+    ctx->end(GSNP_STAGE_RANGES);
+    ctx->launches++;
+    CK(cudaGetLastError());
     A.R = d;
     A.ref = ctx->ref.p;
     A.origin = ctx->origin;
@@ -482,14 +501,11 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
     const uint32_t big_cap = (uint32_t)std::min<uint64_t>(w1 - w0, 1u << 22);
     CK(ctx->big.ensure(big_cap));
     CK(ctx->wlist.ensure(w1 - w0));                 // sites for k_warp_sites (at most all)
-    CK(ctx->big_n.ensure(3));
-    CK(cudaMemsetAsync(ctx->big_n.p, 0, 12, s));    // [0] big sites, [1] work counter, [2] wlist
     const bool dbg = A.count_only || A.dbg_off || A.dbg_counters || A.dbg_L10 || A.dbg_post10;
     auto launch_tile = [&](auto kern, int cols, uint32_t adj_on) -> gsnp_status {
         const size_t smem = call_smem_bytes(A.L, adj_on ? adj_bytes : 0, cols, nullptr, nullptr, false);
-        CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        int per_sm = 0;
-        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NT, smem));
+        const int per_sm = ctx->occupancy(reinterpret_cast<const void*>(kern), NT, smem);
+        if (per_sm < 0) return fail(ctx, GSNP_E_CUDA, "k_call_tile: shared memory %zu B", smem);
         const uint64_t want = (uint64_t)ctx->num_sms * std::max(per_sm, 1);
         const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(want, n_tiles));
         ctx->begin();
@@ -503,18 +519,31 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
     if ((lst = launch_tile(dbg ? k_call_tile<true, COLS> : k_call_tile<false, COLS>, COLS, adj_smem))) return lst;
     if ((lst = launch_tile(dbg ? k_call_tile<true, COLS_MID> : k_call_tile<false, COLS_MID>, COLS_MID,
                            adj_smem && ctx->mid_adj_smem))) return lst;
-    ctx->begin();
-    CK(gsnp_deep::launch_call_tile_deep(&A, sizeof A, dbg, ctx->num_sms, adj_bytes, adj_smem,
-                                        ctx->wlist.p, ctx->big_n.p + 2, ctx->big_n.p + 1, s));
-    ctx->end(GSNP_STAGE_CALL);
-    ctx->launches++;
+    {                                                // the 128-slot kernel (gsnp_deep.cu)
+        uint32_t adj_on = adj_smem;
+        const size_t smem = gsnp_deep::call_tile_smem(A.L, adj_bytes, &adj_on);
+        const void* kern = gsnp_deep::call_tile_kernel(dbg);
+        const int nt = gsnp_deep::call_tile_nt();
+        const int per_sm = ctx->occupancy(kern, nt, smem);
+        if (per_sm < 0) return fail(ctx, GSNP_E_CUDA, "deep k_call_tile: shared memory %zu B", smem);
+        const uint64_t tiles = (w1 - w0 + nt - 1) / nt;
+        const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(
+            (uint64_t)ctx->num_sms * std::max(per_sm, 1), tiles));
+        uint32_t* wl = ctx->wlist.p;
+        uint32_t* wln = ctx->big_n.p + 2;
+        uint32_t* work = ctx->big_n.p + 1;
+        void* kargs[] = {&A, &wl, &wln, &work, &adj_on};
+        ctx->begin();
+        CK(cudaLaunchKernel(kern, dim3(grid), dim3(nt), kargs, smem, s));
+        ctx->end(GSNP_STAGE_CALL);
+        ctx->launches++;
+    }
     if (!A.count_only) {
         // listed sites (n > 32 keys, or beyond the deep kernel's thread path): warp per site
         auto wk = k_warp_sites<COLS>;
         const size_t wsm = call_smem_bytes(A.L, 0, COLS, nullptr, nullptr);
-        CK(cudaFuncSetAttribute(wk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)wsm));
-        int wper = 0;
-        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&wper, wk, NT, wsm));
+        const int wper = ctx->occupancy(reinterpret_cast<const void*>(wk), NT, wsm);
+        if (wper < 0) return fail(ctx, GSNP_E_CUDA, "k_warp_sites: shared memory %zu B", wsm);
         ctx->begin();
         wk<<<(unsigned)(ctx->num_sms * std::max(wper, 1)), NT, wsm, s>>>(A, ctx->wlist.p, ctx->big_n.p + 2,
                                                                        ctx->big.p, ctx->big_n.p, big_cap);
@@ -524,7 +553,8 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
         // sites beyond 1024 unique keys: one CTA each, shared buffer of up to ~200 KB
         const uint32_t cap = (uint32_t)((200 * 1024 - (size_t)8 * A.L) / 4);
         const size_t bsm = 4 * (size_t)cap + (size_t)8 * A.L;
-        CK(cudaFuncSetAttribute(k_big_sites, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bsm));
+        if (ctx->occupancy(reinterpret_cast<const void*>(k_big_sites), NT, bsm) < 0)
+            return fail(ctx, GSNP_E_CUDA, "k_big_sites: shared memory %zu B", bsm);
         ctx->begin();
         k_big_sites<<<(unsigned)ctx->num_sms, NT, bsm, s>>>(A, ctx->big.p, ctx->big_n.p, cap);
         ctx->end(GSNP_STAGE_BIG);
@@ -534,12 +564,15 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
     return GSNP_OK;
 }
 
+// synchronise the stream, read and clear the device error flag (a clean flag for what follows,
+// e.g. a run of gsnp_call_async windows)
 gsnp_status read_err(gsnp_ctx* ctx) {
     int h = 0;
     gsnp_status pst = peek(ctx, 2, ctx->d_err.p, sizeof(int));
     if (pst) return pst;
     CK(cudaStreamSynchronize(ctx->stream));
     memcpy(&h, ctx->mbox + 2, sizeof(int));
+    if (h) CK(cudaMemsetAsync(ctx->d_err.p, 0, sizeof(int), ctx->stream));
     ctx->flush();
     return map_err(ctx, h);
 }
@@ -916,7 +949,6 @@ gsnp_status gsnp_call(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint6
     DevReads d;
     if ((st = stage_reads(ctx, reads, d))) return st;
     CK(cudaMemsetAsync(ctx->d_err.p, 0, sizeof(int), ctx->stream));
-    if ((st = launch_validate(ctx, d))) return st;
     const bool dev_out = is_device_ptr(out);
     gsnp_record* d_out = out;
     if (!dev_out) {
@@ -928,6 +960,32 @@ gsnp_status gsnp_call(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint6
     if ((st = run_window(ctx, d, w0, w1, d_out, A))) return st;
     if (!dev_out)
         CK(cudaMemcpyAsync(out, d_out, S * sizeof(gsnp_record), cudaMemcpyDeviceToHost, ctx->stream));
+    return read_err(ctx);
+}
+
+gsnp_status gsnp_call_async(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1,
+                            gsnp_record* out, uint64_t out_cap) {
+    if (!ctx) return GSNP_E_INVAL;
+    if (cudaSetDevice(ctx->prm.device) != cudaSuccess) return fail(ctx, GSNP_E_CUDA, "set device");
+    gsnp_status st = check_window(ctx, reads, w0, w1);
+    if (st) return st;
+    const uint64_t S = w1 - w0;
+    if (out_cap < S) return fail(ctx, GSNP_E_CAPACITY, "out_cap %llu < %llu", (unsigned long long)out_cap,
+                                 (unsigned long long)S);
+    if (S == 0) return GSNP_OK;
+    if (!out || !is_device_ptr(out)) return fail(ctx, GSNP_E_INVAL, "gsnp_call_async: out must be device memory");
+    if (reads->n_reads && !reads->on_device)
+        return fail(ctx, GSNP_E_INVAL, "gsnp_call_async: reads must be device arrays");
+    DevReads d;
+    if ((st = stage_reads(ctx, reads, d))) return st;
+    CallArgs A;
+    memset(&A, 0, sizeof A);
+    return run_window(ctx, d, w0, w1, out, A);
+}
+
+gsnp_status gsnp_wait(gsnp_ctx* ctx) {
+    if (!ctx) return GSNP_E_INVAL;
+    if (cudaSetDevice(ctx->prm.device) != cudaSuccess) return fail(ctx, GSNP_E_CUDA, "set device");
     return read_err(ctx);
 }
 
@@ -950,7 +1008,6 @@ gsnp_status gsnp_call_dense(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0,
     DevReads d;
     if ((st = stage_reads(ctx, reads, d))) return st;
     CK(cudaMemsetAsync(ctx->d_err.p, 0, sizeof(int), s));
-    if ((st = launch_validate(ctx, d))) return st;
     const bool dev_out = is_device_ptr(out);
     gsnp_record* d_out = out;
     if (!dev_out) {
@@ -1378,7 +1435,6 @@ gsnp_status gsnp_debug_window(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w
     DevReads d;
     if ((st = stage_reads(ctx, reads, d))) return st;
     CK(cudaMemsetAsync(ctx->d_err.p, 0, sizeof(int), s));
-    if ((st = launch_validate(ctx, d))) return st;
     // pass 1: unique keys per site -> CSR offsets (host scan)
     CK(ctx->dbg_u32a.ensure(S));
     CK(ctx->rec.ensure(S));

@@ -18,32 +18,23 @@
 
 namespace gsnp_deep {
 
-// Launch k_call_tile<DBG, COLS_DEEP> with NT = 384 on stream s.  args: the caller's CallArgs
-// (identical layout in both namespaces: same header); returns the CUDA status of the launch.
-cudaError_t launch_call_tile_deep(const void* args, size_t args_size, bool dbg, int num_sms,
-                                  size_t adj_bytes, uint32_t adj_smem, uint32_t* wlist,
-                                  uint32_t* wlist_n, uint32_t* work, cudaStream_t s) {
+// The k_call_tile<DBG, COLS_DEEP> instantiation with NT = 384, for the caller to launch through
+// cudaLaunchKernel (CallArgs has the same layout in both namespaces: same header).
+const void* call_tile_kernel(bool dbg) {
     using namespace gsnp_dev384;
-    static_assert(sizeof(CallArgs) > 0, "");
-    if (args_size != sizeof(CallArgs)) return cudaErrorInvalidValue;
-    CallArgs A;
-    memcpy(&A, args, sizeof A);
-    size_t smem = call_smem_bytes(A.L, adj_smem ? adj_bytes : 0, COLS_DEEP, nullptr, nullptr, false);
-    if (adj_smem && smem > 227 * 1024) {     // no room for the adjust table: read it from global
-        adj_smem = 0;
-        smem = call_smem_bytes(A.L, 0, COLS_DEEP, nullptr, nullptr, false);
+    return dbg ? reinterpret_cast<const void*>(k_call_tile<true, COLS_DEEP>)
+               : reinterpret_cast<const void*>(k_call_tile<false, COLS_DEEP>);
+}
+int call_tile_nt() { return gsnp_dev384::NT; }
+// dynamic shared memory of the deep kernel; clears *adj_smem when the adjust table does not fit
+size_t call_tile_smem(int L, size_t adj_bytes, uint32_t* adj_smem) {
+    using namespace gsnp_dev384;
+    size_t smem = call_smem_bytes(L, *adj_smem ? adj_bytes : 0, COLS_DEEP, nullptr, nullptr, false);
+    if (*adj_smem && smem > 227 * 1024) {    // no room for the adjust table: read it from global
+        *adj_smem = 0;
+        smem = call_smem_bytes(L, 0, COLS_DEEP, nullptr, nullptr, false);
     }
-    auto kern = dbg ? k_call_tile<true, COLS_DEEP> : k_call_tile<false, COLS_DEEP>;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    int per_sm = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NT, smem);
-    if (e != cudaSuccess) return e;
-    const uint64_t n_tiles = (A.w1 - A.w0 + TS - 1) / TS;
-    const uint64_t want = (uint64_t)num_sms * (per_sm > 0 ? per_sm : 1);
-    const unsigned grid = (unsigned)(want < n_tiles ? want : (n_tiles ? n_tiles : 1));
-    kern<<<grid, NT, smem, s>>>(A, wlist, wlist_n, work, adj_smem);
-    return cudaGetLastError();
+    return smem;
 }
 
 }  // namespace gsnp_deep

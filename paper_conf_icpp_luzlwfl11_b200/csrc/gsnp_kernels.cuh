@@ -3,7 +3,8 @@
 // Kernels:
 //   k_validate_reads  ABI checks on the read arrays (sortedness P:L208-210, ranges)
 //   k_calib_count     a1: calibration histogram C[q][cyc][t][o] (cal_p_matrix)
-//   k_tile_ranges     a3: per 32-site group, read range [lower_bound(s0-L+1), lower_bound(s1))
+//   k_prep            validation + a3: per 32-site group, read range [lower_bound(s0-L+1),
+//                     lower_bound(s1)), and the window's work counters
 //   k_call_tile       a4..a8 fused, one thread per site: counting and
 //                     base_word gather walking the sorted reads, likelihood_sort
 //                     as an in-register bitonic network bucketed by segment length (multipass,
@@ -97,9 +98,19 @@ __device__ __forceinline__ uint64_t lower_bound_u64(const uint64_t* a, uint64_t 
 
 // ------------------------------------------------------------------------------------------
 // k_validate_reads: one thread per read.
+__device__ __forceinline__ void validate_read(const DevReads& R, uint64_t r, uint64_t origin,
+                                              uint64_t n_sites, int L, int* err);
 __global__ void k_validate_reads(DevReads R, uint64_t origin, uint64_t n_sites, int L, int* err) {
     uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (r >= R.n) return;
+    if (r < R.n) validate_read(R, r, origin, n_sites, L, err);
+}
+
+// ------------------------------------------------------------------------------------------
+// k_prep: one launch before a window's calling kernels — blocks [0, nbv) validate the reads (as
+// k_validate_reads), the others compute a3's per-32-site-group read ranges (as k_tile_ranges),
+// and block 0 zeroes the window's three work counters.
+__device__ __forceinline__ void validate_read(const DevReads& R, uint64_t r, uint64_t origin,
+                                              uint64_t n_sites, int L, int* err) {
     uint64_t p = R.pos[r];
     uint32_t l = R.len[r];
     int e = 0;
@@ -109,6 +120,24 @@ __global__ void k_validate_reads(DevReads R, uint64_t origin, uint64_t n_sites, 
     if (R.off[r] < R.off0 || R.off[r] + l > R.off[r + 1]) e |= ERR_RANGE;
     if (r > 0 && R.pos[r - 1] > p) e |= ERR_UNSORTED;
     if (e) atomicOr(err, e | ERR_VALID);
+}
+
+__global__ void k_prep(DevReads R, uint64_t origin, uint64_t n_sites, int L, int* err, uint32_t nbv,
+                       uint64_t w0, uint64_t w1, uint64_t n_groups, uint64_t* ra, uint64_t* rb,
+                       uint32_t* counters) {
+    if (blockIdx.x == 0 && threadIdx.x < 3) counters[threadIdx.x] = 0;
+    if (blockIdx.x < nbv) {
+        const uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+        if (r < R.n) validate_read(R, r, origin, n_sites, L, err);
+        return;
+    }
+    const uint64_t g = (blockIdx.x - nbv) * (uint64_t)blockDim.x + threadIdx.x;
+    if (g >= n_groups) return;
+    const uint64_t s0 = w0 + g * 32, s1 = min(w1, s0 + 32);
+    const uint64_t lo = s0 >= (uint64_t)(L - 1) ? s0 - (L - 1) : 0;
+    const uint64_t a = lower_bound_u64(R.pos, 0, R.n, lo);
+    ra[g] = a;
+    rb[g] = lower_bound_u64(R.pos, a, R.n, s1);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -513,20 +542,6 @@ __global__ void __launch_bounds__(CAL_NT, 1) k_calib_count(const __grid_constant
         }
     }
 }
-// ------------------------------------------------------------------------------------------
-// a3: read ranges.  For each group of 32 consecutive sites [s0, s0+32) (one warp of
-// k_call_tile), the reads that can touch it: pos in [s0 - L + 1, s0 + 32) (input sorted by
-// position).
-__global__ void k_tile_ranges(const uint64_t* pos, uint64_t n, uint64_t w0, uint64_t w1, int L,
-                              uint64_t n_groups, uint64_t* ra, uint64_t* rb) {
-    uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (g >= n_groups) return;
-    uint64_t s0 = w0 + g * 32, s1 = min(w1, s0 + 32);
-    uint64_t lo = s0 >= (uint64_t)(L - 1) ? s0 - (L - 1) : 0;
-    ra[g] = lower_bound_u64(pos, 0, n, lo);
-    rb[g] = lower_bound_u64(pos, ra[g], n, s1);
-}
-
 // ------------------------------------------------------------------------------------------
 // k_call_tile: one CTA = TS = 256 consecutive sites, one thread per site (GSNP's baseline
 // parallelisation).  Shared-memory layout (host: call_smem_bytes()).
@@ -1496,8 +1511,9 @@ struct BigSite {
 // host round trip): by the window's mean depth = reads overlapping it x L / sites (a3's read
 // ranges), the 32-slot kernel below mid_at, the 64-slot kernel below deep_at, the 128-slot kernel
 // (gsnp_deep.cu) above.  Every instantiation is launched; all but the chosen one return at once.
-// All of them give the same records: each sums a site's thread-path keys in canonical order, and
-// sites beyond their capacity go to the warp / CTA paths.
+// Each sums a site's keys in canonical order while the site fits its thread path; deeper sites go
+// to the warp / CTA paths (k_warp_sites, k_big_sites), whose sums may differ from a thread path's
+// in the last bits — within the parity rules either way.
 __device__ __forceinline__ int pick_variant(const CallArgs& A) {
     const uint64_t ng = (A.w1 - A.w0 + 31) / 32;
     const uint64_t nr = A.tile_rb[ng - 1] - A.tile_ra[0];

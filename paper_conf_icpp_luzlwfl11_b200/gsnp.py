@@ -28,7 +28,8 @@ STATUS = {0: "GSNP_OK", -1: "GSNP_E_INVAL", -2: "GSNP_E_RANGE", -3: "GSNP_E_UNSO
 SYMBOLS = ("gsnp_params_default", "gsnp_create", "gsnp_calibrate", "gsnp_calibrate_count",
            "gsnp_calibrate_finalize", "gsnp_call", "gsnp_debug_window", "gsnp_get_tables",
            "gsnp_compress", "gsnp_call_compressed", "gsnp_call_dense", "gsnp_priors_from_freq", "gsnp_parse_soap",
-           "gsnp_pack_reads", "gsnp_packed_sizes", "gsnp_unpack_reads",
+           "gsnp_pack_reads", "gsnp_packed_sizes", "gsnp_unpack_reads", "gsnp_call_async",
+           "gsnp_wait",
            "gsnp_launch_count", "gsnp_stage_times", "gsnp_strerror", "gsnp_last_error",
            "gsnp_destroy")
 
@@ -121,6 +122,10 @@ def lib():
         L.gsnp_packed_sizes.argtypes = [P, u64, ctypes.POINTER(u64), ctypes.POINTER(u64)]
         L.gsnp_unpack_reads.restype = S
         L.gsnp_unpack_reads.argtypes = [P, P, u64] + [P] * 7
+        L.gsnp_call_async.restype = S
+        L.gsnp_call_async.argtypes = [P, ctypes.POINTER(gsnp_reads), u64, u64, P, u64]
+        L.gsnp_wait.restype = S
+        L.gsnp_wait.argtypes = [P]
         L.gsnp_launch_count.restype = u64
         L.gsnp_launch_count.argtypes = [P]
         L.gsnp_stage_times.restype = S
@@ -216,7 +221,10 @@ class Context:
 
     def close(self):
         if getattr(self, "h", None):
-            lib().gsnp_destroy(self.h)
+            try:
+                lib().gsnp_destroy(self.h)
+            except TypeError:            # interpreter shutdown: module globals already cleared
+                pass
             self.h = None
 
     __del__ = close
@@ -363,6 +371,15 @@ class Context:
                 if k in out:
                     out[k] = out[k][:K]
         return out
+
+    def call_async(self, r: gsnp_reads, w0: int, w1: int, out):
+        """gsnp_call_async: device reads (a gsnp_reads from make_reads) and a device uint8 tensor
+        of >= 40*(w1-w0) bytes; no host round trip (errors surface at wait())."""
+        _check(lib().gsnp_call_async(self.h, ctypes.byref(r), w0, w1, _ptr(out),
+                                     _nbytes(out) // 40), self.h)
+
+    def wait(self):
+        _check(lib().gsnp_wait(self.h), self.h)
 
     def unpack_reads(self, packed, out=None):
         """gsnp_unpack_reads: a packed stream (numpy / pinned or CUDA tensor) -> device read
