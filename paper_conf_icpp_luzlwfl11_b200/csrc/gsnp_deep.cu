@@ -11,6 +11,12 @@
 #define GSNP_DEEP_NT 384
 #endif
 #define GSNP_NT GSNP_DEEP_NT
+// reads whose bytes the gather keeps in flight: a deep window has ~L reads per 32-site group
+// start, and this kernel has the registers (one CTA per SM) to hide more of their latency
+#ifndef GSNP_DEEP_GB
+#define GSNP_DEEP_GB 4
+#endif
+#define GSNP_GB GSNP_DEEP_GB
 #define GSNP_CALL_MINB 1
 #define gsnp_dev gsnp_dev384
 #include "gsnp_kernels.cuh"

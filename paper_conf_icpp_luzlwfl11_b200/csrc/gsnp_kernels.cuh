@@ -1000,6 +1000,9 @@ __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* ad
     thread_finish<DBG, true>(A, lps, rt, colp, site, n, acc, cu, qs, ca0, ca1, ca2, ca3, rep);
 }
 
+#ifndef GSNP_DEEP_U
+#define GSNP_DEEP_U 3
+#endif
 // Deep thread path (32 < n <= 32*NCH, kernels built with 128 slots per site): each 32-key chunk
 // of the column is sorted in registers, then an NCH-way streaming merge visits the keys in
 // canonical order straight into Alg. 4 (q_adj and the Alg. 3 row per key).
@@ -1029,23 +1032,51 @@ __device__ __forceinline__ void thread_site_deep(const CallArgs& A, const uint8_
     uint64_t cu = 0, qs = 0;
     uint32_t prev_b = 4, distinct = 0;
     const double* __restrict__ T = A.T;
-    for (uint32_t out = 0; out < n; ++out) {
-        uint32_t best = hk[0];
-        int bc = 0;
+    const uint32_t L = (uint32_t)A.L;
+    // U keys are merged ahead and their rows loaded together (U rows in flight per thread): the
+    // 128-slot kernel runs one 384-thread CTA per SM, so it has the registers and needs the
+    // memory-level parallelism; the adds stay in canonical order
+    constexpr int U = NCH >= 4 ? GSNP_DEEP_U : 1;
+    for (uint32_t out0 = 0; out0 < n; out0 += U) {
+        uint32_t rowv[U];
 #pragma unroll
-        for (int c = 1; c < NCH; ++c) if (hk[c] < best) { best = hk[c]; bc = c; }
+        for (int u = 0; u < U; ++u) {
+            rowv[u] = 0xFFFFFFFFu;
+            if (out0 + u < n) {
+                uint32_t best = hk[0];
+                int bc = 0;
 #pragma unroll
-        for (int c = 0; c < NCH; ++c)
-            if (c == bc) { ++hi[c]; hk[c] = hi[c] < he[c] ? colp[hi[c] * TS] : KEY_INF; }
-        const uint32_t kk = best >> 8, b = key_base(kk), q = key_q(kk);
-        if (DBG && dbg) dbg[out] = kk;
-        const uint32_t pcr = (best & 255u) + 1u;
-        if (b != prev_b) { distinct = 0; prev_b = b; }
-        distinct += pcr == 1;
-        const uint32_t qa = (uint32_t)adj_lookup_t(adj, A.adjP, A.adjG, q, pcr, distinct - 1);
-        add_row(T, A.L, qa, key_cyc(kk), b, acc);
-        cu += 1ull << (16 * b);
-        qs += (uint64_t)q << (16 * b);
+                for (int c = 1; c < NCH; ++c) if (hk[c] < best) { best = hk[c]; bc = c; }
+#pragma unroll
+                for (int c = 0; c < NCH; ++c)
+                    if (c == bc) { ++hi[c]; hk[c] = hi[c] < he[c] ? colp[hi[c] * TS] : KEY_INF; }
+                const uint32_t kk = best >> 8, b = key_base(kk), q = key_q(kk);
+                if (DBG && dbg) dbg[out0 + u] = kk;
+                const uint32_t pcr = (best & 255u) + 1u;
+                if (b != prev_b) { distinct = 0; prev_b = b; }
+                distinct += pcr == 1;
+                const uint32_t qa = (uint32_t)adj_lookup_t(adj, A.adjP, A.adjG, q, pcr, distinct - 1);
+                rowv[u] = (qa * L + key_cyc(kk)) * 4u + b;
+                cu += 1ull << (16 * b);
+                qs += (uint64_t)q << (16 * b);
+            }
+        }
+        double v[U][12];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+#pragma unroll
+            for (int k = 0; k < 12; ++k) v[u][k] = 0.0;
+            if (rowv[u] != 0xFFFFFFFFu) {
+                const double* row = T + (size_t)rowv[u] * TROW;
+                ld256(row, v[u][0], v[u][1], v[u][2], v[u][3]);
+                ld256(row + 4, v[u][4], v[u][5], v[u][6], v[u][7]);
+                ld256(row + 8, v[u][8], v[u][9], v[u][10], v[u][11]);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+            for (int k = 0; k < 10; ++k) acc[k] += v[u][k];
     }
     thread_finish<DBG, false>(A, lps, rt, colp, site, n, acc, cu, qs, ca0, ca1, ca2, ca3, rep);
 }
