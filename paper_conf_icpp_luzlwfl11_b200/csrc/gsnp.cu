@@ -57,6 +57,7 @@ struct DevBuf {  // grow-only device buffer
 };
 
 const double kLog10Zero = 0.0;
+constexpr size_t REF_PAD = 64;      // N bytes before and after the device reference
 
 }  // namespace
 
@@ -66,7 +67,8 @@ struct gsnp_ctx {
     std::string err;
     // reference + known SNPs
     uint64_t n_sites = 0, origin = 0;
-    DevBuf<uint8_t> ref;           // code | known << 3
+    DevBuf<uint8_t> ref;           // code | known << 3, with REF_PAD bytes of N on both sides
+    const uint8_t* ref_code = nullptr;   // = ref.p + REF_PAD: code of site origin
     DevBuf<uint64_t> known_pos;
     DevBuf<double> known_lp;
     uint64_t n_known = 0;
@@ -86,6 +88,7 @@ struct gsnp_ctx {
     bool calibrated = false;
     // scratch
     DevBuf<int> d_err;
+    DevBuf<uint32_t> d_flags;      // [0]: the calibration's reads are not uniform (k_calib_flat off)
     DevBuf<unsigned long long> d_counts;
     DevBuf<uint64_t> tile_ra, tile_rb;
     DevBuf<gsnp_record> rec;
@@ -423,12 +426,13 @@ gsnp_status peek(gsnp_ctx* ctx, int slot, const void* src, uint32_t n) {
     return GSNP_OK;
 }
 
-gsnp_status launch_validate(gsnp_ctx* ctx, const DevReads& d) {
+gsnp_status launch_validate(gsnp_ctx* ctx, const DevReads& d, uint32_t* uniform_flag = nullptr) {
     if (d.n == 0) return GSNP_OK;
     unsigned blocks = (unsigned)((d.n + 255) / 256);
     ctx->begin();
     k_validate_reads<<<blocks, 256, 0, ctx->stream>>>(d, ctx->origin, ctx->n_sites,
-                                                      (int)ctx->prm.max_read_len, ctx->d_err.p);
+                                                      (int)ctx->prm.max_read_len, ctx->d_err.p,
+                                                      uniform_flag);
     ctx->end(GSNP_STAGE_VALIDATE);
     ctx->launches++;
     CK(cudaGetLastError());
@@ -454,7 +458,7 @@ gsnp_status prep_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t 
     ctx->launches++;
     CK(cudaGetLastError());
     A.R = d;
-    A.ref = ctx->ref.p;
+    A.ref = ctx->ref_code;
     A.origin = ctx->origin;
     A.n_sites = ctx->n_sites;
     A.known_pos = ctx->known_pos.p;
@@ -585,11 +589,15 @@ gsnp_status count_impl(gsnp_ctx* ctx, const gsnp_reads* reads) {
     CK(ctx->d_counts.ensure(64 * 256 * 16));
     CK(cudaMemsetAsync(ctx->d_counts.p, 0, 64 * 256 * 16 * 8, s));
     CK(cudaMemsetAsync(ctx->d_err.p, 0, sizeof(int), s));
-    if ((st = launch_validate(ctx, d))) return st;
+    // the streaming kernel takes read sets of one length stored back to back (flag 0 after the
+    // validation pass); the staged kernel takes the rest — both launched, each checks the flag
+    CK(ctx->d_flags.ensure(1));
+    CK(cudaMemsetAsync(ctx->d_flags.p, 0, sizeof(uint32_t), s));
+    if ((st = launch_validate(ctx, d, ctx->d_flags.p))) return st;
     if (d.n) {
         CalibArgs A;
         A.R = d;
-        A.ref = ctx->ref.p;
+        A.ref = ctx->ref_code;
         A.origin = ctx->origin;
         A.n_sites = ctx->n_sites;
         A.L = (int)ctx->prm.max_read_len;
@@ -617,11 +625,23 @@ gsnp_status count_impl(gsnp_ctx* ctx, const gsnp_reads* reads) {
         A.Lh = std::min<int>(A.L, (int)((budget - 2 * (2 * 4096 + A.RB) - 16) / per_cyc) & ~3);
         const size_t hist = align16(per_cyc * ((A.Lh + 3) / 4 * 4));
         while (A.SB > 4096 && hist + 2 * (2 * (size_t)A.SB + A.RB) + 16 > budget) A.SB -= 4096;
-        A.CB = std::max(1, std::min<int>(CAL_MAXB, (int)(A.SB - 32) / A.L));
+        A.CB = std::max(1, std::min<int>(std::min(CAL_MAXB, CAL_NT), (int)(A.SB - 32) / A.L));
         const size_t smem = hist + 2 * (2 * (size_t)A.SB + A.RB) + 16;
         unsigned grid = (unsigned)std::min<uint64_t>((uint64_t)ctx->num_sms, (d.n + A.CB - 1) / A.CB);
         grid = std::max(grid, 1u);
         CK(cudaFuncSetAttribute(k_calib_count, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        A.flat_flag = ctx->d_flags.p;
+        {
+            const int ncell = (A.q_max + 1) * 4 * A.Lh;
+            const size_t fsm = align16((size_t)ncell * 4);
+            const int per = ctx->occupancy(reinterpret_cast<const void*>(k_calib_flat), CF_NT, fsm);
+            if (per < 0) return fail(ctx, GSNP_E_CUDA, "k_calib_flat: shared memory %zu B", fsm);
+            ctx->begin();
+            k_calib_flat<<<(unsigned)(ctx->num_sms * std::max(per, 1)), CF_NT, fsm, s>>>(A, ctx->d_flags.p);
+            ctx->end(GSNP_STAGE_CALIB);
+            ctx->launches++;
+            CK(cudaGetLastError());
+        }
         ctx->begin();
         k_calib_count<<<grid, CAL_NT, smem, s>>>(A);
         ctx->end(GSNP_STAGE_CALIB);
@@ -866,9 +886,12 @@ gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
     if ((st = build_adj(ctx))) return bail(st);
     gsnp_ctx* c = ctx;
 #define CKC(x) do { if ((x) != cudaSuccess) { cudaGetLastError(); return bail(fail(c, GSNP_E_CUDA, "%s", #x)); } } while (0)
-    CKC(ctx->ref.ensure(ref->n_sites + 64));       // padded: 16-byte TMA windows may overrun
-    CKC(cudaMemset(ctx->ref.p + ref->n_sites, 4, 64));
-    CKC(cudaMemcpy(ctx->ref.p, code.data(), ref->n_sites, cudaMemcpyHostToDevice));
+    // padded with N on both sides: 16-byte TMA windows and k_calib_flat's 32-bit reference loads
+    // may reach up to REF_PAD bytes past either end
+    CKC(ctx->ref.ensure(ref->n_sites + 2 * REF_PAD));
+    CKC(cudaMemset(ctx->ref.p, 4, ref->n_sites + 2 * REF_PAD));
+    CKC(cudaMemcpy(ctx->ref.p + REF_PAD, code.data(), ref->n_sites, cudaMemcpyHostToDevice));
+    ctx->ref_code = ctx->ref.p + REF_PAD;
     CKC(ctx->known_pos.ensure(std::max<uint64_t>(nk, 1)));
     if (nk) CKC(cudaMemcpy(ctx->known_pos.p, ctx->h_known_pos.data(), nk * 8, cudaMemcpyHostToDevice));
     CKC(ctx->known_lp.ensure(lp.size()));
@@ -1531,7 +1554,7 @@ void gsnp_destroy(gsnp_ctx* ctx) {
     if (!ctx) return;
     cudaSetDevice(ctx->prm.device);
     ctx->ref.release(); ctx->known_pos.release(); ctx->known_lp.release();
-    ctx->adj.release(); ctx->LP.release(); ctx->rank_cdf.release(); ctx->T.release(); ctx->d_err.release();
+    ctx->adj.release(); ctx->LP.release(); ctx->rank_cdf.release(); ctx->T.release(); ctx->d_err.release(); ctx->d_flags.release();
     ctx->d_counts.release(); ctx->tile_ra.release(); ctx->tile_rb.release(); ctx->rec.release();
     ctx->big.release(); ctx->big_n.release(); ctx->wlist.release();
     ctx->dense_occ.release(); ctx->dense_cnt.release();
