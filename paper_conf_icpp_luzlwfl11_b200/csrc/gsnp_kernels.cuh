@@ -604,6 +604,7 @@ __global__ void __launch_bounds__(CF_NT, 1) k_calib_flat(const __grid_constant__
     __syncthreads();
     const uint32_t hbase = smem_u32(hist);
     const uint32_t L = A.R.len[0];
+    const bool full = Lh >= L;
     // floor(x / L) = umul64hi(x, ceil(2^64 / L)) exactly for x < 2^40 (the error x (ceil - 2^64/L)
     // / 2^64 < 2^-16 stays below the 1/L gap to the next integer)
     const uint64_t magic = 0xFFFFFFFFFFFFFFFFull / L + 1;
@@ -658,17 +659,14 @@ __global__ void __launch_bounds__(CF_NT, 1) k_calib_flat(const __grid_constant__
             const uint64_t rb = p - A.origin + ipk0 - k0;               // ref index of chunk byte 0
             uint32_t rw4[4];
             ref16(A.ref, rb, rw4);
-            const uint32_t kmask_lo = k0 >= 16 ? 0u : (0xFFFFu << k0) & 0xFFFFu;
-            const uint32_t kmask = kmask_lo & (k1 >= 16 ? 0xFFFFu : ((1u << k1) - 1u));
+            const uint32_t kmask = ((0xFFFFu << k0) & 0xFFFFu) & (k1 >= 16 ? 0xFFFFu : ((1u << k1) - 1u));
             // cycle of chunk byte k: + strand ip, - strand L-1-ip, ip = ipk0 + k - k0
             const int cbase = minus ? (int)(L - 1 - ipk0 + k0) : (int)ipk0 - (int)k0;
             const int dir = minus ? -1 : 1;
 #pragma unroll
             for (int wd = 0; wd < 4; ++wd) {
-                const uint32_t bm = (kmask >> (4 * wd)) & 15u;          // valid bytes of this word
-                if (!bm) continue;
-                const uint32_t vm = (bm & 1 ? 0x80u : 0u) | (bm & 2 ? 0x8000u : 0u) |
-                                    (bm & 4 ? 0x800000u : 0u) | (bm & 8 ? 0x80000000u : 0u);
+                // valid bytes of this word as bit 7 of each byte (4 mask bits spread by a multiply)
+                const uint32_t vm = ((((kmask >> (4 * wd)) & 15u) * 0x00204081u) & 0x01010101u) * 0x80u;
                 const uint32_t bw = bw4[wd], qw = qw4[wd], rw = rw4[wd];
                 const uint32_t badb = (((bw | H) - 0x05050505u) | bw) & H & vm;
                 const uint32_t badq = (((qw | H) - qlim) | qw) & H & vm;
@@ -676,23 +674,36 @@ __global__ void __launch_bounds__(CF_NT, 1) k_calib_flat(const __grid_constant__
                 eqw |= badq;
                 const uint32_t xd = (rw ^ bw) | (rw & 0xFCFCFCFCu);      // 0 <=> diagonal, t < 4
                 const uint32_t xu = (rw | bw) & 0xFCFCFCFCu;             // 0 <=> t < 4 and o < 4
-                const uint32_t diag = ~(((xd & M) + M) | xd) & H & ~badq & vm;
-                const uint32_t used = ~(((xu & M) + M) | xu) & H & ~badq & vm;
+                const uint32_t ok = vm & ~badq;
+                const uint32_t diag = ~(((xd & M) + M) | xd) & H & ok;
+                const uint32_t used = ~(((xu & M) + M) | xu) & H & ok;
                 const uint32_t qt = ((qw & 0x3F3F3F3Fu) << 2) | (rw & 0x03030303u);
                 const int cw = cbase + dir * 4 * wd;                     // cycle of byte 0 of word
+                if (full) {                                              // every cycle in shared
+                    const uint32_t a0 = hbase + 4u * (uint32_t)cw, ad = 4u * (uint32_t)dir, qs = 4u * Lh;
 #pragma unroll
-                for (int u = 0; u < 4; ++u) {
-                    const uint32_t cyc = (uint32_t)(cw + u * dir);
-                    const uint32_t hit = (diag & (0x80u << (8 * u))) && cyc < Lh;
-                    red_shared_inc_if(hbase + 4u * (((qt >> (8 * u)) & 255u) * Lh + cyc), hit);
+                    for (int u = 0; u < 4; ++u)
+                        red_shared_inc_if(a0 + ad * u + qs * ((qt >> (8 * u)) & 255u), diag & (0x80u << (8 * u)));
+                } else {
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                        const uint32_t cyc = (uint32_t)(cw + u * dir);
+                        if ((diag & (0x80u << (8 * u))) && cyc < Lh)
+                            red_shared_add(&hist[((qt >> (8 * u)) & 255u) * Lh + cyc], 1u);
+                    }
                 }
-                if (!(used & ~diag) && Lh >= L) continue;                // ~2% of words go on
-#pragma unroll 1
-                for (int u = 0; u < 4; ++u) {
-                    const uint32_t mis = used & ~diag;
+                // the rest to global REDs: mismatches (~2% of bases) and, when the shared histogram
+                // stops at Lh < L, the diagonal cells of later cycles
+                uint32_t rest = used & ~diag;
+                if (!full) {
+#pragma unroll
+                    for (int u = 0; u < 4; ++u)
+                        if ((uint32_t)(cw + u * dir) >= Lh) rest |= diag & (0x80u << (8 * u));
+                }
+                while (rest) {
+                    const int u = (__ffs(rest) - 1) >> 3;
+                    rest &= rest - 1;
                     const uint32_t cyc = (uint32_t)(cw + u * dir);
-                    const bool d = (diag & (0x80u << (8 * u))) != 0;
-                    if (!(mis & (0x80u << (8 * u))) && !(d && cyc >= Lh)) continue;
                     atomicAdd(&A.C[((qw >> (8 * u)) & 63u) << 12 | cyc << 4 |
                                    ((rw >> (8 * u)) & 3u) << 2 | ((bw >> (8 * u)) & 3u)], 1ull);
                 }
