@@ -9,6 +9,9 @@
 #include <algorithm>
 #include <atomic>
 #include <chrono>
+#include <condition_variable>
+#include <functional>
+#include <mutex>
 #include <cmath>
 #include <cstdarg>
 #include <cstdlib>
@@ -61,7 +64,62 @@ constexpr size_t REF_PAD = 64;      // N bytes before and after the device refer
 
 }  // namespace
 
+namespace {
+// Persistent host worker threads of a context (the table build of every calibration runs on
+// them; creating threads per call would cost more than the work).  run(f) executes f on every
+// worker and on the caller, and returns when all are done.
+struct HostPool {
+    std::vector<std::thread> th;
+    std::mutex m;
+    std::condition_variable cv, done_cv;
+    std::function<void()> job;
+    uint64_t gen = 0;
+    int busy = 0;
+    bool stop = false;
+    void start(int n) {
+        for (int i = 0; i < n; ++i)
+            th.emplace_back([this] {
+                uint64_t seen = 0;
+                for (;;) {
+                    std::function<void()> j;
+                    {
+                        std::unique_lock<std::mutex> l(m);
+                        cv.wait(l, [&] { return stop || gen != seen; });
+                        if (stop) return;
+                        seen = gen;
+                        j = job;
+                    }
+                    j();
+                    std::lock_guard<std::mutex> l(m);
+                    if (--busy == 0) done_cv.notify_all();
+                }
+            });
+    }
+    void run(const std::function<void()>& f) {
+        {
+            std::lock_guard<std::mutex> l(m);
+            job = f;
+            busy = (int)th.size();
+            ++gen;
+        }
+        cv.notify_all();
+        f();
+        std::unique_lock<std::mutex> l(m);
+        done_cv.wait(l, [&] { return busy == 0; });
+    }
+    ~HostPool() {
+        {
+            std::lock_guard<std::mutex> l(m);
+            stop = true;
+        }
+        cv.notify_all();
+        for (auto& t : th) t.join();
+    }
+};
+}  // namespace
+
 struct gsnp_ctx {
+    HostPool pool;                 // started at gsnp_create
     gsnp_params prm{};
     cudaStream_t stream = nullptr;
     std::string err;
@@ -85,10 +143,10 @@ struct gsnp_ctx {
     size_t h_T_n = 0;
     uint64_t* h_cnt_pinned = nullptr;   // staging for device-resident counts
     DevBuf<double> T;
+    bool T_zeroed = false;
     bool calibrated = false;
     // scratch
     DevBuf<int> d_err;
-    DevBuf<uint32_t> d_flags;      // [0]: the calibration's reads are not uniform (k_calib_flat off)
     DevBuf<unsigned long long> d_counts;
     DevBuf<uint64_t> tile_ra, tile_rb;
     DevBuf<gsnp_record> rec;
@@ -426,13 +484,12 @@ gsnp_status peek(gsnp_ctx* ctx, int slot, const void* src, uint32_t n) {
     return GSNP_OK;
 }
 
-gsnp_status launch_validate(gsnp_ctx* ctx, const DevReads& d, uint32_t* uniform_flag = nullptr) {
+gsnp_status launch_validate(gsnp_ctx* ctx, const DevReads& d) {
     if (d.n == 0) return GSNP_OK;
     unsigned blocks = (unsigned)((d.n + 255) / 256);
     ctx->begin();
     k_validate_reads<<<blocks, 256, 0, ctx->stream>>>(d, ctx->origin, ctx->n_sites,
-                                                      (int)ctx->prm.max_read_len, ctx->d_err.p,
-                                                      uniform_flag);
+                                                      (int)ctx->prm.max_read_len, ctx->d_err.p);
     ctx->end(GSNP_STAGE_VALIDATE);
     ctx->launches++;
     CK(cudaGetLastError());
@@ -589,11 +646,7 @@ gsnp_status count_impl(gsnp_ctx* ctx, const gsnp_reads* reads) {
     CK(ctx->d_counts.ensure(64 * 256 * 16));
     CK(cudaMemsetAsync(ctx->d_counts.p, 0, 64 * 256 * 16 * 8, s));
     CK(cudaMemsetAsync(ctx->d_err.p, 0, sizeof(int), s));
-    // the streaming kernel takes read sets of one length stored back to back (flag 0 after the
-    // validation pass); the staged kernel takes the rest — both launched, each checks the flag
-    CK(ctx->d_flags.ensure(1));
-    CK(cudaMemsetAsync(ctx->d_flags.p, 0, sizeof(uint32_t), s));
-    if ((st = launch_validate(ctx, d, ctx->d_flags.p))) return st;
+    if ((st = launch_validate(ctx, d))) return st;
     if (d.n) {
         CalibArgs A;
         A.R = d;
@@ -630,18 +683,6 @@ gsnp_status count_impl(gsnp_ctx* ctx, const gsnp_reads* reads) {
         unsigned grid = (unsigned)std::min<uint64_t>((uint64_t)ctx->num_sms, (d.n + A.CB - 1) / A.CB);
         grid = std::max(grid, 1u);
         CK(cudaFuncSetAttribute(k_calib_count, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        A.flat_flag = ctx->d_flags.p;
-        {
-            const int ncell = (A.q_max + 1) * 4 * A.Lh;
-            const size_t fsm = align16((size_t)ncell * 4);
-            const int per = ctx->occupancy(reinterpret_cast<const void*>(k_calib_flat), CF_NT, fsm);
-            if (per < 0) return fail(ctx, GSNP_E_CUDA, "k_calib_flat: shared memory %zu B", fsm);
-            ctx->begin();
-            k_calib_flat<<<(unsigned)(ctx->num_sms * std::max(per, 1)), CF_NT, fsm, s>>>(A, ctx->d_flags.p);
-            ctx->end(GSNP_STAGE_CALIB);
-            ctx->launches++;
-            CK(cudaGetLastError());
-        }
         ctx->begin();
         k_calib_count<<<grid, CAL_NT, smem, s>>>(A);
         ctx->end(GSNP_STAGE_CALIB);
@@ -656,7 +697,7 @@ gsnp_status finalize_impl(gsnp_ctx* ctx, const uint64_t* counts_host) {
     const int L = (int)ctx->prm.max_read_len;
     const int qmax = (int)ctx->prm.q_max;
     ctx->h_counts.assign(counts_host, counts_host + 64 * 256 * 16);
-    ctx->h_p.assign((size_t)64 * 256 * 16, 0.0);
+    if (ctx->h_p.size() != (size_t)64 * 256 * 16) ctx->h_p.assign((size_t)64 * 256 * 16, 0.0);
     const size_t tn = (size_t)64 * L * 4 * TROW;
     if (!ctx->h_T || ctx->h_T_n != tn) {
         if (ctx->h_T) cudaFreeHost(ctx->h_T);
@@ -690,12 +731,15 @@ gsnp_status finalize_impl(gsnp_ctx* ctx, const uint64_t* counts_host) {
     static const int nt_env = [] { const char* e = getenv("GSNP_HOST_THREADS"); return e ? atoi(e) : 0; }();
     const int nt = nt_env > 0 ? nt_env
                               : (int)std::max(1u, std::min(32u, std::thread::hardware_concurrency()));
-    std::vector<std::thread> th;
-    for (int i = 1; i < nt; ++i) th.emplace_back(work);
-    work();
-    for (auto& t : th) t.join();
+    if (ctx->pool.th.empty() && nt > 1) ctx->pool.start(nt - 1);
+    ctx->pool.run(work);
     CK(ctx->T.ensure(tn));
-    CK(cudaMemcpyAsync(ctx->T.p, ctx->h_T, tn * 8, cudaMemcpyHostToDevice, ctx->stream));
+    if (!ctx->T_zeroed) {                                  // rows of q > q_max stay zero
+        CK(cudaMemsetAsync(ctx->T.p, 0, tn * 8, ctx->stream));
+        ctx->T_zeroed = true;
+    }
+    const size_t tq = (size_t)(qmax + 1) * L * 4 * TROW;  // rows q = 0..q_max (the built ones)
+    CK(cudaMemcpyAsync(ctx->T.p, ctx->h_T, tq * 8, cudaMemcpyHostToDevice, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
     ctx->calibrated = true;
     if (ctx->timing()) {
@@ -886,8 +930,7 @@ gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
     if ((st = build_adj(ctx))) return bail(st);
     gsnp_ctx* c = ctx;
 #define CKC(x) do { if ((x) != cudaSuccess) { cudaGetLastError(); return bail(fail(c, GSNP_E_CUDA, "%s", #x)); } } while (0)
-    // padded with N on both sides: 16-byte TMA windows and k_calib_flat's 32-bit reference loads
-    // may reach up to REF_PAD bytes past either end
+    // padded with N on both sides: 16-byte TMA reference windows may reach past either end
     CKC(ctx->ref.ensure(ref->n_sites + 2 * REF_PAD));
     CKC(cudaMemset(ctx->ref.p, 4, ref->n_sites + 2 * REF_PAD));
     CKC(cudaMemcpy(ctx->ref.p + REF_PAD, code.data(), ref->n_sites, cudaMemcpyHostToDevice));
@@ -1554,7 +1597,7 @@ void gsnp_destroy(gsnp_ctx* ctx) {
     if (!ctx) return;
     cudaSetDevice(ctx->prm.device);
     ctx->ref.release(); ctx->known_pos.release(); ctx->known_lp.release();
-    ctx->adj.release(); ctx->LP.release(); ctx->rank_cdf.release(); ctx->T.release(); ctx->d_err.release(); ctx->d_flags.release();
+    ctx->adj.release(); ctx->LP.release(); ctx->rank_cdf.release(); ctx->T.release(); ctx->d_err.release();
     ctx->d_counts.release(); ctx->tile_ra.release(); ctx->tile_rb.release(); ctx->rec.release();
     ctx->big.release(); ctx->big_n.release(); ctx->wlist.release();
     ctx->dense_occ.release(); ctx->dense_cnt.release();

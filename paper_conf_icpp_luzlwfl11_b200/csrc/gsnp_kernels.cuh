@@ -100,14 +100,9 @@ __device__ __forceinline__ uint64_t lower_bound_u64(const uint64_t* a, uint64_t 
 // k_validate_reads: one thread per read.
 __device__ __forceinline__ void validate_read(const DevReads& R, uint64_t r, uint64_t origin,
                                               uint64_t n_sites, int L, int* err);
-__device__ __forceinline__ void check_uniform(const DevReads& R, uint64_t r, uint32_t* flag);
-__global__ void k_validate_reads(DevReads R, uint64_t origin, uint64_t n_sites, int L, int* err,
-                                 uint32_t* uniform_flag) {
+__global__ void k_validate_reads(DevReads R, uint64_t origin, uint64_t n_sites, int L, int* err) {
     uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (r < R.n) {
-        validate_read(R, r, origin, n_sites, L, err);
-        if (uniform_flag) check_uniform(R, r, uniform_flag);
-    }
+    if (r < R.n) validate_read(R, r, origin, n_sites, L, err);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -243,8 +238,6 @@ struct CalibArgs {
     unsigned long long* C;            // [64][256][4][4]
     int* err;
     int tma_ok;                       // bases and quals 16-byte aligned (TMA bulk copies allowed)
-    const uint32_t* flat_flag;        // k_validate_reads' uniformity flag when k_calib_flat was
-                                      // launched too (0 there = k_calib_flat counts), else null
 };
 
 #ifndef GSNP_CAL_NT
@@ -278,7 +271,7 @@ __global__ void __launch_bounds__(CAL_NT, 1) k_calib_count(const __grid_constant
     __shared__ uint32_t m_flat[2][CAL_MAXB];
     __shared__ uint32_t m_fl[2][5];                   // uniform flag, reads in batch, length Lb,
                                                       // ceil(2^32 / Lb), stage byte offset
-    if (reads_invalid(A.err) || (A.flat_flag && *A.flat_flag == 0)) return;
+    if (reads_invalid(A.err)) return;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int L = A.L, Lh = A.Lh;
     const uint32_t qmax = (uint32_t)A.q_max;
@@ -556,172 +549,6 @@ __global__ void __launch_bounds__(CAL_NT, 1) k_calib_count(const __grid_constant
         }
     }
 }
-// ------------------------------------------------------------------------------------------
-// a1, streaming form for read sets of one length L >= 16 stored back to back (off[r] = off[0] +
-// r L — what sequencers emit and what k_validate_reads' uniformity check, below, confirms on the
-// device).  No batches, no barriers in the loop: each lane takes one 16-byte chunk of the base and
-// quality arrays (two 128-bit loads), finds its read by a multiply-high (a chunk meets at most two
-// reads since L >= 16), takes the 16 reference codes under it through 32-bit loads and funnel
-// shifts, tests the 16 bases four at a time in registers (SIMD within a word) and adds the
-// diagonal cells to the CTA's shared [q][t][cycle] histogram with predicated shared reductions;
-// mismatches (~2%) go to global u64 REDs.  k_calib_count (staged through TMA) handles every other
-// read set; the two kernels pick themselves on the device from the uniformity flag.
-constexpr int CF_NT = 1024;
-
-// flag word written by k_validate_reads: bit 0 = the reads are NOT of one length L0 >= 16 stored
-// back to back (then k_calib_count counts them)
-__device__ __forceinline__ void check_uniform(const DevReads& R, uint64_t r, uint32_t* flag) {
-    const uint32_t L0 = R.len[0];
-    const uint32_t l = R.len[r];
-    bool bad = l != L0 || L0 < 16 || R.off[r] - R.off[0] != r * (uint64_t)L0;
-    if (r == 0) {                             // 128-bit loads need both arrays 16-byte aligned
-        const uint64_t o0 = R.off[0] - R.off0;
-        bad |= ((reinterpret_cast<uintptr_t>(R.bases + o0) | reinterpret_cast<uintptr_t>(R.quals + o0)) & 15) != 0;
-    }
-    if (bad) atomicOr(flag, 1u);
-}
-
-// 16 reference bytes starting at ref[i] (ref padded by >= 20 bytes past its end)
-__device__ __forceinline__ void ref16(const uint8_t* ref, uint64_t i, uint32_t (&w)[4]) {
-    const uint32_t* p = reinterpret_cast<const uint32_t*>(ref + (i & ~3ull));
-    const uint32_t sh = (uint32_t)(i & 3) * 8;
-    const uint32_t a0 = __ldg(p), a1 = __ldg(p + 1), a2 = __ldg(p + 2), a3 = __ldg(p + 3), a4 = __ldg(p + 4);
-    w[0] = __funnelshift_r(a0, a1, sh);
-    w[1] = __funnelshift_r(a1, a2, sh);
-    w[2] = __funnelshift_r(a2, a3, sh);
-    w[3] = __funnelshift_r(a3, a4, sh);
-}
-
-__global__ void __launch_bounds__(CF_NT, 1) k_calib_flat(const __grid_constant__ CalibArgs A,
-                                                         const uint32_t* nonuniform) {
-    extern __shared__ __align__(16) unsigned char smem[];
-    if (reads_invalid(A.err) || *nonuniform) return;
-    const int tid = threadIdx.x, lane = tid & 31;
-    const uint32_t Lh = (uint32_t)A.Lh, qmax = (uint32_t)A.q_max;
-    const int ncell = (A.q_max + 1) * 4 * A.Lh;
-    uint32_t* hist = reinterpret_cast<uint32_t*>(smem);              // [q*4 + t][cycle]
-    for (int i = tid; i < ncell; i += CF_NT) hist[i] = 0;
-    __syncthreads();
-    const uint32_t hbase = smem_u32(hist);
-    const uint32_t L = A.R.len[0];
-    const bool full = Lh >= L;
-    // floor(x / L) = umul64hi(x, ceil(2^64 / L)) exactly for x < 2^40 (the error x (ceil - 2^64/L)
-    // / 2^64 < 2^-16 stays below the 1/L gap to the next integer)
-    const uint64_t magic = 0xFFFFFFFFFFFFFFFFull / L + 1;
-    const uint64_t o0 = A.R.off[0] - A.R.off0;                          // byte of read 0, base 0
-    const uint64_t nb = (uint64_t)A.R.n * L;
-    const uint8_t* gb = A.R.bases + o0;                                 // 16-byte aligned (host)
-    const uint8_t* gq = A.R.quals + o0;
-    const uint64_t nchunk = (nb + 15) / 16;
-    const uint32_t qlim = (qmax + 1) * 0x01010101u;
-    const uint32_t H = 0x80808080u, M = 0x7F7F7F7Fu;
-    uint32_t ebw = 0, eqw = 0;
-    const uint64_t nwarp = (uint64_t)gridDim.x * (CF_NT / 32);
-    // warp-tiles of 32 consecutive chunks (512 bases, ~5 reads: metadata and reference in L1)
-    for (uint64_t tile = blockIdx.x * (uint64_t)(CF_NT / 32) + (tid >> 5); tile * 32 < nchunk; tile += nwarp) {
-        const uint64_t c = tile * 32 + lane;
-        if (c >= nchunk) continue;
-        const uint64_t x = c * 16;
-        // the chunk's reads: j0 = x / L (exact: split x = L * hi + lo with hi a multiple of 65536)
-        const uint64_t jj = __umul64hi(x, magic);
-        const uint32_t i0 = (uint32_t)(x - jj * L);
-        uint32_t bw4[4], qw4[4];
-        if (x + 16 <= nb) {
-            const uint4 bv = *reinterpret_cast<const uint4*>(gb + x);
-            const uint4 qv = *reinterpret_cast<const uint4*>(gq + x);
-            bw4[0] = bv.x; bw4[1] = bv.y; bw4[2] = bv.z; bw4[3] = bv.w;
-            qw4[0] = qv.x; qw4[1] = qv.y; qw4[2] = qv.z; qw4[3] = qv.w;
-        } else {                                                        // last chunk: bytewise
-#pragma unroll
-            for (int wd = 0; wd < 4; ++wd) {
-                uint32_t b = 0, q = 0;
-                for (int u = 0; u < 4; ++u) {
-                    const uint64_t g = x + 4 * wd + u;
-                    if (g < nb) { b |= (uint32_t)gb[g] << (8 * u); q |= (uint32_t)gq[g] << (8 * u); }
-                }
-                bw4[wd] = b;
-                qw4[wd] = q;
-            }
-        }
-        // up to two reads: part 0 = read jj from position i0, part 1 = read jj + 1 from 0
-        const uint32_t n0 = min(L - i0, 16u);                           // bytes of part 0
-#pragma unroll 1
-        for (int part = 0; part < 2; ++part) {
-            const uint64_t r = jj + part;
-            const uint32_t k0 = part ? n0 : 0u, k1 = part ? 16u : n0;      // chunk bytes [k0, k1)
-            if (k0 >= k1 || r >= A.R.n) break;
-            if (A.R.hits[r] != 1) continue;                           // multi-hit: not counted
-            const uint64_t p = A.R.pos[r];
-            if (p < A.origin || p + L > A.origin + A.n_sites) continue;   // (validated already)
-            const bool minus = A.R.strand[r] != 0;
-            // chunk byte k is read position ip = k - k0 + (part ? 0 : i0)
-            const uint32_t ipk0 = part ? 0u : i0;                       // position of byte k0
-            const uint64_t rb = p - A.origin + ipk0 - k0;               // ref index of chunk byte 0
-            uint32_t rw4[4];
-            ref16(A.ref, rb, rw4);
-            const uint32_t kmask = ((0xFFFFu << k0) & 0xFFFFu) & (k1 >= 16 ? 0xFFFFu : ((1u << k1) - 1u));
-            // cycle of chunk byte k: + strand ip, - strand L-1-ip, ip = ipk0 + k - k0
-            const int cbase = minus ? (int)(L - 1 - ipk0 + k0) : (int)ipk0 - (int)k0;
-            const int dir = minus ? -1 : 1;
-#pragma unroll
-            for (int wd = 0; wd < 4; ++wd) {
-                // valid bytes of this word as bit 7 of each byte (4 mask bits spread by a multiply)
-                const uint32_t vm = ((((kmask >> (4 * wd)) & 15u) * 0x00204081u) & 0x01010101u) * 0x80u;
-                const uint32_t bw = bw4[wd], qw = qw4[wd], rw = rw4[wd];
-                const uint32_t badb = (((bw | H) - 0x05050505u) | bw) & H & vm;
-                const uint32_t badq = (((qw | H) - qlim) | qw) & H & vm;
-                ebw |= badb;
-                eqw |= badq;
-                const uint32_t xd = (rw ^ bw) | (rw & 0xFCFCFCFCu);      // 0 <=> diagonal, t < 4
-                const uint32_t xu = (rw | bw) & 0xFCFCFCFCu;             // 0 <=> t < 4 and o < 4
-                const uint32_t ok = vm & ~badq;
-                const uint32_t diag = ~(((xd & M) + M) | xd) & H & ok;
-                const uint32_t used = ~(((xu & M) + M) | xu) & H & ok;
-                const uint32_t qt = ((qw & 0x3F3F3F3Fu) << 2) | (rw & 0x03030303u);
-                const int cw = cbase + dir * 4 * wd;                     // cycle of byte 0 of word
-                if (full) {                                              // every cycle in shared
-                    const uint32_t a0 = hbase + 4u * (uint32_t)cw, ad = 4u * (uint32_t)dir, qs = 4u * Lh;
-#pragma unroll
-                    for (int u = 0; u < 4; ++u)
-                        red_shared_inc_if(a0 + ad * u + qs * ((qt >> (8 * u)) & 255u), diag & (0x80u << (8 * u)));
-                } else {
-#pragma unroll
-                    for (int u = 0; u < 4; ++u) {
-                        const uint32_t cyc = (uint32_t)(cw + u * dir);
-                        if ((diag & (0x80u << (8 * u))) && cyc < Lh)
-                            red_shared_add(&hist[((qt >> (8 * u)) & 255u) * Lh + cyc], 1u);
-                    }
-                }
-                // the rest to global REDs: mismatches (~2% of bases) and, when the shared histogram
-                // stops at Lh < L, the diagonal cells of later cycles
-                uint32_t rest = used & ~diag;
-                if (!full) {
-#pragma unroll
-                    for (int u = 0; u < 4; ++u)
-                        if ((uint32_t)(cw + u * dir) >= Lh) rest |= diag & (0x80u << (8 * u));
-                }
-                while (rest) {
-                    const int u = (__ffs(rest) - 1) >> 3;
-                    rest &= rest - 1;
-                    const uint32_t cyc = (uint32_t)(cw + u * dir);
-                    atomicAdd(&A.C[((qw >> (8 * u)) & 63u) << 12 | cyc << 4 |
-                                   ((rw >> (8 * u)) & 3u) << 2 | ((bw >> (8 * u)) & 3u)], 1ull);
-                }
-            }
-        }
-    }
-    const int err = (ebw ? ERR_RANGE : 0) | (eqw ? ERR_QUAL : 0);
-    if (err) atomicOr(A.err, err);
-    __syncthreads();
-    for (int i = tid; i < ncell; i += CF_NT) {
-        const uint32_t v = hist[i];
-        if (v) {
-            const uint32_t qt = (uint32_t)(i / (int)Lh), cc = (uint32_t)(i % (int)Lh), q = qt >> 2, t = qt & 3;
-            atomicAdd(&A.C[q << 12 | cc << 4 | t << 2 | t], (unsigned long long)v);
-        }
-    }
-}
-
 // ------------------------------------------------------------------------------------------
 // k_call_tile: one CTA = TS = 256 consecutive sites, one thread per site (GSNP's baseline
 // parallelisation).  Shared-memory layout (host: call_smem_bytes()).
