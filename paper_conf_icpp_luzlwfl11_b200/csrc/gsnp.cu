@@ -496,7 +496,7 @@ gsnp_status launch_validate(gsnp_ctx* ctx, const DevReads& d) {
     return GSNP_OK;
 }
 
-// a3: per-32-site-group read ranges of [w0, w1) (k_tile_ranges) and the kernels' arguments
+// a3: per-32-site-group read ranges of [w0, w1) (k_prep, with read validation) and the kernels' arguments
 gsnp_status prep_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w1,
                         gsnp_record* d_out, CallArgs& A) {
     cudaStream_t s = ctx->stream;
