@@ -1024,9 +1024,12 @@ gsnp_status gsnp_call(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint6
     CallArgs A;
     memset(&A, 0, sizeof A);
     if ((st = run_window(ctx, d, w0, w1, d_out, A))) return st;
-    if (!dev_out)
+    if ((st = read_err(ctx))) return st;           // on an error the records were not written
+    if (!dev_out) {
         CK(cudaMemcpyAsync(out, d_out, S * sizeof(gsnp_record), cudaMemcpyDeviceToHost, ctx->stream));
-    return read_err(ctx);
+        CK(cudaStreamSynchronize(ctx->stream));
+    }
+    return GSNP_OK;
 }
 
 gsnp_status gsnp_call_async(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0, uint64_t w1,
@@ -1111,12 +1114,15 @@ gsnp_status gsnp_call_dense(gsnp_ctx* ctx, const gsnp_reads* reads, uint64_t w0,
         CK(cudaMemsetAsync(D.occ, 0, n * DENSE_SITE_BYTES, s));
         ctx->end(GSNP_STAGE_DENSE_RECYCLE);
     }
-    if (!dev_out)
-        CK(cudaMemcpyAsync(out, d_out, S * sizeof(gsnp_record), cudaMemcpyDeviceToHost, s));
     st = read_err(ctx);
     if (st == GSNP_E_CAPACITY)              // a saturated cell leaves residue behind: start clean
         cudaMemsetAsync(ctx->dense_occ.p, 0, ctx->dense_occ.n, s);
-    return st;
+    if (st) return st;                      // on an error the records were not all written
+    if (!dev_out) {
+        CK(cudaMemcpyAsync(out, d_out, S * sizeof(gsnp_record), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+    }
+    return GSNP_OK;
 }
 
 gsnp_status gsnp_parse_soap(gsnp_ctx* ctx, const char* text, uint64_t n_bytes, const char* chr_name,

@@ -1609,14 +1609,7 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
     // Positions are handled relative to the group's first site g0 (32-bit).  If every read in
     // the range has the same length, '-' strand reads share a coordinate only within one start
     // run and the end tracking below is skipped.
-#ifndef GSNP_PF_NEXT
-#define GSNP_PF_NEXT 0
-#endif
-#ifndef GSNP_LEN_PRECHECK
-#define GSNP_LEN_PRECHECK 1
-#endif
-    uint32_t one_len = GSNP_LEN_PRECHECK;
-#if GSNP_LEN_PRECHECK
+    uint32_t one_len = 1;
     {
         const uint32_t L0 = wra < wrb ? A.R.len[wra] : 0u;
         for (uint64_t r0 = wra; r0 < wrb; r0 += 32) {          // warp-uniform trip count
@@ -1624,7 +1617,6 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
             one_len &= (uint32_t)__all_sync(FULL, r >= wrb || A.R.len[r] == L0);
         }
     }
-#endif
     uint32_t ca0 = 0, ca1 = 0, ca2 = 0, ca3 = 0, rep = 0, n = 0;
     bool slow_pcr = false, have_minus = false;
     int run_pos = INT32_MIN;
@@ -1712,17 +1704,6 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
         }
         ca0 += cpack & 255u; ca1 += (cpack >> 8) & 255u; ca2 += (cpack >> 16) & 255u; ca3 += cpack >> 24;
     }
-#if GSNP_PF_NEXT
-    // the next group's read bytes into L2 while this group sorts and sums (its gather then waits
-    // for L2, not HBM)
-    if (nxt < n_groups && nra < nrb) {
-        const uint64_t pa = A.R.off[nra] - A.R.off0, pb = A.R.off[nrb] - A.R.off0;
-        for (uint64_t x = (pa & ~127ull) + 128ull * lane; x < pb; x += 4096) {
-            asm volatile("prefetch.global.L2 [%0];" ::"l"(A.R.bases + x));
-            asm volatile("prefetch.global.L2 [%0];" ::"l"(A.R.quals + x));
-        }
-    }
-#endif
     if (err) atomicOr(A.err, err);
     if (DBG && A.count_only) {
         if (active) A.dbg_nuni[site - A.w0] = n;
