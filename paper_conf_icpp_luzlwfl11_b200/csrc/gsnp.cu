@@ -780,14 +780,18 @@ gsnp_status compress_impl(gsnp_ctx* ctx, const gsnp_record* d_rec, uint64_t n, u
     A.dict = ctx->cz_dict.p;
     A.off = ctx->cz_off.p;
     const size_t sm_size = SMEM_SIZE_WORDS * 4, sm_write = SMEM_WRITE_WORDS * 4;
+    const size_t sm_light = SMEM_LIGHT_WORDS * 4;
     CK(cudaFuncSetAttribute(k_cz_sections<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_size));
     CK(cudaFuncSetAttribute(k_cz_sections<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_write));
+    // sections [0, SEC_S): header, planes, exception lists (light); [SEC_S, NSEC): dictionaries
+    const int nlight = SEC_S, nheavy = NSEC - SEC_S;
     ctx->begin();
     const unsigned g0 = (unsigned)std::min<uint64_t>((n + 255) / 256, (uint64_t)ctx->num_sms * 8);
     k_cz_columns<<<g0, 256, 0, s>>>(d_rec, n, A.col);
-    k_cz_sections<false><<<(unsigned)(nblk * NSEC), gsnp_cz::NT, sm_size, s>>>(A);
+    k_cz_sections<false><<<(unsigned)(nblk * nlight), gsnp_cz::NT, sm_light, s>>>(A, 0, nlight);
+    k_cz_sections<false><<<(unsigned)(nblk * nheavy), gsnp_cz::NT, sm_size, s>>>(A, SEC_S, nheavy);
     k_cz_scan<<<1, 1024, 0, s>>>(ctx->cz_meta.p, nblk * NSEC, ctx->cz_off.p);
-    ctx->launches += 3;
+    ctx->launches += 4;
     CK(cudaGetLastError());
     gsnp_status pst = peek(ctx, 3, ctx->cz_off.p + nblk * NSEC, 8);
     if (pst) return pst;
@@ -806,8 +810,9 @@ gsnp_status compress_impl(gsnp_ctx* ctx, const gsnp_record* d_rec, uint64_t n, u
         CK(ctx->cz_out.ensure(total));
         A.out = ctx->cz_out.p;
     }
-    k_cz_sections<true><<<(unsigned)(nblk * NSEC), gsnp_cz::NT, sm_write, s>>>(A);
-    ctx->launches += 1;
+    k_cz_sections<true><<<(unsigned)(nblk * nlight), gsnp_cz::NT, sm_light, s>>>(A, 0, nlight);
+    k_cz_sections<true><<<(unsigned)(nblk * nheavy), gsnp_cz::NT, sm_write, s>>>(A, SEC_S, nheavy);
+    ctx->launches += 2;
     ctx->end(GSNP_STAGE_COMPRESS);
     CK(cudaGetLastError());
     if (!dev_out) {              // host output: the words must have landed when we return

@@ -535,13 +535,15 @@ __device__ void sec_rle(const CzArgs& A, const BlockCtx& bk, int ci, Smem& S, ui
     }
 }
 
-// grid nblk * NSEC; WRITE = false sizes the sections, true writes them
+// grid nblk * nsec: sections [sec0, sec0 + nsec) of every block (the exception-list sections and
+// the dictionary sections are launched apart, each with the shared memory it needs, so the light
+// ones run four CTAs per SM); WRITE = false sizes the sections, true writes them
 template <bool WRITE>
-__global__ void __launch_bounds__(NT) k_cz_sections(CzArgs A) {
+__global__ void __launch_bounds__(NT) k_cz_sections(CzArgs A, int sec0, int nsec) {
     extern __shared__ __align__(16) uint32_t sm[];
     __shared__ Smem S;
-    const int sec = (int)(blockIdx.x % NSEC);           // the 16 sections of a block are
-    const uint32_t blk = blockIdx.x / NSEC;            // adjacent in launch order
+    const int sec = sec0 + (int)(blockIdx.x % nsec);    // a block's sections are adjacent in
+    const uint32_t blk = blockIdx.x / nsec;            // launch order
     BlockCtx bk;
     bk.blk = blk;
     bk.g0 = (uint64_t)blk * A.B;
@@ -618,7 +620,9 @@ __global__ void __launch_bounds__(1024) k_cz_scan(const uint32_t* meta, uint64_t
     if (threadIdx.x == 0) off[nsec] = carry;
 }
 
-// dynamic shared memory of k_cz_sections (words): the RLE section is the largest user
+// dynamic shared memory of k_cz_sections (words): the RLE section is the largest user; the
+// header, plane and exception sections need only the packer's staging window
+constexpr size_t SMEM_LIGHT_WORDS = PKW;
 constexpr size_t SMEM_SIZE_WORDS = 2 * CH + 2 * HS + 4 + DICT_MAX;
 constexpr size_t SMEM_WRITE_WORDS = 2 * CH + 2 * DICT_MAX + 2 * PKW;
 static_assert(HS + 2 + DICT_MAX <= SMEM_SIZE_WORDS, "S section (size pass) fits");
