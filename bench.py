@@ -371,7 +371,7 @@ def run_gpu(args):
     # — and every e2e step ships them through the C ABI's host-buffer path
     # (gsnp_unpack_reads: chunked H2D on the library's copy stream, decoded in HBM as chunks land)
     t_pack = time.perf_counter()
-    packed = torch.from_numpy(gsnp.pack_reads(w, 1024)).pin_memory()
+    packed = torch.from_numpy(gsnp.pack_reads(w, 1024, ref=w["ref"], origin=int(w["origin"]))).pin_memory()
     t_pack = time.perf_counter() - t_pack
     h2d_packed = packed.numel()
 
@@ -493,9 +493,10 @@ def run_gpu(args):
     ok_pk = check_cz() and all(bool(torch.equal(dev2[k], dev[k])) for k in ("pos", "bases", "quals"))
     e2e = {"value": total_sites / (te_pk / 1e3), "unit": UNIT, "h2d_bytes_per_step": h2d_packed,
            "d2h_bytes_per_step": 4 * sum(znw), "ms_per_step": te_pk, "check": ok_pk,
-           "input": "packed reads R21 in pinned host memory (%.2f B/base; packed once by "
-                    "gsnp_pack_reads in %.2f s on the host, outside the step) -> gsnp_unpack_reads "
-                    "(C ABI, host buffer: chunked H2D + k_unpack)" % (h2d_packed / max(1, len(w["bases"])), t_pack),
+           "input": "packed reads R21 v2 (bases relative to the reference) in pinned host memory "
+                    "(%.2f B/base; packed once by gsnp_pack_reads in %.2f s on the host, outside the "
+                    "step) -> gsnp_unpack_reads (C ABI, host buffer: chunked H2D + k_unpack against the "
+                    "context's device reference)" % (h2d_packed / max(1, len(w["bases"])), t_pack),
            "result": "RLE-DICT-compressed records (gsnp_call_compressed, §V-B) in %d window chunks "
                      "(geometric, 2:1 per step), each chunk's download overlapped with the next call" % K,
            "breakdown_ms": bd_pk,

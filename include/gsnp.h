@@ -191,10 +191,15 @@ gsnp_status gsnp_parse_soap(gsnp_ctx* ctx, const char* text, uint64_t n_bytes, c
  * against 221 unpacked.
  *
  * gsnp_pack_reads: encode host reads (on_device 0; bases contiguous per read at off[r]) on the
- *   host's cores.  block_reads 1..4096.  out: host buffer of cap bytes; *n_bytes receives the
+ *   host's cores.  ref NULL: version 1 (2-bit bases); ref given (host codes, the reference the
+ *   reads are aligned to): version 2 — a base is predicted as the reference code at its site and
+ *   only the bases that differ are stored (u32 block-relative index << 3 | code), ~0.3 B/base
+ *   instead of ~0.5; such a stream must be unpacked by a context created on the same reference.
+ *   block_reads 1..4096.  out: host buffer of cap bytes; *n_bytes receives the
  *   stream size (also on GSNP_E_CAPACITY, when out is NULL or cap too small — a size query).
- *   A length outside 1..256, base > 4, quality > 63, strand > 1, hits 0, or a position before its
- *   block's first read or >= 2^32 past it -> GSNP_E_RANGE.  No context needed.
+ *   A length outside 1..256, base > 4, quality > 63, strand > 1, hits 0, a position before its
+ *   block's first read or >= 2^32 past it, or (version 2) a read outside ref -> GSNP_E_RANGE.
+ *   No context needed.
  * gsnp_packed_sizes: n_reads / n_bases of a stream (host memory; the header is checked).
  * gsnp_unpack_reads: decode a stream (host — copied H2D in chunks on the library's copy stream,
  *   overlapped with the decode — or device memory) into DEVICE arrays sized by gsnp_packed_sizes
@@ -202,8 +207,8 @@ gsnp_status gsnp_parse_soap(gsnp_ctx* ctx, const char* text, uint64_t n_bytes, c
  *   params.stream; the call returns once a host stream has been copied (it may be reused).  The
  *   decoded reads are then passed to gsnp_calibrate / gsnp_call like any device reads (they are
  *   validated there).  A bad header -> GSNP_E_INVAL. */
-gsnp_status gsnp_pack_reads(const gsnp_reads* reads, uint32_t block_reads, void* out, uint64_t cap,
-                            uint64_t* n_bytes);
+gsnp_status gsnp_pack_reads(const gsnp_reads* reads, const gsnp_reference* ref, uint32_t block_reads,
+                            void* out, uint64_t cap, uint64_t* n_bytes);
 gsnp_status gsnp_packed_sizes(const void* packed, uint64_t n_bytes, uint64_t* n_reads,
                               uint64_t* n_bases);
 gsnp_status gsnp_unpack_reads(gsnp_ctx* ctx, const void* packed, uint64_t n_bytes, uint64_t* pos,

@@ -12,7 +12,7 @@ loops over reads (numpy only for the bit packing), sharing nothing with libgsnp'
 GPU decoder.  Layout (all little-endian; every section starts 16-byte aligned):
 
   header, 128 bytes:
-    0 magic b"GSR1"  4 version u32 = 1  8 n_reads u64  16 n_bases u64  24 n_runs u64
+    0 magic b"GSR1"  4 version u32 (1; 2 below)  8 n_reads u64  16 n_bases u64  24 n_runs u64
     32 n_nexc u64  40 n_hexc u64  48 n_blocks u32  52 block_reads u32
     56 section offsets u64[6]: blocks, meta, bases, runs, nexc, hexc   104..127 zero
   blocks  n_blocks x 5 u64: pos0 (first read's position), and the numbers of bases, runs,
@@ -28,6 +28,13 @@ GPU decoder.  Layout (all little-endian; every section starts 16-byte aligned):
 
 Reads are blocks of block_reads consecutive reads; within a block pos - pos0 must fit in 32 bits.
 Unpacking yields off = [0, len0, len0+len1, ...] (bases contiguous).
+
+Version 2 (reference-relative bases): aligned reads mostly repeat the reference under them, so
+with the reference at hand (it is resident on the device anyway) a base is predicted as the
+reference code at its site (N where the reference is N) and only the bases that differ are
+stored: the bases section is empty and the nexc section lists u32 (base index minus the block's
+first base index) << 3 | code for every mismatching base (codes 0..4).  Everything else is as in
+version 1.  A version-2 stream decodes only against the same reference.
 """
 from __future__ import annotations
 
@@ -43,8 +50,12 @@ def _a16(x: int) -> int:
     return (x + 15) & ~15
 
 
-def pack(w: dict, block_reads: int = 1024) -> bytes:
-    """Encode the read arrays of w (pos, len, off, bases, quals, strand, hits) in format R21."""
+def pack(w: dict, block_reads: int = 1024, ref=None, origin: int = 0) -> bytes:
+    """Encode the read arrays of w (pos, len, off, bases, quals, strand, hits) in format R21;
+    with ref (codes, known-SNP bit 3 allowed) and origin, version 2 (reference-relative)."""
+    v2 = ref is not None
+    if v2:
+        ref = np.asarray(ref, np.uint8)
     pos = np.asarray(w["pos"], np.uint64)
     ln = np.asarray(w["len"], np.int64)
     off = np.asarray(w["off"], np.int64)
@@ -82,10 +93,20 @@ def pack(w: dict, block_reads: int = 1024) -> bytes:
                 hexc += [r - r0, int(hits[r])]
             bb = bases_in[int(off[r]):int(off[r]) + L]
             qq = quals_in[int(off[r]):int(off[r]) + L]
+            if v2:
+                s0 = int(pos[r]) - origin
+                if s0 < 0 or s0 + L > len(ref):
+                    raise ValueError(f"read {r}: outside the reference")
             for i in range(L):
                 c = int(bb[i])
                 if c > 4 or int(qq[i]) > 63:
                     raise ValueError(f"read {r}: base/quality out of range")
+                if v2:
+                    rc = int(ref[s0 + i]) & 7
+                    pred = rc if rc < 4 else 4
+                    if c != pred:
+                        nexc.append((n_bases + i - base0) << 3 | c)
+                    continue
                 if c == 4:
                     nexc.append(n_bases + i - base0)
                     c = 0
@@ -102,10 +123,13 @@ def pack(w: dict, block_reads: int = 1024) -> bytes:
                 k = e
             nrun_m1[r] = nr - 1
             n_bases += L
-    cd = np.zeros(_a16((n_bases + 3) // 4) * 4, np.uint8)
-    cd[:n_bases] = codes
-    packed_bases = (cd[0::4] | cd[1::4] << 2 | cd[2::4] << 4 | cd[3::4] << 6).astype(np.uint8)
-    packed_bases = packed_bases[:(n_bases + 3) // 4]
+    if v2:
+        packed_bases = np.zeros(0, np.uint8)
+    else:
+        cd = np.zeros(_a16((n_bases + 3) // 4) * 4, np.uint8)
+        cd[:n_bases] = codes
+        packed_bases = (cd[0::4] | cd[1::4] << 2 | cd[2::4] << 4 | cd[3::4] << 6).astype(np.uint8)
+        packed_bases = packed_bases[:(n_bases + 3) // 4]
     secs = [blocks.tobytes(), None, packed_bases.tobytes(), np.asarray(runs, np.uint16).tobytes(),
             np.asarray(nexc, np.uint32).tobytes(), np.asarray(hexc, np.uint32).tobytes()]
     meta = b""
@@ -117,7 +141,7 @@ def pack(w: dict, block_reads: int = 1024) -> bytes:
     for sct in secs:
         offs.append(cur)
         cur = _a16(cur + len(sct))
-    hdr = MAGIC + struct.pack("<IQQQQQII6Q", 1, n, n_bases, len(runs), len(nexc), len(hexc) // 2,
+    hdr = MAGIC + struct.pack("<IQQQQQII6Q", 2 if v2 else 1, n, n_bases, len(runs), len(nexc), len(hexc) // 2,
                               nblk, block_reads, *offs)
     hdr += b"\0" * (HDR - len(hdr))
     out = bytearray(cur)
@@ -138,9 +162,13 @@ def header(buf: bytes) -> dict:
     return d
 
 
-def unpack(buf: bytes) -> dict:
-    """Decode a GSR1 stream back to read arrays (off rebuilt contiguous from 0)."""
+def unpack(buf: bytes, ref=None, origin: int = 0) -> dict:
+    """Decode a GSR1 stream back to read arrays (off rebuilt contiguous from 0); a version-2
+    stream needs the reference it was packed against."""
     h = header(buf)
+    v2 = h["version"] == 2
+    if v2 and ref is None:
+        raise ValueError("version-2 stream: the reference is needed")
     n, nb, B = h["n_reads"], h["n_bases"], h["block_reads"]
     s_blk, s_meta, s_bases, s_runs, s_nexc, s_hexc = h["sections"]
     blocks = np.frombuffer(buf, np.uint64, h["n_blocks"] * 5, s_blk).reshape(-1, 5)
@@ -152,7 +180,7 @@ def unpack(buf: bytes) -> dict:
     sh = np.frombuffer(buf, np.uint8, n, o)
     o = _a16(o + n)
     nrun_m1 = np.frombuffer(buf, np.uint8, n, o)
-    pb = np.frombuffer(buf, np.uint8, (nb + 3) // 4, s_bases)
+    pb = np.frombuffer(buf, np.uint8, 0 if v2 else (nb + 3) // 4, s_bases)
     runs = np.frombuffer(buf, np.uint16, h["n_runs"], s_runs)
     nexc = np.frombuffer(buf, np.uint32, h["n_nexc"], s_nexc)
     hexc = np.frombuffer(buf, np.uint32, 2 * h["n_hexc"], s_hexc).reshape(-1, 2)
@@ -163,8 +191,16 @@ def unpack(buf: bytes) -> dict:
     strand = (sh >> 7).astype(np.uint8)
     hits = ((sh & 127).astype(np.uint16) + 1)
     bases = np.zeros(nb, np.uint8)
-    for k in range(4):
-        bases[k::4] = (pb >> (2 * k)) & 3
+    if v2:                                   # the reference under every base
+        ref = np.asarray(ref, np.uint8)
+        for b in range(h["n_blocks"]):
+            for r in range(b * B, min(n, (b + 1) * B)):
+                s0 = int(blocks[b][0]) + int(pos_rel[r]) - origin
+                rc = ref[s0:s0 + int(ln[r])] & 7
+                bases[int(off[r]):int(off[r + 1])] = np.where(rc < 4, rc, 4)
+    else:
+        for k in range(4):
+            bases[k::4] = (pb >> (2 * k)) & 3
     quals = np.zeros(nb, np.uint8)
     ri = 0
     for b in range(h["n_blocks"]):
@@ -183,7 +219,10 @@ def unpack(buf: bytes) -> dict:
             assert k == int(off[r + 1])
         ne1 = int(blocks[b + 1][3]) if b + 1 < h["n_blocks"] else h["n_nexc"]
         for e in nexc[ne0:ne1]:
-            bases[base0 + int(e)] = 4
+            if v2:
+                bases[base0 + (int(e) >> 3)] = int(e) & 7
+            else:
+                bases[base0 + int(e)] = 4
         he1 = int(blocks[b + 1][4]) if b + 1 < h["n_blocks"] else h["n_hexc"]
         for rr, hv in hexc[he0:he1]:
             hits[r0 + int(rr)] = hv

@@ -1280,8 +1280,8 @@ gsnp_status gsnp_parse_soap(gsnp_ctx* ctx, const char* text, uint64_t n_bytes, c
     return GSNP_OK;
 }
 
-gsnp_status gsnp_pack_reads(const gsnp_reads* reads, uint32_t block_reads, void* out, uint64_t cap,
-                            uint64_t* n_bytes) {
+gsnp_status gsnp_pack_reads(const gsnp_reads* reads, const gsnp_reference* ref, uint32_t block_reads,
+                            void* out, uint64_t cap, uint64_t* n_bytes) {
     using namespace gsnp_pk;
     if (n_bytes) *n_bytes = 0;
     if (!reads || reads->on_device) return GSNP_E_INVAL;
@@ -1289,8 +1289,11 @@ gsnp_status gsnp_pack_reads(const gsnp_reads* reads, uint32_t block_reads, void*
     const uint64_t n = reads->n_reads;
     if (n && (!reads->pos || !reads->len || !reads->off || !reads->bases || !reads->quals ||
               !reads->strand || !reads->hits)) return GSNP_E_INVAL;
-    HostReads R{n, reads->pos, reads->len, reads->off, reads->bases, reads->quals, reads->strand,
+    if (ref && (!ref->code || ref->n_sites == 0)) return GSNP_E_INVAL;
+    HostReads R{ref ? ref->code : nullptr, ref ? ref->origin : 0, ref ? ref->n_sites : 0,
+                n, reads->pos, reads->len, reads->off, reads->bases, reads->quals, reads->strand,
                 reads->hits};
+    const uint32_t version = ref ? 2u : 1u;
     const uint64_t nblk = (n + block_reads - 1) / block_reads;
     std::vector<BlockSize> bs(nblk);
     const int nt = (int)std::max(1u, std::min(32u, std::thread::hardware_concurrency()));
@@ -1321,7 +1324,8 @@ gsnp_status gsnp_pack_reads(const gsnp_reads* reads, uint32_t block_reads, void*
     h.sec[1] = a16(h.sec[0] + 40 * nblk);
     meta_offsets(h);
     h.sec[2] = a16(h.m_nrun + n);
-    h.sec[3] = a16(h.sec[2] + (h.n_bases + 3) / 4);
+    h.version = version;
+    h.sec[3] = a16(h.sec[2] + (version == 1 ? (h.n_bases + 3) / 4 : 0));
     h.sec[4] = a16(h.sec[3] + 2 * h.n_runs);
     h.sec[5] = a16(h.sec[4] + 4 * h.n_nexc);
     const uint64_t total = a16(h.sec[5] + 8 * h.n_hexc);
@@ -1329,7 +1333,7 @@ gsnp_status gsnp_pack_reads(const gsnp_reads* reads, uint32_t block_reads, void*
     if (!out || cap < total) return GSNP_E_CAPACITY;
     uint8_t* o = static_cast<uint8_t*>(out);
     memset(o, 0, HDR);
-    const uint32_t magic = MAGIC, ver = 1;
+    const uint32_t magic = MAGIC, ver = version;
     memcpy(o, &magic, 4); memcpy(o + 4, &ver, 4);
     memcpy(o + 8, &h.n_reads, 8); memcpy(o + 16, &h.n_bases, 8); memcpy(o + 24, &h.n_runs, 8);
     memcpy(o + 32, &h.n_nexc, 8); memcpy(o + 40, &h.n_hexc, 8); memcpy(o + 48, &h.n_blocks, 4);
@@ -1386,6 +1390,9 @@ gsnp_status gsnp_unpack_reads(gsnp_ctx* ctx, const void* packed, uint64_t n_byte
     UnpackArgs U;
     memset(&U, 0, sizeof U);
     U.h = h;
+    U.ref = ctx->ref_code;
+    U.origin = ctx->origin;
+    U.n_sites = ctx->n_sites;
     U.pos = pos; U.len = len; U.off = off; U.bases = bases; U.quals = quals; U.strand = strand;
     U.hits = hits;
     if (h.n_reads == 0) {
@@ -1444,7 +1451,7 @@ gsnp_status gsnp_unpack_reads(gsnp_ctx* ctx, const void* packed, uint64_t n_byte
         CK(cp(h.m_len + r0, h.m_len + r1));
         CK(cp(h.m_sh + r0, h.m_sh + r1));
         CK(cp(h.m_nrun + r0, h.m_nrun + r1));
-        CK(cp(h.sec[2] + brow(b0, 1) / 4, h.sec[2] + (brow(b1, 1) + 3) / 4));
+        if (h.version == 1) CK(cp(h.sec[2] + brow(b0, 1) / 4, h.sec[2] + (brow(b1, 1) + 3) / 4));
         CK(cp(h.sec[3] + 2 * brow(b0, 2), h.sec[3] + 2 * brow(b1, 2)));
         CK(cp(h.sec[4] + 4 * brow(b0, 3), h.sec[4] + 4 * brow(b1, 3)));
         CK(cp(h.sec[5] + 8 * brow(b0, 4), h.sec[5] + 8 * brow(b1, 4)));

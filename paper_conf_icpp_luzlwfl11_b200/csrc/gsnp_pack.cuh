@@ -22,6 +22,7 @@ constexpr int UNT = 256;                      // k_unpack threads per CTA
 __host__ __device__ inline uint64_t a16(uint64_t x) { return (x + 15) & ~uint64_t(15); }
 
 struct Header {                               // the 128-byte header, parsed
+    uint32_t version;                         // 1: 2-bit bases; 2: reference-relative bases
     uint64_t n_reads, n_bases, n_runs, n_nexc, n_hexc;
     uint32_t n_blocks, block_reads;
     uint64_t sec[6];                          // blocks, meta, bases, runs, nexc, hexc
@@ -43,7 +44,8 @@ inline bool parse_header(const uint8_t* p, uint64_t n_bytes, Header& h) {
     uint32_t magic, ver;
     memcpy(&magic, p, 4);
     memcpy(&ver, p + 4, 4);
-    if (magic != MAGIC || ver != 1) return false;
+    if (magic != MAGIC || (ver != 1 && ver != 2)) return false;
+    h.version = ver;
     memcpy(&h.n_reads, p + 8, 8);
     memcpy(&h.n_bases, p + 16, 8);
     memcpy(&h.n_runs, p + 24, 8);
@@ -56,7 +58,7 @@ inline bool parse_header(const uint8_t* p, uint64_t n_bytes, Header& h) {
     if ((uint64_t)h.n_blocks != (h.n_reads + h.block_reads - 1) / h.block_reads) return false;
     meta_offsets(h);
     const uint64_t end[6] = {h.sec[0] + 40ull * h.n_blocks, a16(h.m_nrun + h.n_reads),
-                             h.sec[2] + (h.n_bases + 3) / 4, h.sec[3] + 2 * h.n_runs,
+                             h.sec[2] + (h.version == 1 ? (h.n_bases + 3) / 4 : 0), h.sec[3] + 2 * h.n_runs,
                              h.sec[4] + 4 * h.n_nexc, h.sec[5] + 8 * h.n_hexc};
     for (int k = 0; k < 6; ++k)
         if (h.sec[k] < HDR || end[k] > n_bytes || end[k] < h.sec[k]) return false;
@@ -72,6 +74,8 @@ inline bool parse_header(const uint8_t* p, uint64_t n_bytes, Header& h) {
 struct UnpackArgs {
     const uint8_t* buf;                       // device copy of the stream (same byte offsets)
     Header h;
+    const uint8_t* ref;                       // version 2: the context's reference codes
+    uint64_t origin, n_sites;                 //            (code | known << 3) and its span
     uint32_t blk0;                            // first block of this launch
     uint64_t* pos;
     uint16_t* len;
@@ -155,13 +159,20 @@ __global__ void __launch_bounds__(UNT) k_unpack(const __grid_constant__ UnpackAr
             carry += __shfl_sync(0xFFFFFFFFu, x, 31);
         }
         __syncwarp();
+        // version 2: the predicted base is the reference code at the site (N where it is N)
+        const uint64_t rs = h.version == 2 ? pos0 + m_pos[i] - U.origin : 0;
         for (uint32_t p0 = 4 * lane; p0 < L; p0 += 128) {
 #pragma unroll
             for (uint32_t u = 0; u < 4; ++u) {
                 const uint32_t p = p0 + u;
                 if (p >= L) break;
                 const uint64_t k = kb + p;
-                const uint32_t code = (plane[k >> 2] >> (2 * (uint32_t)(k & 3))) & 3u;
+                uint32_t code;
+                if (h.version == 1) code = (plane[k >> 2] >> (2 * (uint32_t)(k & 3))) & 3u;
+                else {
+                    const uint32_t rc = rs + p < U.n_sites ? U.ref[rs + p] & 7u : 4u;
+                    code = rc < 4 ? rc : 4u;
+                }
                 uint32_t lo = 0, hi = nrun;                   // last run with start <= p
                 while (hi - lo > 1) {
                     const uint32_t mid = (lo + hi) >> 1;
@@ -176,7 +187,10 @@ __global__ void __launch_bounds__(UNT) k_unpack(const __grid_constant__ UnpackAr
     __syncthreads();
     // ---- exceptions of this block
     const uint32_t* nexc = reinterpret_cast<const uint32_t*>(U.buf + h.sec[4]);
-    for (uint64_t e = ne0 + tid; e < ne1; e += UNT) U.bases[base0 + nexc[e]] = 4;
+    if (h.version == 1)
+        for (uint64_t e = ne0 + tid; e < ne1; e += UNT) U.bases[base0 + nexc[e]] = 4;
+    else                                      // (block-relative base << 3 | code) of mismatches
+        for (uint64_t e = ne0 + tid; e < ne1; e += UNT) U.bases[base0 + (nexc[e] >> 3)] = (uint8_t)(nexc[e] & 7u);
     const uint32_t* hexc = reinterpret_cast<const uint32_t*>(U.buf + h.sec[5]);
     for (uint64_t e = he0 + tid; e < he1; e += UNT) U.hits[r0 + hexc[2 * e]] = (uint16_t)hexc[2 * e + 1];
 }
@@ -192,6 +206,8 @@ __global__ void __launch_bounds__(UNT) k_unpack(const __grid_constant__ UnpackAr
 namespace gsnp_pk {
 
 struct HostReads {
+    const uint8_t* ref;               // version 2: reference codes (NULL: version 1)
+    uint64_t origin, n_sites;
     uint64_t n;
     const uint64_t* pos;
     const uint16_t* len;
@@ -213,9 +229,19 @@ inline BlockSize size_block(const HostReads& R, uint64_t r0, uint64_t r1) {
             R.pos[r] - p0 >= (1ull << 32)) { s.bad = 1; return s; }
         const uint8_t* b = R.bases + R.off[r];
         const uint8_t* q = R.quals + R.off[r];
+        const uint8_t* rf = nullptr;
+        if (R.ref) {
+            if (R.pos[r] < R.origin || R.pos[r] - R.origin + L > R.n_sites) { s.bad = 1; return s; }
+            rf = R.ref + (R.pos[r] - R.origin);
+        }
         for (uint32_t i = 0; i < L; ++i) {
             if (b[i] > 4 || q[i] > 63) { s.bad = 1; return s; }
-            s.nexc += b[i] == 4;
+            if (rf) {
+                const uint32_t rc = rf[i] & 7u;
+                s.nexc += b[i] != (rc < 4 ? rc : 4u);
+            } else {
+                s.nexc += b[i] == 4;
+            }
             s.runs += (i == 0 || q[i] != q[i - 1]);
         }
         s.bases += L;
@@ -252,12 +278,18 @@ inline void write_block(const HostReads& R, uint64_t r0, uint64_t r1, const Head
         if (hm >= 127) { *hexc++ = (uint32_t)(r - r0); *hexc++ = R.hits[r]; }
         const uint8_t* b = R.bases + R.off[r];
         const uint8_t* q = R.quals + R.off[r];
+        const uint8_t* rf = R.ref ? R.ref + (R.pos[r] - R.origin) : nullptr;
         uint32_t nrun = 0;
         for (uint32_t i = 0; i < L; ++i, ++k) {
             uint32_t c = b[i];
-            if (c == 4) { *nexc++ = (uint32_t)(k - kb0); c = 0; }
-            acc |= c << (2 * (k & 3));
-            if ((k & 3) == 3) { put_byte(k >> 2, (uint8_t)acc); acc = 0; }
+            if (rf) {                                  // version 2: mismatches vs the reference
+                const uint32_t rc = rf[i] & 7u;
+                if (c != (rc < 4 ? rc : 4u)) *nexc++ = (uint32_t)(k - kb0) << 3 | c;
+            } else {
+                if (c == 4) { *nexc++ = (uint32_t)(k - kb0); c = 0; }
+                acc |= c << (2 * (k & 3));
+                if ((k & 3) == 3) { put_byte(k >> 2, (uint8_t)acc); acc = 0; }
+            }
             if (i == 0 || q[i] != q[i - 1]) {
                 uint32_t e = i + 1;
                 while (e < L && q[e] == q[i]) ++e;
@@ -267,7 +299,7 @@ inline void write_block(const HostReads& R, uint64_t r0, uint64_t r1, const Head
         }
         m_nrun[r] = (uint8_t)(nrun - 1);
     }
-    if (k & 3) put_byte(k >> 2, (uint8_t)acc);
+    if (!R.ref && (k & 3)) put_byte(k >> 2, (uint8_t)acc);
 }
 
 }  // namespace gsnp_pk

@@ -116,8 +116,8 @@ def lib():
         L.gsnp_parse_soap.argtypes = [P, P, u64, ctypes.c_char_p, ctypes.c_uint32, u64] + [P] * 7 + \
             [u64, u64, ctypes.POINTER(u64), ctypes.POINTER(u64)]
         L.gsnp_pack_reads.restype = S
-        L.gsnp_pack_reads.argtypes = [ctypes.POINTER(gsnp_reads), ctypes.c_uint32, P, u64,
-                                      ctypes.POINTER(u64)]
+        L.gsnp_pack_reads.argtypes = [ctypes.POINTER(gsnp_reads), ctypes.POINTER(gsnp_reference),
+                                      ctypes.c_uint32, P, u64, ctypes.POINTER(u64)]
         L.gsnp_packed_sizes.restype = S
         L.gsnp_packed_sizes.argtypes = [P, u64, ctypes.POINTER(u64), ctypes.POINTER(u64)]
         L.gsnp_unpack_reads.restype = S
@@ -438,15 +438,22 @@ def _nbytes(a) -> int:
     return np.asarray(a).nbytes
 
 
-def pack_reads(reads: dict, block_reads: int = 1024) -> np.ndarray:
-    """gsnp_pack_reads: host read arrays -> the packed stream R21 (numpy uint8)."""
+def pack_reads(reads: dict, block_reads: int = 1024, ref=None, origin: int = 0) -> np.ndarray:
+    """gsnp_pack_reads: host read arrays -> the packed stream R21 (numpy uint8); with ref (the
+    reference codes the reads are aligned to, origin = coordinate of ref[0]) version 2."""
     r = make_reads(reads)
+    rr = None
+    if ref is not None:
+        refa = np.ascontiguousarray(ref, np.uint8)
+        rr = gsnp_reference(_ptr(refa), len(refa), int(origin))
+        rr._keep = refa
     n = ctypes.c_uint64(0)
-    st = lib().gsnp_pack_reads(ctypes.byref(r), block_reads, None, 0, ctypes.byref(n))
+    rp = ctypes.byref(rr) if rr is not None else None
+    st = lib().gsnp_pack_reads(ctypes.byref(r), rp, block_reads, None, 0, ctypes.byref(n))
     if st not in (0, -7):
         _check(st, None)
     out = np.zeros(max(int(n.value), 1), np.uint8)
-    _check(lib().gsnp_pack_reads(ctypes.byref(r), block_reads, _ptr(out), out.nbytes,
+    _check(lib().gsnp_pack_reads(ctypes.byref(r), rp, block_reads, _ptr(out), out.nbytes,
                                  ctypes.byref(n)), None)
     return out[:int(n.value)]
 

@@ -89,3 +89,30 @@ def test_bad_stream_is_an_error():
             assert st == -1
         dev = ctx.unpack_reads(good)                      # the context is still usable
         assert int(dev["off"][-1]) == gsnp.packed_sizes(good)[1]
+
+
+@pytest.mark.parametrize("block_reads", [5, 1024])
+def test_reference_relative_stream_decodes_exactly(block_reads):
+    """Version 2 streams (bases predicted from the context's reference, mismatches listed):
+    written by the oracle, decoded on the GPU against the context's device reference."""
+    import torch
+    w = synth.generate("C1", n_sites=40_000, depth=15.0, seed=29)
+    w = dict(w, ref=np.asarray(w["ref"]).copy())
+    w["ref"][9000:9200] = 4                            # reads over an N stretch
+    buf = np.frombuffer(opk.pack(w, block_reads, ref=w["ref"], origin=int(w["origin"])), np.uint8)
+    with gsnp.Context.from_workload(w) as ctx:
+        _same(ctx.unpack_reads(buf), w)
+        _same(ctx.unpack_reads(torch.from_numpy(buf.copy()).cuda()), w)
+        torch.cuda.synchronize()
+
+
+def test_c2_reference_relative_roundtrip():
+    import torch
+    w = synth.generate("C2")
+    lo = int(w["origin"])
+    buf = gsnp.pack_reads(w, 1024, ref=w["ref"], origin=lo)
+    assert len(buf) < 0.35 * len(w["bases"])              # < 0.35 B per base on the wire
+    with gsnp.Context.from_workload(w, stream=torch.cuda.current_stream()) as ctx:
+        dev = ctx.unpack_reads(torch.from_numpy(buf).pin_memory())
+        torch.cuda.synchronize()
+        _same(dev, w)

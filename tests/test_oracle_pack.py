@@ -87,3 +87,37 @@ def test_rejects_out_of_range():
     bad = dict(w, pos=np.array([0, 2 ** 33], np.uint64))
     with pytest.raises(ValueError):
         opk.pack(bad)
+
+
+def test_hand_encoded_reference_relative_example():
+    """Version 2: the same two reads against reference ACGTACGTACGTACGT.  Read 0 at 7: reference
+    TACGT, read ACGTN -> every base differs (codes 0 1 3 2 4); read 1 at 9: reference CG, read
+    GG -> base 0 differs (code 3).  Exceptions: block-relative base index << 3 | code."""
+    w = _tiny()
+    buf = opk.pack(w, 1024, ref=w["ref"], origin=0)
+    v = struct.unpack_from("<IQQQQQII6Q", buf, 4)
+    assert v[:8] == (2, 2, 7, 4, 6, 1, 1, 1024)
+    s_blk, s_meta, s_bases, s_runs, s_nexc, s_hexc = v[8:]
+    assert s_bases == s_runs == 240                    # no base plane
+    assert struct.unpack_from("<6I", buf, s_nexc) == (0 << 3 | 0, 1 << 3 | 1, 2 << 3 | 3,
+                                                      3 << 3 | 2, 4 << 3 | 4, 5 << 3 | 3)
+    assert struct.unpack_from("<2I", buf, s_hexc) == (1, 200)
+    u = opk.unpack(buf, ref=w["ref"])
+    assert list(u["bases"]) == [0, 1, 3, 2, 4, 3, 3]
+    with pytest.raises(ValueError):
+        opk.unpack(buf)                                # needs the reference
+
+
+@pytest.mark.parametrize("block_reads", [7, 1024])
+def test_reference_relative_roundtrip(block_reads):
+    w = synth.generate("C1", n_sites=20_000, depth=10.0, seed=9)
+    ref = np.asarray(w["ref"]).copy()
+    ref[5000:5100] = 4                                 # an N block under some reads
+    ref[7000] |= 8                                     # a known-SNP flag (ignored by the code)
+    buf1 = opk.pack(w, block_reads)
+    buf2 = opk.pack(w, block_reads, ref=ref, origin=int(w["origin"]))
+    assert len(buf2) < 0.75 * len(buf1)
+    u = opk.unpack(buf2, ref=ref, origin=int(w["origin"]))
+    for k in ("bases", "quals", "pos", "strand", "hits"):
+        assert np.array_equal(u[k], opk.unpack(buf1)[k]), k
+    assert np.array_equal(u["bases"], np.asarray(w["bases"]))

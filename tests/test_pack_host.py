@@ -46,3 +46,18 @@ def test_encoder_errors():
     assert e.value.status == -1
     with pytest.raises(gsnp.GsnpError):
         gsnp.packed_sizes(np.zeros(200, np.uint8))
+
+
+@pytest.mark.parametrize("block_reads", [3, 1024])
+def test_library_reference_relative_encoder_equals_oracle(block_reads):
+    w = synth.generate("C1", n_sites=30_000, depth=12.0, seed=21)
+    ref = np.asarray(w["ref"]).copy()
+    ref[100:300] = 4
+    a = gsnp.pack_reads(w, block_reads, ref=ref, origin=int(w["origin"]))
+    b = np.frombuffer(opk.pack(w, block_reads, ref=ref, origin=int(w["origin"])), np.uint8)
+    assert a.tobytes() == b.tobytes()
+    bad = dict(w, pos=np.asarray(w["pos"]).copy())
+    bad["pos"][-1] = len(ref) - 5                      # past the reference end
+    with pytest.raises(gsnp.GsnpError) as e:
+        gsnp.pack_reads(bad, block_reads, ref=ref, origin=int(w["origin"]))
+    assert e.value.status == -2
