@@ -339,8 +339,8 @@ def run_gpu(args):
     # the window is called in K chunks of geometrically shrinking size (geometric, 2:1 per step), so each chunk's
     # result download hides under the next chunk's compute and the exposed tail is the smallest
     KR = int(os.environ.get("GSNP_E2E_READ_CHUNKS", "8"))
-    K = int(os.environ.get("GSNP_E2E_CHUNKS", "3"))   # 2/3/4: 58.39/58.22/58.49 ms
-    CZ_B = 65536
+    K = int(os.environ.get("GSNP_E2E_CHUNKS", "4"))   # packed input, B 32768: 2/3/4 chunks 30.6/30.3/29.9 ms
+    CZ_B = int(os.environ.get("GSNP_E2E_CZ_B", "32768"))     # 65536 / 16384: +0.7% / +1.6% e2e time
     pinned = {k: v.pin_memory() for k, v in host.items()}
     out_h = torch.empty(40 * S, dtype=torch.uint8).pin_memory()
     dev2 = {k: torch.empty_like(v, device="cuda") for k, v in host.items()}
