@@ -703,19 +703,12 @@ __device__ __forceinline__ int64_t site_ref(const CallArgs& A, uint64_t site, in
     return (int64_t)lower_bound_u64(A.known_pos, 0, A.n_known, site);
 }
 
-// C8/C9 and the 40-byte record (R8, R9).  Inlined into each path (measured 0.8% faster than one
-// shared out-of-line copy at C2); GSNP_RECORD_INLINE=0 restores the shared copy.
+// C8/C9 and the 40-byte record (R8, R9).  The 32-slot kernel has one calling path and inlines it
+// (measured 0.8% faster at C2); kernels with several paths share one out-of-line copy
+// (site_record_ool) — their code must stay within the instruction cache.
 // cu/qs: unique counts / quality sums per base; ca: all-hits counts; delta = lp[t1] - lp[t2];
 // wsum/tie: rank-sum pieces (valid for heterozygous calls with both alleles observed).
-#ifndef GSNP_RECORD_INLINE
-#define GSNP_RECORD_INLINE 1
-#endif
-#if GSNP_RECORD_INLINE
-__device__ __forceinline__
-#else
-__device__ __noinline__
-#endif
-void site_record(const CallArgs& A, uint64_t site, int refb, int known,
+__device__ __forceinline__ void site_record(const CallArgs& A, uint64_t site, int refb, int known,
                                          int t1, double delta, double post1, uint32_t cu0,
                                          uint32_t cu1, uint32_t cu2, uint32_t cu3, uint32_t qs0,
                                          uint32_t qs1, uint32_t qs2, uint32_t qs3, uint32_t ca0,
@@ -814,6 +807,16 @@ void site_record(const CallArgs& A, uint64_t site, int refb, int known,
     }
 }
 
+__device__ __noinline__ void site_record_ool(const CallArgs& A, uint64_t site, int refb, int known,
+                                            int t1, double delta, double post1, uint32_t cu0,
+                                            uint32_t cu1, uint32_t cu2, uint32_t cu3, uint32_t qs0,
+                                            uint32_t qs1, uint32_t qs2, uint32_t qs3, uint32_t ca0,
+                                            uint32_t ca1, uint32_t ca2, uint32_t ca3, uint32_t repeat,
+                                            double wsum, double tie) {
+    site_record(A, site, refb, known, t1, delta, post1, cu0, cu1, cu2, cu3, qs0, qs1, qs2, qs3, ca0,
+                ca1, ca2, ca3, repeat, wsum, tie);
+}
+
 // ------------------------------------------------------------------------------------------
 // Thread-per-site likelihood for n <= N <= 32 keys (the common case).  Each key was stored as
 // key << 8 | (pcr - 1) by the gather (pcr = occurrences of its (base, strand, coord) so far in
@@ -858,7 +861,7 @@ __device__ __forceinline__ void sort_column(uint32_t* colp, uint32_t n) {
 
 // C6-C9 for one site held by one thread: priors, posterior, top-2, rank-sum pieces, record.
 // SORTED: the column holds the site's keys in canonical order (rank-sum by one merge).
-template <bool DBG, bool SORTED>
+template <bool DBG, bool SORTED, bool INL>
 // lps: the novel log10 prior rows (R6) staged in shared memory; rt: the site's reference byte
 // (code | known << 3), loaded when the site's group was taken.
 __device__ __forceinline__ void thread_finish(const CallArgs& A, const double* lps, uint32_t rt,
@@ -946,12 +949,17 @@ __device__ __forceinline__ void thread_finish(const CallArgs& A, const double* l
             if (A.dbg_post10) A.dbg_post10[s * 10 + j] = exp10(lp[j] - m) / esum;
         }
     }
-    site_record(A, site, refb, kidx >= 0, t1, delta, 1.0 / esum, f16(cu, 0), f16(cu, 1),
-                f16(cu, 2), f16(cu, 3), f16(qs, 0), f16(qs, 1), f16(qs, 2), f16(qs, 3), ca0, ca1,
-                ca2, ca3, rep, wsum, tie);
+    if (INL)
+        site_record(A, site, refb, kidx >= 0, t1, delta, 1.0 / esum, f16(cu, 0), f16(cu, 1),
+                    f16(cu, 2), f16(cu, 3), f16(qs, 0), f16(qs, 1), f16(qs, 2), f16(qs, 3), ca0, ca1,
+                    ca2, ca3, rep, wsum, tie);
+    else
+        site_record_ool(A, site, refb, kidx >= 0, t1, delta, 1.0 / esum, f16(cu, 0), f16(cu, 1),
+                        f16(cu, 2), f16(cu, 3), f16(qs, 0), f16(qs, 1), f16(qs, 2), f16(qs, 3), ca0,
+                        ca1, ca2, ca3, rep, wsum, tie);
 }
 
-template <bool DBG>
+template <bool DBG, bool INL>
 __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* adj, const double* lps,
                                             uint32_t rt, uint32_t* colp,
                                             uint64_t site, uint32_t n, bool slow_pcr, uint32_t ca0,
@@ -1013,7 +1021,7 @@ __device__ __forceinline__ void thread_site(const CallArgs& A, const uint8_t* ad
         add_row(T, (int)L, kk >> 17, key_cyc(kk), key_base(kk), acc);
     }
 #endif
-    thread_finish<DBG, true>(A, lps, rt, colp, site, n, acc, cu, qs, ca0, ca1, ca2, ca3, rep);
+    thread_finish<DBG, true, INL>(A, lps, rt, colp, site, n, acc, cu, qs, ca0, ca1, ca2, ca3, rep);
 }
 
 #ifndef GSNP_DEEP_U
@@ -1094,7 +1102,7 @@ __device__ __forceinline__ void thread_site_deep(const CallArgs& A, const uint8_
 #pragma unroll
             for (int k = 0; k < 10; ++k) acc[k] += v[u][k];
     }
-    thread_finish<DBG, false>(A, lps, rt, colp, site, n, acc, cu, qs, ca0, ca1, ca2, ca3, rep);
+    thread_finish<DBG, false, false>(A, lps, rt, colp, site, n, acc, cu, qs, ca0, ca1, ca2, ca3, rep);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -1725,9 +1733,9 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
     const bool mid = CC > COLS && active && n > COLS && n <= CC && !slow_pcr;
     const uint32_t maxn = __reduce_max_sync(FULL, small ? n : 0u);
     if (small) {
-        if (maxn <= 16) sort_column<16>(colp, n);
-        else sort_column<32>(colp, n);
-        thread_site<DBG>(A, adj, lp_s, rt, colp, site, n, slow_pcr, ca0, ca1, ca2, ca3, rep);
+        if (CC == COLS && maxn <= 16) sort_column<16>(colp, n);   // (one network in the deeper
+        else sort_column<32>(colp, n);                           //  kernels: instruction cache)
+        thread_site<DBG, CC == COLS>(A, adj, lp_s, rt, colp, site, n, slow_pcr, ca0, ca1, ca2, ca3, rep);
     } else if (mid) {
         thread_site_deep<DBG, CC / 32>(A, adj, lp_s, rt, colp, site, n, ca0, ca1, ca2, ca3, rep);
     }
