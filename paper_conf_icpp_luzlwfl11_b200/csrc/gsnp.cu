@@ -758,7 +758,8 @@ gsnp_status compress_impl(gsnp_ctx* ctx, const gsnp_record* d_rec, uint64_t n, u
     const uint64_t nblk = (n + B - 1) / B;
     if (nblk * NSEC > 0x7FFFFFFFull) return fail(ctx, GSNP_E_RANGE, "too many compression blocks");
     const uint32_t DC = std::min<uint32_t>(DICT_MAX, B);
-    CK(ctx->cz_cols.ensure(32 * n));
+    const uint64_t npad = (n + 15) & ~15ull;         // every column 16-byte aligned (vector loads)
+    CK(ctx->cz_cols.ensure(32 * npad));
     CK(ctx->cz_meta.ensure(nblk * NSEC * 2));
     CK(ctx->cz_dD.ensure(nblk * NDICT));
     CK(ctx->cz_dict.ensure(nblk * NDICT * DC));
@@ -772,25 +773,26 @@ gsnp_status compress_impl(gsnp_ctx* ctx, const gsnp_record* d_rec, uint64_t n, u
     A.nblk = (uint32_t)nblk;
     A.DC = DC;
     uint8_t* base = ctx->cz_cols.p;                  // u32 columns, then u16, then u8
-    for (int k = 0; k < 4; ++k) A.col.u32[k] = reinterpret_cast<uint32_t*>(base + (size_t)4 * n * k);
-    for (int k = 0; k < 4; ++k) A.col.u16[k] = reinterpret_cast<uint16_t*>(base + 16 * n + (size_t)2 * n * k);
-    for (int k = 0; k < 8; ++k) A.col.u8[k] = base + 24 * n + (size_t)n * k;
+    for (int k = 0; k < 4; ++k) A.col.u32[k] = reinterpret_cast<uint32_t*>(base + (size_t)4 * npad * k);
+    for (int k = 0; k < 4; ++k) A.col.u16[k] = reinterpret_cast<uint16_t*>(base + 16 * npad + (size_t)2 * npad * k);
+    for (int k = 0; k < 8; ++k) A.col.u8[k] = base + 24 * npad + (size_t)npad * k;
     A.meta = ctx->cz_meta.p;
     A.dD = ctx->cz_dD.p;
     A.dict = ctx->cz_dict.p;
     A.off = ctx->cz_off.p;
-    const size_t sm_size = SMEM_SIZE_WORDS * 4, sm_write = SMEM_WRITE_WORDS * 4;
+    const size_t sm_size = SMEM_DSIZE_WORDS * 4, sm_write = SMEM_DWRITE_WORDS * 4;
     const size_t sm_light = SMEM_LIGHT_WORDS * 4;
-    CK(cudaFuncSetAttribute(k_cz_sections<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_size));
-    CK(cudaFuncSetAttribute(k_cz_sections<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_write));
-    // sections [0, SEC_S): header, planes, exception lists (light); [SEC_S, NSEC): dictionaries
-    const int nlight = SEC_S, nheavy = NSEC - SEC_S;
+    CK(cudaFuncSetAttribute(k_cz_dicts<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_size));
+    CK(cudaFuncSetAttribute(k_cz_dicts<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm_write));
+    // sections [0, SEC_S): header, planes, exception lists (k_cz_sections, one CTA per block and
+    // section); [SEC_S, NSEC): dictionary sections (k_cz_dicts, one CTA per block and dictionary)
+    const int nlight = SEC_S;
     ctx->begin();
     const unsigned g0 = (unsigned)std::min<uint64_t>((n + 255) / 256, (uint64_t)ctx->num_sms * 8);
     k_cz_columns<<<g0, 256, 0, s>>>(d_rec, n, A.col);
     k_cz_sections<false><<<(unsigned)(nblk * nlight), gsnp_cz::NT, sm_light, s>>>(A, 0, nlight);
-    k_cz_sections<false><<<(unsigned)(nblk * nheavy), gsnp_cz::NT, sm_size, s>>>(A, SEC_S, nheavy);
-    k_cz_scan<<<1, 1024, 0, s>>>(ctx->cz_meta.p, nblk * NSEC, ctx->cz_off.p);
+    k_cz_dicts<false><<<(unsigned)(nblk * NDICT), gsnp_cz::NT, sm_size, s>>>(A);
+    k_cz_scan<<<1, 1024, 0, s>>>(A, ctx->cz_off.p);
     ctx->launches += 4;
     CK(cudaGetLastError());
     gsnp_status pst = peek(ctx, 3, ctx->cz_off.p + nblk * NSEC, 8);
@@ -811,7 +813,7 @@ gsnp_status compress_impl(gsnp_ctx* ctx, const gsnp_record* d_rec, uint64_t n, u
         A.out = ctx->cz_out.p;
     }
     k_cz_sections<true><<<(unsigned)(nblk * nlight), gsnp_cz::NT, sm_light, s>>>(A, 0, nlight);
-    k_cz_sections<true><<<(unsigned)(nblk * nheavy), gsnp_cz::NT, sm_write, s>>>(A, SEC_S, nheavy);
+    k_cz_dicts<true><<<(unsigned)(nblk * NDICT), gsnp_cz::NT, sm_write, s>>>(A);
     ctx->launches += 2;
     ctx->end(GSNP_STAGE_COMPRESS);
     CK(cudaGetLastError());

@@ -21,6 +21,12 @@
 namespace gsnp_cz {
 
 constexpr int NT = 512;                    // threads per CTA
+#ifndef GSNP_CZ_MINB
+#define GSNP_CZ_MINB 4                     // CTAs per SM the section kernels are built for
+#endif
+#ifndef GSNP_CZ_MINB_W
+#define GSNP_CZ_MINB_W 4                   // (the dictionary write pass; 3 measured slower)
+#endif
 constexpr int NWP = NT / 32;
 constexpr int IT = 4;                      // consecutive sites per thread per chunk
 constexpr int CH = NT * IT;                // sites per chunk
@@ -131,18 +137,28 @@ __host__ __device__ __forceinline__ uint64_t dict_words(uint64_t m, uint32_t D) 
     return 1 + D + (m * b + 31) / 32;
 }
 
-// --- hash set of distinct values (dictionary construction, "sort + unique")
-struct HSet {
+// --- set of distinct values (dictionary construction, "sort + unique"): values below
+// BMV in a bitmap (sorted by construction), the rest in a hash set sorted at the end
+constexpr uint32_t BMV = 65536;            // bitmap range (2048 words)
+constexpr uint32_t BMW = BMV / 32;
+struct VSet {
+    uint32_t* bm;             // BMW words
     uint32_t* slot;           // HS words, EMPTY = free
-    uint32_t* cnt;            // [0] distinct non-EMPTY values, [1] saw 0xFFFFFFFF
+    uint32_t* cnt;            // [0] distinct hashed values, [1] saw 0xFFFFFFFF
 };
 
-__device__ __forceinline__ void hs_clear(HSet h) {
+__device__ __forceinline__ void vs_clear(VSet h) {
     for (int i = threadIdx.x; i < HS; i += NT) h.slot[i] = EMPTY;
+    for (int i = threadIdx.x; i < (int)BMW; i += NT) h.bm[i] = 0;
     if (threadIdx.x == 0) { h.cnt[0] = 0; h.cnt[1] = 0; }
 }
 
-__device__ __forceinline__ void hs_insert(HSet h, uint32_t v) {
+__device__ __forceinline__ void vs_insert(VSet h, uint32_t v) {
+    if (v < BMV) {
+        const uint32_t bit = 1u << (v & 31);
+        if (!(h.bm[v >> 5] & bit)) atomicOr(&h.bm[v >> 5], bit);
+        return;
+    }
     if (v == EMPTY) { h.cnt[1] = 1; return; }
     if (*(volatile uint32_t*)h.cnt > DICT_MAX) return;      // RAW already: stop (bounded fill)
     uint32_t s = (v * 2654435761u) >> 19;                  // 13 bits
@@ -158,40 +174,54 @@ __device__ __forceinline__ void hs_insert(HSet h, uint32_t v) {
     }
 }
 
-// Sorted unique list of the set into gdict (capacity >= D); returns D or RAW.  sb: DICT_MAX words.
-__device__ uint32_t hs_finalize(HSet h, uint32_t* sb, uint32_t* gdict, Smem& S) {
+// Sorted unique list of the set into gdict (capacity >= D); returns D or RAW.  sb: DICT_MAX words
+// of sort buffer (may overlap the bitmap: it is read first).
+__device__ uint32_t vs_finalize(VSet h, uint32_t* sb, uint32_t* gdict, Smem& S) {
     __syncthreads();
+    constexpr int PW = BMW / NT;
+    uint32_t w[PW], k = 0;
+#pragma unroll
+    for (int i = 0; i < PW; ++i) { w[i] = h.bm[threadIdx.x * PW + i]; k += __popc(w[i]); }
+    uint32_t nsmall;
+    uint32_t at = cta_scan(k, S, &nsmall);               // (ends with a barrier: bm is free)
     const uint32_t c = h.cnt[0], hasmax = h.cnt[1];
-    const uint32_t D = c + hasmax;
-    __syncthreads();
+    const uint32_t D = nsmall + c + hasmax;
     if (D > DICT_MAX) return RAW;
-    constexpr int PER = HS / NT;
-    uint32_t k = 0;
-    for (int i = 0; i < PER; ++i) k += h.slot[threadIdx.x * PER + i] != EMPTY;
-    uint32_t tot;
-    uint32_t at = cta_scan(k, S, &tot);
-    for (int i = 0; i < PER; ++i) {
-        uint32_t v = h.slot[threadIdx.x * PER + i];
-        if (v != EMPTY) sb[at++] = v;
-    }
-    uint32_t P2 = 1;
-    while (P2 < c) P2 <<= 1;
-    for (uint32_t i = c + threadIdx.x; i < P2; i += NT) sb[i] = EMPTY;
-    __syncthreads();
-    for (uint32_t kk = 2; kk <= P2; kk <<= 1)
-        for (uint32_t j = kk >> 1; j > 0; j >>= 1) {
-            for (uint32_t i = threadIdx.x; i < P2; i += NT) {
-                uint32_t ixj = i ^ j;
-                if (ixj > i) {
-                    uint32_t a = sb[i], b = sb[ixj];
-                    bool up = (i & kk) == 0;
-                    if ((a > b) == up) { sb[i] = b; sb[ixj] = a; }
-                }
-            }
-            __syncthreads();
+#pragma unroll
+    for (int i = 0; i < PW; ++i)
+        while (w[i]) {
+            gdict[at++] = (threadIdx.x * PW + i) * 32 + __ffs(w[i]) - 1;
+            w[i] &= w[i] - 1;
         }
-    for (uint32_t i = threadIdx.x; i < c; i += NT) gdict[i] = sb[i];
-    if (hasmax && threadIdx.x == 0) gdict[c] = 0xFFFFFFFFu;
+    if (c) {                                             // hashed values: compact, bitonic sort
+        constexpr int PER = HS / NT;
+        uint32_t kk = 0;
+        for (int i = 0; i < PER; ++i) kk += h.slot[threadIdx.x * PER + i] != EMPTY;
+        uint32_t tot;
+        uint32_t a2 = cta_scan(kk, S, &tot);
+        for (int i = 0; i < PER; ++i) {
+            uint32_t v = h.slot[threadIdx.x * PER + i];
+            if (v != EMPTY) sb[a2++] = v;
+        }
+        uint32_t P2 = 1;
+        while (P2 < c) P2 <<= 1;
+        for (uint32_t i = c + threadIdx.x; i < P2; i += NT) sb[i] = EMPTY;
+        __syncthreads();
+        for (uint32_t q = 2; q <= P2; q <<= 1)
+            for (uint32_t j = q >> 1; j > 0; j >>= 1) {
+                for (uint32_t i = threadIdx.x; i < P2; i += NT) {
+                    uint32_t ixj = i ^ j;
+                    if (ixj > i) {
+                        uint32_t x = sb[i], y = sb[ixj];
+                        bool up = (i & q) == 0;
+                        if ((x > y) == up) { sb[i] = y; sb[ixj] = x; }
+                    }
+                }
+                __syncthreads();
+            }
+        for (uint32_t i = threadIdx.x; i < c; i += NT) gdict[nsmall + i] = sb[i];
+    }
+    if (hasmax && threadIdx.x == 0) gdict[nsmall + c] = 0xFFFFFFFFu;
     __syncthreads();
     return D;
 }
@@ -234,30 +264,46 @@ __device__ __forceinline__ void pk_final(const Packer& p, uint64_t m) {
     if (p.b && m * p.b > p.base && threadIdx.x == 0) p.g[p.base >> 5] = p.st[0];
 }
 
-// --- DICT output of one array: header, dictionary, packed indices (or RAW values)
+// --- DICT output of one array: header, dictionary, packed indices (or RAW values).
+// The index of a value is found by the paper's binary search in the sorted dictionary
+// (P:L779-780); values below LUTN take it from a direct table filled from the same dictionary
+// (the same index, one shared-memory load instead of ~12 dependent ones).
+constexpr uint32_t LUTN = 4096;
 struct DictOut {
     uint32_t D;
     const uint32_t* sd;       // sorted dictionary in shared memory (D words) unless RAW
+    const uint16_t* lut;      // lut[v] = index of v, for dictionary values v < LUTN
     uint32_t* g;              // section start in the output
     Packer pk;
 };
 
-__device__ __forceinline__ void do_init(DictOut& d, uint32_t D, uint32_t* sd, const uint32_t* gdict,
-                                        uint32_t* g, uint32_t* st, uint64_t m) {
-    d.D = D; d.sd = sd; d.g = g;
+__device__ __forceinline__ void do_init(DictOut& d, uint32_t D, uint32_t* sd, uint16_t* lut,
+                                        const uint32_t* gdict, uint32_t* g, uint32_t* st, uint64_t m) {
+    d.D = D; d.sd = sd; d.lut = lut; d.g = g;
     if (m == 0) { d.pk.b = 0; return; }
     if (threadIdx.x == 0) g[0] = D;
     if (D == RAW) { d.pk.b = 0; return; }
-    for (uint32_t i = threadIdx.x; i < D; i += NT) { uint32_t v = gdict[i]; sd[i] = v; g[1 + i] = v; }
+    for (uint32_t i = threadIdx.x; i < D; i += NT) {
+        uint32_t v = gdict[i];
+        sd[i] = v;
+        g[1 + i] = v;
+        if (v < LUTN) lut[v] = (uint16_t)i;
+    }
     pk_init(d.pk, st, g + 1 + D, D <= 1 ? 0 : bitlen(D - 1));
 }
 
 __device__ __forceinline__ void do_add(const DictOut& d, uint64_t j, uint32_t v) {
     if (d.D == RAW) { d.g[1 + j] = v; return; }
-    uint32_t lo = 0, hi = d.D;                 // parallel binary search
-    while (lo < hi) {
-        uint32_t mid = (lo + hi) >> 1;
-        if (d.sd[mid] < v) lo = mid + 1; else hi = mid;
+    uint32_t lo;
+    if (v < LUTN) {
+        lo = d.lut[v];
+    } else {
+        uint32_t hi = d.D;                     // parallel binary search
+        lo = 0;
+        while (lo < hi) {
+            uint32_t mid = (lo + hi) >> 1;
+            if (d.sd[mid] < v) lo = mid + 1; else hi = mid;
+        }
     }
     pk_add(d.pk, j, lo);
 }
@@ -359,187 +405,200 @@ __device__ __forceinline__ bool s_mask(const Cols& C, uint64_t gi) {
     return (C.u8[C_AVGQ2][gi] | C.u16[C_CU2 - 8][gi] | C.u16[C_CA2 - 8][gi]) != 0;
 }
 
-template <bool WRITE>
-__device__ void sec_second(const CzArgs& A, const BlockCtx& bk, Smem& S, uint32_t* sm) {
-    const Cols& C = A.col;
-    const uint32_t blk = bk.blk;
-    uint32_t* meta = A.meta + ((size_t)blk * NSEC + SEC_S) * 2;
-    uint32_t* dD = A.dD + (size_t)blk * NDICT;
-    uint32_t* gd = A.dict + (size_t)blk * NDICT * A.DC;
-    const uint32_t nbw = (bk.n + 31) / 32;
-    uint32_t* o = WRITE ? A.out + A.off[(size_t)blk * NSEC + SEC_S] : nullptr;
-    const uint32_t m = WRITE ? meta[1] : 0;
-    if (WRITE)
-        for (uint32_t w = threadIdx.x; w < nbw; w += NT) {
-            uint32_t v = 0;
-            for (uint32_t i = w * 32; i < bk.n && i < w * 32 + 32; ++i)
-                v |= (uint32_t)s_mask(C, bk.g0 + i) << (i % 32);
-            o[w] = v;
-        }
-    uint64_t words = nbw, at = nbw;
-    uint32_t mm = 0;
-    HSet h{sm, sm + HS};
-    uint32_t* sb = sm + HS + 2;
-    uint32_t* sd = sm;                               // write pass: dictionary
-    uint32_t* st = sm + DICT_MAX;                    //             packer staging
-    for (int k = 0; k < 3; ++k) {
-        const int c = k == 0 ? C_AVGQ2 : k == 1 ? C_CU2 : C_CA2;
-        DictOut d;
-        if (WRITE) {
-            __syncthreads();
-            do_init(d, dD[k], sd, gd + (size_t)k * A.DC, o + at, st, m);
-            __syncthreads();
-        } else {
-            hs_clear(h);
-            __syncthreads();
-        }
-        uint32_t run = 0;
-        for (uint32_t c0 = 0; c0 < bk.n; c0 += CH) {
-            uint32_t fl[IT], cnt = 0;
-#pragma unroll
-            for (int u = 0; u < IT; ++u) {
-                const uint32_t s = c0 + threadIdx.x * IT + u;
-                fl[u] = s < bk.n && s_mask(C, bk.g0 + s);
-                cnt += fl[u];
-                if (!WRITE && fl[u]) hs_insert(h, colv(C, c, bk.g0 + s));
-            }
-            if (WRITE) {
-                uint32_t tot, j;
-                j = run + cta_scan(cnt, S, &tot);
-#pragma unroll
-                for (int u = 0; u < IT; ++u)
-                    if (fl[u]) do_add(d, j++, colv(C, c, bk.g0 + c0 + threadIdx.x * IT + u));
-                run += tot;
-                __syncthreads();
-                if (d.D != RAW) pk_flush(d.pk, run);
-            } else {
-                uint32_t tot;
-                cta_scan(cnt, S, &tot);
-                run += tot;
-            }
-        }
-        if (WRITE) {
-            if (d.D != RAW) pk_final(d.pk, m);
-            at += dict_words(m, dD[k]);
-        } else {
-            mm = run;
-            const uint32_t D = hs_finalize(h, sb, gd + (size_t)k * A.DC, S);
-            if (threadIdx.x == 0) dD[k] = D;
-            words += dict_words(run, D);
-        }
-    }
-    if (!WRITE && threadIdx.x == 0) {
-        meta[0] = (uint32_t)words;
-        meta[1] = mm;
-    }
+__device__ __forceinline__ int rle_col(int ci) {
+    return ci == 0 ? C_QUAL : ci == 1 ? C_AVGQ1 : ci == 2 ? C_CU1 : ci == 3 ? C_CA1
+         : ci == 4 ? C_DEPTH : C_COPYN;
 }
 
-// quality column sections C0..C5: R, DICT(run values), DICT(run lengths)
-template <bool WRITE>
-__device__ void sec_rle(const CzArgs& A, const BlockCtx& bk, int ci, Smem& S, uint32_t* sm) {
+// IT (= 4) consecutive elements of a column from element i (n_left of them valid, the rest 0);
+// vec: the column and i are aligned for one vector load
+static_assert(IT == 4, "vector loads take four elements");
+template <typename T>
+__device__ __forceinline__ void ld4(const T* col, uint64_t i, bool vec, uint32_t n_left,
+                                    uint32_t (&v)[IT]) {
+    if (vec && n_left >= 4) {
+        if constexpr (sizeof(T) == 1) {
+            const uint32_t w = *reinterpret_cast<const uint32_t*>(col + i);
+#pragma unroll
+            for (int u = 0; u < 4; ++u) v[u] = (w >> (8 * u)) & 255u;
+        } else if constexpr (sizeof(T) == 2) {
+            const uint2 w = *reinterpret_cast<const uint2*>(col + i);
+            v[0] = w.x & 0xFFFFu; v[1] = w.x >> 16; v[2] = w.y & 0xFFFFu; v[3] = w.y >> 16;
+        } else {
+            const uint4 w = *reinterpret_cast<const uint4*>(col + i);
+            v[0] = w.x; v[1] = w.y; v[2] = w.z; v[3] = w.w;
+        }
+        return;
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) v[u] = (uint32_t)u < n_left ? (uint32_t)col[i + u] : 0u;
+}
+
+// One dictionary of one block per CTA (grid nblk x NDICT; dictionary d in dD order): d 0..2 the
+// S section's avgq2 / cnt_uni2 / cnt_all2 over the sites with a second allele;
+// d = 3 + 2 ci (+1) the run values (lengths) of quality column C<ci>.
+// KIND 0: masked values, 1: run values, 2: run lengths.
+//   size pass: set of the distinct values -> sorted dictionary in scratch, its size in dD, the
+//              element count (S: masked sites, C: runs) in meta[1] (section sizes: k_cz_scan)
+//   write pass: the DICT array at its place in the section (S: after the bitmap, written by d = 0
+//              and the dictionaries before it; C: R, then the values array, then the lengths)
+// shared layout  size:  hash HS + 2 | bitmap BMW | starts CH (bitmap + starts: the sort buffer)
+//                write: sd DICT_MAX | lut LUTN/2 | packer PKW | starts CH
+constexpr size_t SMEM_DSIZE_WORDS = HS + 2 + BMW + CH;
+constexpr size_t SMEM_DWRITE_WORDS = DICT_MAX + LUTN / 2 + PKW + CH;
+static_assert(BMW + CH >= DICT_MAX, "sort buffer");
+static_assert(BMW % NT == 0, "bitmap words per thread");
+
+template <bool WRITE, int KIND, typename T>
+__device__ __forceinline__ void dict_body(const CzArgs& A, const T* col, int d, uint32_t blk,
+                                          uint64_t g0, uint32_t n, uint32_t* sm, Smem& S) {
     const Cols& C = A.col;
-    const uint32_t blk = bk.blk;
-    const int sec = SEC_C + ci;
-    const int c = ci == 0 ? C_QUAL : ci == 1 ? C_AVGQ1 : ci == 2 ? C_CU1 : ci == 3 ? C_CA1
-                : ci == 4 ? C_DEPTH : C_COPYN;
+    const int sec = KIND == 0 ? SEC_S : SEC_C + (d - 3) / 2;
     uint32_t* meta = A.meta + ((size_t)blk * NSEC + sec) * 2;
-    uint32_t* dD = A.dD + (size_t)blk * NDICT + 3 + 2 * ci;
-    uint32_t* gd = A.dict + ((size_t)blk * NDICT + 3 + 2 * ci) * A.DC;
-    // shared layout: starts[CH], startv[CH], then (size) 2 hash sets + sort buffer
-    //                                               (write) 2 dictionaries + 2 packer windows
-    uint32_t* starts = sm;
-    uint32_t* startv = sm + CH;
-    uint32_t* rest = sm + 2 * CH;
-    HSet hv{rest, rest + 2 * HS}, hl{rest + HS, rest + 2 * HS + 2};
-    uint32_t* sb = rest + 2 * HS + 4;
-    DictOut dv, dl;
-    const uint32_t R = WRITE ? meta[1] : 0;
+    const uint32_t* dDb = A.dD + (size_t)blk * NDICT;
+    uint32_t* gd = A.dict + ((size_t)blk * NDICT + d) * A.DC;
+    VSet h{sm + HS + 2, sm, sm + HS};
+    uint32_t* starts = WRITE ? sm + DICT_MAX + LUTN / 2 + PKW : sm + HS + 2 + BMW;
+    const bool vec = (g0 & 3) == 0;                      // columns are 16-byte aligned
+    DictOut dout;
     if (WRITE) {
+        const uint32_t m = meta[1];
         uint32_t* o = A.out + A.off[(size_t)blk * NSEC + sec];
-        if (threadIdx.x == 0) o[0] = R;
-        do_init(dv, dD[0], rest, gd, o + 1, rest + 2 * DICT_MAX, R);
-        do_init(dl, dD[1], rest + DICT_MAX, gd + A.DC, o + 1 + dict_words(R, dD[0]),
-                rest + 2 * DICT_MAX + PKW, R);
+        uint64_t at = 1;
+        if (KIND == 0) {
+            const uint32_t nbw = (n + 31) / 32;
+            at = nbw;
+            for (int k = 0; k < d; ++k) at += dict_words(m, dDb[k]);
+            if (d == 0)
+                for (uint32_t w = threadIdx.x; w < nbw; w += NT) {
+                    uint32_t v = 0;
+                    for (uint32_t i = w * 32; i < n && i < w * 32 + 32; ++i)
+                        v |= (uint32_t)s_mask(C, g0 + i) << (i % 32);
+                    o[w] = v;
+                }
+        } else if (KIND == 1) {
+            if (threadIdx.x == 0) o[0] = m;
+        } else {
+            at = 1 + dict_words(m, dDb[d - 1]);
+        }
+        do_init(dout, dDb[d], sm, reinterpret_cast<uint16_t*>(sm + DICT_MAX), gd, o + at,
+                sm + DICT_MAX + LUTN / 2, m);
     } else {
-        hs_clear(hv);
-        hs_clear(hl);
+        vs_clear(h);
     }
     __syncthreads();
-    uint32_t R0 = 0, pend_s = 0, pend_v = 0;          // runs started so far; the open run
-    for (uint32_t c0 = 0; c0 < bk.n; c0 += CH) {
+    uint32_t R0 = 0, pend_s = 0, mine = 0;
+    for (uint32_t c0 = 0; c0 < n; c0 += CH) {
         uint32_t fl[IT], v[IT], cnt = 0;
         const uint32_t s0 = c0 + threadIdx.x * IT;
-        uint32_t prev = s0 > 0 && s0 < bk.n ? colv(C, c, bk.g0 + s0 - 1) : 0;
+        const uint32_t left = s0 < n ? n - s0 : 0;
+        ld4(col, g0 + s0, vec, left, v);
+        if (KIND == 0) {
+            uint32_t a[IT], b[IT], e[IT];
+            ld4(C.u8[C_AVGQ2], g0 + s0, vec, left, a);
+            ld4(C.u16[C_CU2 - 8], g0 + s0, vec, left, b);
+            ld4(C.u16[C_CA2 - 8], g0 + s0, vec, left, e);
 #pragma unroll
-        for (int u = 0; u < IT; ++u) {
-            const uint32_t s = s0 + u;
-            fl[u] = 0;
-            if (s >= bk.n) continue;
-            v[u] = colv(C, c, bk.g0 + s);
-            fl[u] = s == 0 || v[u] != prev;
-            prev = v[u];
-            cnt += fl[u];
+            for (int u = 0; u < IT; ++u) {
+                fl[u] = (a[u] | b[u] | e[u]) != 0;
+                cnt += fl[u];
+            }
+        } else {
+            uint32_t prev = s0 > 0 && s0 < n ? (uint32_t)col[g0 + s0 - 1] : 0;
+#pragma unroll
+            for (int u = 0; u < IT; ++u) {
+                fl[u] = (uint32_t)u < left && (s0 + u == 0 || v[u] != prev);
+                prev = v[u];
+                cnt += fl[u];
+            }
+        }
+        if (KIND < 2 && !WRITE) {                       // no order needed: insert, count
+#pragma unroll
+            for (int u = 0; u < IT; ++u)
+                if (fl[u]) vs_insert(h, v[u]);
+            mine += cnt;
+            continue;
         }
         uint32_t k;
         uint32_t r = cta_scan(cnt, S, &k);
+        if (KIND < 2) {                                 // write: element R0 + r is this value
 #pragma unroll
-        for (int u = 0; u < IT; ++u)
-            if (fl[u]) { starts[r] = s0 + u; startv[r] = v[u]; ++r; }
+            for (int u = 0; u < IT; ++u)
+                if (fl[u]) do_add(dout, R0 + r++, v[u]);
+            R0 += k;
+            __syncthreads();
+            if (dout.D != RAW) pk_flush(dout.pk, R0);
+            continue;
+        }
+#pragma unroll
+        for (int u = 0; u < IT; ++u)                    // lengths: run R0+e-1 ends at starts[e]
+            if (fl[u]) starts[r++] = s0 + u;
         __syncthreads();
-        // run R0+e-1 ends at starts[e]
         for (uint32_t e = threadIdx.x; e < k; e += NT) {
             if (R0 + e == 0) continue;
-            const uint32_t rs = e == 0 ? pend_s : starts[e - 1];
-            const uint32_t rv = e == 0 ? pend_v : startv[e - 1];
-            const uint32_t len = starts[e] - rs;
-            if (WRITE) {
-                do_add(dv, R0 + e - 1, rv);
-                do_add(dl, R0 + e - 1, len);
-            } else {
-                hs_insert(hv, rv);
-                hs_insert(hl, len);
-            }
+            const uint32_t len = starts[e] - (e == 0 ? pend_s : starts[e - 1]);
+            if (WRITE) do_add(dout, R0 + e - 1, len);
+            else vs_insert(h, len);
         }
         __syncthreads();
-        if (k) { pend_s = starts[k - 1]; pend_v = startv[k - 1]; }
+        if (k) pend_s = starts[k - 1];
         R0 += k;
-        if (WRITE) {
-            if (dv.D != RAW) pk_flush(dv.pk, R0 - 1);
-            if (dl.D != RAW) pk_flush(dl.pk, R0 - 1);
-        }
+        if (WRITE && dout.D != RAW) pk_flush(dout.pk, R0 - 1);
         __syncthreads();
     }
-    // the last run ends at the block end
-    if (threadIdx.x == 0) {
-        if (WRITE) {
-            do_add(dv, R0 - 1, pend_v);
-            do_add(dl, R0 - 1, bk.n - pend_s);
-        } else {
-            hs_insert(hv, pend_v);
-            hs_insert(hl, bk.n - pend_s);
-        }
+    if (KIND == 2 && threadIdx.x == 0) {                // the last run ends at the block end
+        if (WRITE) do_add(dout, R0 - 1, n - pend_s);
+        else vs_insert(h, n - pend_s);
     }
     __syncthreads();
     if (WRITE) {
-        if (dv.D != RAW) { pk_flush(dv.pk, R); pk_final(dv.pk, R); }
-        if (dl.D != RAW) { pk_flush(dl.pk, R); pk_final(dl.pk, R); }
-    } else {
-        const uint32_t DV = hs_finalize(hv, sb, gd, S);
-        const uint32_t DL = hs_finalize(hl, sb, gd + A.DC, S);
-        if (threadIdx.x == 0) {
-            dD[0] = DV;
-            dD[1] = DL;
-            meta[0] = (uint32_t)(1 + dict_words(R0, DV) + dict_words(R0, DL));
-            meta[1] = R0;
-        }
+        const uint32_t m = meta[1];
+        if (dout.D != RAW) { pk_flush(dout.pk, m); pk_final(dout.pk, m); }
+        return;
+    }
+    if (KIND < 2) cta_scan(mine, S, &R0);
+    const uint32_t D = vs_finalize(h, sm + HS + 2, gd, S);
+    if (threadIdx.x == 0) {
+        A.dD[(size_t)blk * NDICT + d] = D;
+        if (d == 0 || KIND == 1) meta[1] = R0;
     }
 }
 
-// grid nblk * nsec: sections [sec0, sec0 + nsec) of every block (the exception-list sections and
-// the dictionary sections are launched apart, each with the shared memory it needs, so the light
-// ones run four CTAs per SM); WRITE = false sizes the sections, true writes them
 template <bool WRITE>
-__global__ void __launch_bounds__(NT) k_cz_sections(CzArgs A, int sec0, int nsec) {
+__global__ void __launch_bounds__(NT, WRITE ? GSNP_CZ_MINB_W : GSNP_CZ_MINB) k_cz_dicts(CzArgs A) {
+    extern __shared__ __align__(16) uint32_t sm[];
+    __shared__ Smem S;
+    const int d = (int)(blockIdx.x % NDICT);
+    const uint32_t blk = blockIdx.x / NDICT;
+    const uint64_t g0 = (uint64_t)blk * A.B;
+    const uint32_t n = (uint32_t)(A.n - g0 < A.B ? A.n - g0 : A.B);
+    const Cols& C = A.col;
+    switch (d) {
+    case 0: dict_body<WRITE, 0>(A, C.u8[C_AVGQ2], d, blk, g0, n, sm, S); break;
+    case 1: dict_body<WRITE, 0>(A, C.u16[C_CU2 - 8], d, blk, g0, n, sm, S); break;
+    case 2: dict_body<WRITE, 0>(A, C.u16[C_CA2 - 8], d, blk, g0, n, sm, S); break;
+    default: {
+        const int ci = (d - 3) / 2, c = rle_col(ci);
+        const bool len = (d - 3) & 1;
+        if (c < 8) {
+            if (len) dict_body<WRITE, 2>(A, C.u8[c], d, blk, g0, n, sm, S);
+            else dict_body<WRITE, 1>(A, C.u8[c], d, blk, g0, n, sm, S);
+        } else if (c < 12) {
+            if (len) dict_body<WRITE, 2>(A, C.u16[c - 8], d, blk, g0, n, sm, S);
+            else dict_body<WRITE, 1>(A, C.u16[c - 8], d, blk, g0, n, sm, S);
+        } else {
+            if (len) dict_body<WRITE, 2>(A, C.u32[c - 12], d, blk, g0, n, sm, S);
+            else dict_body<WRITE, 1>(A, C.u32[c - 12], d, blk, g0, n, sm, S);
+        }
+    }
+    }
+}
+
+// grid nblk * nsec: sections [sec0, sec0 + nsec) < SEC_S of every block (header, planes,
+// exception lists; the dictionary sections are k_cz_dicts); WRITE = false sizes the sections, true
+// writes them
+template <bool WRITE>
+__global__ void __launch_bounds__(NT, GSNP_CZ_MINB) k_cz_sections(CzArgs A, int sec0, int nsec) {
     extern __shared__ __align__(16) uint32_t sm[];
     __shared__ Smem S;
     const int sec = sec0 + (int)(blockIdx.x % nsec);    // a block's sections are adjacent in
@@ -583,19 +642,34 @@ __global__ void __launch_bounds__(NT) k_cz_sections(CzArgs A, int sec0, int nsec
         }
         return;
     }
-    if (sec < SEC_S) sec_exceptions<WRITE>(A, bk, sec, S, sm);
-    else if (sec == SEC_S) sec_second<WRITE>(A, bk, S, sm);
-    else sec_rle<WRITE>(A, bk, sec - SEC_C, S, sm);
+    sec_exceptions<WRITE>(A, bk, sec, S, sm);
+}
+
+// words of section sec of block blk: the light sections' size pass stored them in meta[0]; the
+// dictionary sections' come from the element counts and dictionary sizes (k_cz_dicts)
+__device__ __forceinline__ uint64_t section_words(const CzArgs& A, uint32_t blk, int sec) {
+    const uint32_t* meta = A.meta + ((size_t)blk * NSEC + sec) * 2;
+    if (sec < SEC_S) return meta[0];
+    const uint32_t* dDb = A.dD + (size_t)blk * NDICT;
+    const uint32_t m = meta[1];
+    if (sec == SEC_S) {
+        const uint64_t g0 = (uint64_t)blk * A.B;
+        const uint32_t n = (uint32_t)(A.n - g0 < A.B ? A.n - g0 : A.B);
+        return (n + 31) / 32 + dict_words(m, dDb[0]) + dict_words(m, dDb[1]) + dict_words(m, dDb[2]);
+    }
+    const int d = 3 + 2 * (sec - SEC_C);
+    return 1 + dict_words(m, dDb[d]) + dict_words(m, dDb[d + 1]);
 }
 
 // exclusive scan of the section sizes (block-major, section-minor = stream order)
-__global__ void __launch_bounds__(1024) k_cz_scan(const uint32_t* meta, uint64_t nsec, uint64_t* off) {
+__global__ void __launch_bounds__(1024) k_cz_scan(const CzArgs A, uint64_t* off) {
+    const uint64_t nsec = (uint64_t)A.nblk * NSEC;
     __shared__ uint64_t ws[33];
     uint64_t carry = 0;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     for (uint64_t c0 = 0; c0 < nsec; c0 += 1024) {
         const uint64_t i = c0 + threadIdx.x;
-        const uint64_t v = i < nsec ? meta[i * 2] : 0;
+        const uint64_t v = i < nsec ? section_words(A, (uint32_t)(i / NSEC), (int)(i % NSEC)) : 0;
         uint64_t x = v;
         for (int d = 1; d < 32; d <<= 1) {
             uint64_t y = __shfl_up_sync(0xFFFFFFFFu, x, d);
@@ -620,13 +694,9 @@ __global__ void __launch_bounds__(1024) k_cz_scan(const uint32_t* meta, uint64_t
     if (threadIdx.x == 0) off[nsec] = carry;
 }
 
-// dynamic shared memory of k_cz_sections (words): the RLE section is the largest user; the
-// header, plane and exception sections need only the packer's staging window
+// dynamic shared memory of k_cz_sections (words): the header, plane and exception sections need
+// only the packer's staging window
 constexpr size_t SMEM_LIGHT_WORDS = PKW;
-constexpr size_t SMEM_SIZE_WORDS = 2 * CH + 2 * HS + 4 + DICT_MAX;
-constexpr size_t SMEM_WRITE_WORDS = 2 * CH + 2 * DICT_MAX + 2 * PKW;
-static_assert(HS + 2 + DICT_MAX <= SMEM_SIZE_WORDS, "S section (size pass) fits");
-static_assert(DICT_MAX + PKW <= SMEM_WRITE_WORDS, "S section (write pass) fits");
 static_assert(PKW * 32 >= (CH + 1) * 12 + 64, "packer window");
 
 }  // namespace gsnp_cz
