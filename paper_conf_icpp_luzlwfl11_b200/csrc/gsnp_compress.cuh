@@ -315,101 +315,6 @@ struct BlockCtx {
     uint32_t blk;             // block number
 };
 
-// exception-list sections N / G / K / R / Q
-template <bool WRITE>
-__device__ void sec_exceptions(const CzArgs& A, const BlockCtx& bk, int sec, Smem& S,
-                               uint32_t* st) {
-    const Cols& C = A.col;
-    const uint32_t blk = bk.blk;
-    uint32_t* meta = A.meta + ((size_t)blk * NSEC + sec) * 2;
-    const uint32_t m = WRITE ? meta[1] : 0;
-    uint32_t* o = WRITE ? A.out + A.off[(size_t)blk * NSEC + sec] : nullptr;
-    const int ncol = sec == SEC_N ? C_REF : sec == SEC_N + 1 ? C_BASE1 : C_BASE2;   // N: base column
-    Packer pk;
-    if (WRITE && (sec == SEC_G || sec == SEC_K)) pk_init(pk, st, o + 1 + m, 8);
-    if (WRITE && threadIdx.x == 0) o[0] = m;
-    uint32_t run = 0, runE = 0;                              // exceptions (N: run starts, ends)
-                                                             // before this chunk
-    for (uint32_t c0 = 0; c0 < bk.n; c0 += CH) {
-        uint32_t fl[IT], vals[IT], cnt = 0;
-#pragma unroll
-        for (int u = 0; u < IT; ++u) {
-            const uint32_t s = c0 + threadIdx.x * IT + u;
-            fl[u] = 0;
-            vals[u] = 0;
-            if (s >= bk.n) continue;
-            const uint64_t gi = bk.g0 + s;
-            if (sec <= SEC_N + 2) {                          // runs of code 4: start (lo16), end (hi16)
-                const bool f = C.u8[ncol][gi] == 4;
-                const bool pf = s > 0 && C.u8[ncol][gi - 1] == 4;
-                const bool nf = s + 1 < bk.n && C.u8[ncol][gi + 1] == 4;
-                fl[u] = (f && !pf ? 1u : 0u) | (f && !nf ? 0x10000u : 0u);
-            } else if (sec == SEC_G) {
-                const uint32_t r = C.u8[C_REF][gi];
-                const uint32_t pred = r < 4 ? (0x09070400u >> (8 * r)) & 255 : 255;   // HOM[ref]
-                vals[u] = C.u8[C_GENO][gi];
-                fl[u] = vals[u] != pred;
-            } else if (sec == SEC_K) {
-                vals[u] = C.u8[C_KNOWN][gi];
-                fl[u] = vals[u] != 0;
-            } else {
-                vals[u] = C.u32[sec == SEC_R ? C_RANKP - 12 : C_POST1 - 12][gi];
-                fl[u] = vals[u] != ONE;
-            }
-            cnt += fl[u];
-        }
-        uint32_t tot;
-        uint32_t r = cta_scan(cnt, S, &tot);
-        if (WRITE) {
-            if (sec <= SEC_N + 2) {
-                uint32_t rs = run + (r & 0xFFFF), re = runE + (r >> 16);
-#pragma unroll
-                for (int u = 0; u < IT; ++u) {
-                    const uint32_t s = c0 + threadIdx.x * IT + u;
-                    if (fl[u] & 1) o[1 + rs++] = s;
-                    if (fl[u] >> 16) o[1 + m + re++] = s + 1;
-                }
-            } else {
-                uint32_t j = run + r;
-#pragma unroll
-                for (int u = 0; u < IT; ++u) {
-                    if (!fl[u]) continue;
-                    const uint32_t s = c0 + threadIdx.x * IT + u;
-                    o[1 + j] = s;
-                    if (sec == SEC_G || sec == SEC_K) pk_add(pk, j, vals[u]);
-                    else o[1 + m + j] = vals[u];
-                    ++j;
-                }
-            }
-        }
-        run += sec <= SEC_N + 2 ? (tot & 0xFFFF) : tot;
-        runE += tot >> 16;
-        if (WRITE && (sec == SEC_G || sec == SEC_K)) {
-            __syncthreads();
-            pk_flush(pk, run);
-        }
-    }
-    if (WRITE) {
-        if (sec == SEC_G || sec == SEC_K) pk_final(pk, m);
-    } else if (threadIdx.x == 0) {
-        uint64_t words = sec <= SEC_N + 2 || sec == SEC_R || sec == SEC_Q ? 1 + 2ull * run
-                                                                           : 1 + run + (run + 3) / 4;
-        meta[0] = (uint32_t)words;
-        meta[1] = run;
-    }
-}
-
-// second-allele section S (P:L756-758): bitmap of sites with a non-zero second allele, then
-// DICT of avgq2, cnt_uni2, cnt_all2 over those sites in order
-__device__ __forceinline__ bool s_mask(const Cols& C, uint64_t gi) {
-    return (C.u8[C_AVGQ2][gi] | C.u16[C_CU2 - 8][gi] | C.u16[C_CA2 - 8][gi]) != 0;
-}
-
-__device__ __forceinline__ int rle_col(int ci) {
-    return ci == 0 ? C_QUAL : ci == 1 ? C_AVGQ1 : ci == 2 ? C_CU1 : ci == 3 ? C_CA1
-         : ci == 4 ? C_DEPTH : C_COPYN;
-}
-
 // IT (= 4) consecutive elements of a column from element i (n_left of them valid, the rest 0);
 // vec: the column and i are aligned for one vector load
 static_assert(IT == 4, "vector loads take four elements");
@@ -432,6 +337,116 @@ __device__ __forceinline__ void ld4(const T* col, uint64_t i, bool vec, uint32_t
     }
 #pragma unroll
     for (int u = 0; u < 4; ++u) v[u] = (uint32_t)u < n_left ? (uint32_t)col[i + u] : 0u;
+}
+
+// exception-list sections N / G / K / R / Q.  The size pass only counts (one
+// reduction at the end); the write pass orders the exceptions with a CTA scan per chunk.
+template <bool WRITE>
+__device__ void sec_exceptions(const CzArgs& A, const BlockCtx& bk, int sec, Smem& S,
+                               uint32_t* st) {
+    const Cols& C = A.col;
+    const uint32_t blk = bk.blk;
+    uint32_t* meta = A.meta + ((size_t)blk * NSEC + sec) * 2;
+    const uint32_t m = WRITE ? meta[1] : 0;
+    uint32_t* o = WRITE ? A.out + A.off[(size_t)blk * NSEC + sec] : nullptr;
+    const bool nsec = sec <= SEC_N + 2;
+    const uint8_t* ncol = C.u8[sec == SEC_N ? C_REF : sec == SEC_N + 1 ? C_BASE1 : C_BASE2];
+    const bool vec = (bk.g0 & 3) == 0;
+    Packer pk;
+    if (WRITE && (sec == SEC_G || sec == SEC_K)) pk_init(pk, st, o + 1 + m, 8);
+    if (WRITE && threadIdx.x == 0) o[0] = m;
+    uint32_t run = 0, runE = 0, mine = 0;                    // exceptions (N: run starts, ends)
+                                                             // before this chunk
+    for (uint32_t c0 = 0; c0 < bk.n; c0 += CH) {
+        uint32_t fl[IT], vals[IT], cnt = 0;
+        const uint32_t s0 = c0 + threadIdx.x * IT;
+        const uint32_t left = s0 < bk.n ? bk.n - s0 : 0;
+        const uint64_t gi = bk.g0 + s0;
+        if (nsec) {                                          // runs of code 4: start (lo16), end (hi16)
+            uint32_t x[IT];
+            ld4(ncol, gi, vec, left, x);
+            bool pf = s0 > 0 && left && ncol[gi - 1] == 4;
+            const bool last_nf = left > 4 && ncol[gi + 4] == 4;
+#pragma unroll
+            for (int u = 0; u < IT; ++u) {
+                const bool f = (uint32_t)u < left && x[u] == 4;
+                const bool nf = u + 1 < IT ? ((uint32_t)(u + 1) < left && x[u + 1] == 4) : last_nf;
+                fl[u] = (f && !pf ? 1u : 0u) | (f && !nf ? 0x10000u : 0u);
+                pf = f;
+                vals[u] = 0;
+            }
+        } else if (sec == SEC_G) {
+            uint32_t r[IT];
+            ld4(C.u8[C_REF], gi, vec, left, r);
+            ld4(C.u8[C_GENO], gi, vec, left, vals);
+#pragma unroll
+            for (int u = 0; u < IT; ++u) {
+                const uint32_t pred = r[u] < 4 ? (0x09070400u >> (8 * r[u])) & 255 : 255;   // HOM[ref]
+                fl[u] = (uint32_t)u < left && vals[u] != pred;
+            }
+        } else if (sec == SEC_K) {
+            ld4(C.u8[C_KNOWN], gi, vec, left, vals);
+#pragma unroll
+            for (int u = 0; u < IT; ++u) fl[u] = vals[u] != 0;
+        } else {
+            ld4(C.u32[sec == SEC_R ? C_RANKP - 12 : C_POST1 - 12], gi, vec, left, vals);
+#pragma unroll
+            for (int u = 0; u < IT; ++u) fl[u] = (uint32_t)u < left && vals[u] != ONE;
+        }
+#pragma unroll
+        for (int u = 0; u < IT; ++u) cnt += fl[u];
+        if (!WRITE) {
+            mine += nsec ? (cnt & 0xFFFF) : cnt;
+            continue;
+        }
+        uint32_t tot;
+        uint32_t r = cta_scan(cnt, S, &tot);
+        if (nsec) {
+            uint32_t rs = run + (r & 0xFFFF), re = runE + (r >> 16);
+#pragma unroll
+            for (int u = 0; u < IT; ++u) {
+                if (fl[u] & 1) o[1 + rs++] = s0 + u;
+                if (fl[u] >> 16) o[1 + m + re++] = s0 + u + 1;
+            }
+        } else {
+            uint32_t j = run + r;
+#pragma unroll
+            for (int u = 0; u < IT; ++u) {
+                if (!fl[u]) continue;
+                o[1 + j] = s0 + u;
+                if (sec == SEC_G || sec == SEC_K) pk_add(pk, j, vals[u]);
+                else o[1 + m + j] = vals[u];
+                ++j;
+            }
+        }
+        run += nsec ? (tot & 0xFFFF) : tot;
+        runE += tot >> 16;
+        if (sec == SEC_G || sec == SEC_K) {
+            __syncthreads();
+            pk_flush(pk, run);
+        }
+    }
+    if (WRITE) {
+        if (sec == SEC_G || sec == SEC_K) pk_final(pk, m);
+        return;
+    }
+    cta_scan(mine, S, &run);
+    if (threadIdx.x == 0) {
+        uint64_t words = nsec || sec == SEC_R || sec == SEC_Q ? 1 + 2ull * run : 1 + run + (run + 3) / 4;
+        meta[0] = (uint32_t)words;
+        meta[1] = run;
+    }
+}
+
+// second-allele section S (P:L756-758): bitmap of sites with a non-zero second allele, then
+// DICT of avgq2, cnt_uni2, cnt_all2 over those sites in order
+__device__ __forceinline__ bool s_mask(const Cols& C, uint64_t gi) {
+    return (C.u8[C_AVGQ2][gi] | C.u16[C_CU2 - 8][gi] | C.u16[C_CA2 - 8][gi]) != 0;
+}
+
+__device__ __forceinline__ int rle_col(int ci) {
+    return ci == 0 ? C_QUAL : ci == 1 ? C_AVGQ1 : ci == 2 ? C_CU1 : ci == 3 ? C_CA1
+         : ci == 4 ? C_DEPTH : C_COPYN;
 }
 
 // One dictionary of one block per CTA (grid nblk x NDICT; dictionary d in dD order): d 0..2 the
@@ -472,8 +487,22 @@ __device__ __forceinline__ void dict_body(const CzArgs& A, const T* col, int d, 
             if (d == 0)
                 for (uint32_t w = threadIdx.x; w < nbw; w += NT) {
                     uint32_t v = 0;
-                    for (uint32_t i = w * 32; i < n && i < w * 32 + 32; ++i)
-                        v |= (uint32_t)s_mask(C, g0 + i) << (i % 32);
+                    if (vec && w * 32 + 32 <= n) {              // eight four-element loads each
+#pragma unroll
+                        for (int q = 0; q < 8; ++q) {
+                            uint32_t a[IT], b[IT], e[IT];
+                            const uint64_t i = g0 + w * 32 + 4 * q;
+                            ld4(C.u8[C_AVGQ2], i, true, 4, a);
+                            ld4(C.u16[C_CU2 - 8], i, true, 4, b);
+                            ld4(C.u16[C_CA2 - 8], i, true, 4, e);
+#pragma unroll
+                            for (int u = 0; u < IT; ++u)
+                                v |= (uint32_t)((a[u] | b[u] | e[u]) != 0) << (4 * q + u);
+                        }
+                    } else {
+                        for (uint32_t i = w * 32; i < n && i < w * 32 + 32; ++i)
+                            v |= (uint32_t)s_mask(C, g0 + i) << (i % 32);
+                    }
                     o[w] = v;
                 }
         } else if (KIND == 1) {
@@ -636,8 +665,18 @@ __global__ void __launch_bounds__(NT, GSNP_CZ_MINB) k_cz_sections(CzArgs A, int 
             const int c = t < pw ? C_REF : t < 2 * pw ? C_BASE1 : C_BASE2;
             const uint32_t w = t % pw;
             uint32_t v = 0;
-            for (uint32_t i = w * 16; i < bk.n && i < w * 16 + 16; ++i)
-                v |= (A.col.u8[c][bk.g0 + i] & 3u) << (2 * (i % 16));
+            const uint8_t* col = A.col.u8[c] + bk.g0 + w * 16;
+            if ((bk.g0 & 15) == 0 && w * 16 + 16 <= bk.n) {      // one 16-byte load
+                const uint4 q = *reinterpret_cast<const uint4*>(col);
+                const uint32_t qw[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+                for (int k = 0; k < 4; ++k)
+#pragma unroll
+                    for (int b = 0; b < 4; ++b) v |= ((qw[k] >> (8 * b)) & 3u) << (2 * (4 * k + b));
+            } else {
+                for (uint32_t i = w * 16; i < bk.n && i < w * 16 + 16; ++i)
+                    v |= (col[i - w * 16] & 3u) << (2 * (i % 16));
+            }
             o[t] = v;
         }
         return;
