@@ -696,7 +696,7 @@ gsnp_status finalize_impl(gsnp_ctx* ctx, const uint64_t* counts_host) {
     auto t0 = std::chrono::steady_clock::now();
     const int L = (int)ctx->prm.max_read_len;
     const int qmax = (int)ctx->prm.q_max;
-    ctx->h_counts.assign(counts_host, counts_host + 64 * 256 * 16);
+    if (ctx->h_counts.size() != (size_t)64 * 256 * 16) ctx->h_counts.assign((size_t)64 * 256 * 16, 0);
     if (ctx->h_p.size() != (size_t)64 * 256 * 16) ctx->h_p.assign((size_t)64 * 256 * 16, 0.0);
     const size_t tn = (size_t)64 * L * 4 * TROW;
     if (!ctx->h_T || ctx->h_T_n != tn) {
@@ -719,6 +719,8 @@ gsnp_status finalize_impl(gsnp_ctx* ctx, const uint64_t* counts_host) {
     std::atomic<int> next_p{0}, done_p{0}, next_t{0};
     auto work = [&]() {
         for (int q; (q = next_p.fetch_add(1)) < 64;) {
+            // this quality's counts into the context's copy (rows copied in parallel)
+            memcpy(ctx->h_counts.data() + ((size_t)q << 12), counts_host + ((size_t)q << 12), 4096 * 8);
             estimate_p_q(prm, C, p, q);
             done_p.fetch_add(1);
         }
@@ -739,8 +741,9 @@ gsnp_status finalize_impl(gsnp_ctx* ctx, const uint64_t* counts_host) {
         ctx->T_zeroed = true;
     }
     const size_t tq = (size_t)(qmax + 1) * L * 4 * TROW;  // rows q = 0..q_max (the built ones)
+    // no host wait: the calls that read T are queued behind the copy on the same stream, and h_T is
+    // rewritten only by the next finalize, after the next count's synchronising read-back
     CK(cudaMemcpyAsync(ctx->T.p, ctx->h_T, tq * 8, cudaMemcpyHostToDevice, ctx->stream));
-    CK(cudaStreamSynchronize(ctx->stream));
     ctx->calibrated = true;
     if (ctx->timing()) {
         ctx->stage_ms[GSNP_STAGE_FINALIZE] +=
@@ -978,9 +981,15 @@ gsnp_status gsnp_calibrate_finalize(gsnp_ctx* ctx, const uint64_t* counts) {
     if (!ctx || !counts) return GSNP_E_INVAL;
     if (cudaSetDevice(ctx->prm.device) != cudaSuccess) return fail(ctx, GSNP_E_CUDA, "set device");
     if (is_device_ptr(counts)) {
-        if (!ctx->h_cnt_pinned) CK(cudaMallocHost(&ctx->h_cnt_pinned, 64 * 256 * 16 * 8));
-        CK(cudaMemcpyAsync(ctx->h_cnt_pinned, counts, 64 * 256 * 16 * 8, cudaMemcpyDeviceToHost,
-                           ctx->stream));
+        if (!ctx->h_cnt_pinned) {
+            CK(cudaMallocHost(&ctx->h_cnt_pinned, 64 * 256 * 16 * 8));
+            memset(ctx->h_cnt_pinned, 0, 64 * 256 * 16 * 8);
+        }
+        // only the cells a count can reach (q <= q_max, cycle < max_read_len): k_calib_count rejects
+        // the other qualities and never forms a later cycle, so the rest stays zero
+        CK(cudaMemcpy2DAsync(ctx->h_cnt_pinned, 4096 * 8, counts, 4096 * 8,
+                             (size_t)ctx->prm.max_read_len * 16 * 8, (size_t)ctx->prm.q_max + 1,
+                             cudaMemcpyDeviceToHost, ctx->stream));
         CK(cudaStreamSynchronize(ctx->stream));
         return finalize_impl(ctx, ctx->h_cnt_pinned);
     }

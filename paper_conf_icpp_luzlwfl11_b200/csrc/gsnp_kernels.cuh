@@ -352,7 +352,11 @@ __global__ void __launch_bounds__(CAL_NT, 1) k_calib_count(const __grid_constant
             m_flat[sidx][tid] = keep ? (uint32_t)(m.p - A.origin - r0) | m.st << 31 : 0xFFFFFFFFu;
         // (flat mode needs Lb >= 2: its read index is a multiply-high by ceil(2^32 / Lb), which
         // wraps to 0 at Lb == 1 — batches of 1-bp reads take the staged path)
+#ifdef GSNP_CAL_NOFLAT
+        const bool uni = false;
+#else
         const bool uni = m.l0 >= 2 && (!m.in || (m.l == m.l0 && m.o - m.ob0 == (uint64_t)tid * m.l0));
+#endif
         const int all_uni = __syncthreads_and(uni);
         if (tid == 0) {
             m_fl[sidx][0] = all_uni; m_fl[sidx][1] = m.nall; m_fl[sidx][2] = m.l0;
