@@ -250,6 +250,10 @@ constexpr int CAL_MAXB = 512;         // max reads per batch (metadata arrays)
 __device__ __forceinline__ void red_shared_add(uint32_t* p, uint32_t v) {
     asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
 }
+// shared add at a shared-window byte address
+__device__ __forceinline__ void red_shared_add_at(uint32_t saddr, uint32_t v) {
+    asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(saddr), "r"(v) : "memory");
+}
 // predicated shared increment (no branch around it)
 __device__ __forceinline__ void red_shared_inc_if(uint32_t saddr, uint32_t pred) {
     asm volatile("{\n .reg .pred p;\n setp.ne.u32 p, %1, 0;\n @p red.shared.add.u32 [%0], 1;\n}"
@@ -424,17 +428,18 @@ __global__ void __launch_bounds__(CAL_NT, 1) k_calib_count(const __grid_constant
             const uint32_t* sw = reinterpret_cast<const uint32_t*>(sb);
             const uint32_t w_lo = xb >> 2, w_hi = (xb + nb + 3) >> 2;
             const uint32_t qlim = (qmax + 1) * 0x01010101u;
+            const uint32_t L4 = 4u * (uint32_t)Lh, sbw = A.SB >> 2;
             for (uint32_t w = w_lo + tid; w < w_hi; w += CAL_NT) {
                 const int64_t x0 = (int64_t)(4 * w) - (int64_t)xb;
                 const uint32_t xc = x0 > 0 ? (uint32_t)x0 : 0u;
                 const uint32_t j = __umulhi(xc, magic), i0 = xc - j * Lb;
-                if (x0 < 0 || x0 + 4 > (int64_t)nb || i0 + 4 > Lb) {    // edge / read boundary
+                if (x0 < 0 || x0 + 4 > (int64_t)nb || i0 + 4 > Lb || Lh != L) {   // edge / read boundary
                     for (int u = 0; u < 4; ++u) one(x0 + u);
                     continue;
                 }
                 const uint32_t fd = mf[j];
                 if (fd == 0xFFFFFFFFu) continue;                        // not a counted read
-                const uint32_t bw = sw[w], qw = sw[(A.SB >> 2) + w];
+                const uint32_t bw = sw[w], qw = sw[sbw + w];
                 const uint32_t ro = (fd & 0xFFFFu) + i0;
                 const uint32_t* rw2 = reinterpret_cast<const uint32_t*>(rr + (ro & ~3u));
                 const uint32_t rw = __funnelshift_r(rw2[0], rw2[1], (ro & 3u) * 8);
@@ -451,23 +456,20 @@ __global__ void __launch_bounds__(CAL_NT, 1) k_calib_count(const __grid_constant
                 const uint32_t qt = ((qw & 0x3F3F3F3Fu) << 2) | (rw & 0x03030303u);
                 const bool minus = (fd >> 31) != 0;
                 const uint32_t c0 = minus ? Lb - 1 - i0 : i0;
-                if (Lh == L) {
-                    const int dir = minus ? -1 : 1;
-#pragma unroll
-                    for (int u = 0; u < 4; ++u)
-                        red_shared_inc_if(hbase + 4u * (((qt >> (8 * u)) & 255u) * (uint32_t)Lh +
-                                                        (uint32_t)((int)c0 + u * dir)),
-                                          diag & (0x80u << (8 * u)));
-                    uint32_t mis = used & ~diag;                      // ~2% of bases: global
-                    while (mis) {
-                        const int u = (__ffs(mis) - 1) >> 3;
-                        mis &= mis - 1;
-                        const uint32_t cyc = minus ? c0 - u : c0 + u;
-                        atomicAdd(&A.C[((qw >> (8 * u)) & 63u) << 12 | cyc << 4 |
-                                       ((rw >> (8 * u)) & 3u) << 2 | ((bw >> (8 * u)) & 3u)], 1ull);
-                    }
-                } else {
-                    for (int u = 0; u < 4; ++u) one(x0 + u);
+                // byte u -> hist[qt_u][c0 +- u]: one unconditional shared add of 0 or 1 per byte
+                // (no branch, no warp aggregation)
+                const uint32_t a0 = hbase + 4u * c0, st = minus ? 0xFFFFFFFCu : 4u;
+                red_shared_add_at(__byte_perm(qt, 0, 0x4440) * L4 + a0, (diag >> 7) & 1u);
+                red_shared_add_at(__byte_perm(qt, 0, 0x4441) * L4 + a0 + st, (diag >> 15) & 1u);
+                red_shared_add_at(__byte_perm(qt, 0, 0x4442) * L4 + a0 + 2u * st, (diag >> 23) & 1u);
+                red_shared_add_at(__byte_perm(qt, 0, 0x4443) * L4 + a0 + 3u * st, diag >> 31);
+                uint32_t mis = used & ~diag;                          // ~2% of bases: global
+                while (mis) {
+                    const int u = (__ffs(mis) - 1) >> 3;
+                    mis &= mis - 1;
+                    const uint32_t cyc = minus ? c0 - u : c0 + u;
+                    atomicAdd(&A.C[((qw >> (8 * u)) & 63u) << 12 | cyc << 4 |
+                                   ((rw >> (8 * u)) & 3u) << 2 | ((bw >> (8 * u)) & 3u)], 1ull);
                 }
             }
             err |= (eb || ebw ? ERR_RANGE : 0) | (eq || eqw ? ERR_QUAL : 0);
