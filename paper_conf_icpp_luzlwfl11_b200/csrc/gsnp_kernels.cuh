@@ -709,6 +709,32 @@ __device__ __forceinline__ int64_t site_ref(const CallArgs& A, uint64_t site, in
     return (int64_t)lower_bound_u64(A.known_pos, 0, A.n_known, site);
 }
 
+// C8 p-value from the rank-sum pieces (het calls only: kept out of line, away from the hot path's
+// instruction stream).  n1, n2: unique keys of allele 1 / 2; wsum, tie: see thread_finish_tail.
+#ifndef GSNP_PIECES_INLINE
+#define GSNP_PIECES_INLINE 1   // A/B: inline 10.75 ms vs out of line 11.24 at C2 (layout)
+#endif
+#ifndef GSNP_COLD_INLINE
+__device__ __noinline__
+#else
+__device__ __forceinline__
+#endif
+double rank_sum_p(const CallArgs& A, uint32_t n1, uint32_t n2, double wsum, double tie) {
+    if (n1 == 0 || n2 == 0) return 0.0;
+    double n1d = (double)n1, n2d = (double)n2, Nd = (double)(n1 + n2);
+    double mu = n1d * (Nd + 1.0) / 2.0;
+    double var = n1d * n2d / 12.0 * ((Nd + 1.0) - tie / (Nd * (Nd - 1.0)));
+    if (A.rank_cdf && tie == 0.0 && n1 <= GSNP_RANK_EXACT_MAX && n2 <= GSNP_RANK_EXACT_MAX) {
+        // R20 exact: U = W - n1(n1+1)/2 is an integer when nothing ties
+        const int u = (int)llrint(wsum - n1d * (n1d + 1.0) / 2.0);
+        const double* F = A.rank_cdf + (size_t)(n1 * 33 + n2) * 1025;
+        return fmin(1.0, 2.0 * fmin(F[u], F[(int)(n1 * n2) - u]));
+    }
+    if (!(var > 0.0)) return 1.0;
+    double z = (wsum - mu) / sqrt(var);
+    return erfc(fabs(z) / sqrt(2.0));
+}
+
 // C8/C9 and the 40-byte record (R8, R9).  The 32-slot kernel has one calling path and inlines it
 // (measured 0.8% faster at C2); kernels with several paths share one out-of-line copy
 // (site_record_ool) — their code must stay within the instruction cache.
@@ -726,26 +752,8 @@ __device__ __forceinline__ void site_record(const CallArgs& A, uint64_t site, in
     const uint32_t depth = ca0 + ca1 + ca2 + ca3;
     // C8 rank-sum (normal approximation with tie correction)
     double rank_p = 1.0;
-    if (a1 != a2 && (A.flags & GSNP_RANK_SUM)) {
-        const uint32_t n1 = pick4(cu0, cu1, cu2, cu3, a1), n2 = pick4(cu0, cu1, cu2, cu3, a2);
-        if (n1 == 0 || n2 == 0) rank_p = 0.0;
-        else {
-            double n1d = (double)n1, n2d = (double)n2, Nd = (double)(n1 + n2);
-            double mu = n1d * (Nd + 1.0) / 2.0;
-            double var = n1d * n2d / 12.0 * ((Nd + 1.0) - tie / (Nd * (Nd - 1.0)));
-            if (A.rank_cdf && tie == 0.0 && n1 <= GSNP_RANK_EXACT_MAX &&
-                n2 <= GSNP_RANK_EXACT_MAX) {
-                // R20 exact: U = W - n1(n1+1)/2 is an integer when nothing ties
-                const int u = (int)llrint(wsum - n1d * (n1d + 1.0) / 2.0);
-                const double* F = A.rank_cdf + (size_t)(n1 * 33 + n2) * 1025;
-                rank_p = fmin(1.0, 2.0 * fmin(F[u], F[(int)(n1 * n2) - u]));
-            } else if (!(var > 0.0)) rank_p = 1.0;
-            else {
-                double z = (wsum - mu) / sqrt(var);
-                rank_p = erfc(fabs(z) / sqrt(2.0));
-            }
-        }
-    }
+    if (a1 != a2 && (A.flags & GSNP_RANK_SUM))
+        rank_p = rank_sum_p(A, pick4(cu0, cu1, cu2, cu3, a1), pick4(cu0, cu1, cu2, cu3, a2), wsum, tie);
     // C9 best / second base: rank by q_sum among unique bases (by count_all if none), ties to
     // the lower code.  rank(b) = #{b' present: score(b') > score(b) or (== and b' < b)}.
     const bool uni = dep_uni > 0;
@@ -865,6 +873,37 @@ __device__ __forceinline__ void sort_column(uint32_t* colp, uint32_t n) {
 #define COLKEY(w) ((w) & 0x1FFFFu)
 #endif
 
+// C8 pieces of a het call from a column in canonical order (W = sum of pooled mid-ranks of the
+// allele-1 qualities, tie = sum(t^3 - t)): each allele's keys are one run with qualities
+// descending, so the pooled mid-ranks come from one merge from the low-quality ends.  Het calls
+// only, so out of line.
+#if !GSNP_PIECES_INLINE
+__device__ __noinline__
+#else
+__device__ __forceinline__
+#endif
+double2 rank_pieces_sorted(const uint32_t* colp, uint64_t cu, int a1, int a2) {
+    double wsum = 0.0, tie = 0.0;
+    uint32_t sx = 0, sy = 0;
+    for (int b = 0; b < a1; ++b) sx += f16(cu, b);
+    for (int b = 0; b < a2; ++b) sy += f16(cu, b);
+    uint32_t ix = sx + f16(cu, a1), iy = sy + f16(cu, a2);
+    double less = 0.0;
+    while (ix > sx || iy > sy) {
+        const uint32_t qx = ix > sx ? key_q(COLKEY(colp[(ix - 1) * TS])) : 99u;
+        const uint32_t qy = iy > sy ? key_q(COLKEY(colp[(iy - 1) * TS])) : 99u;
+        const uint32_t v = min(qx, qy);
+        uint32_t cx = 0, cy = 0;
+        while (ix > sx && key_q(COLKEY(colp[(ix - 1) * TS])) == v) { ++cx; --ix; }
+        while (iy > sy && key_q(COLKEY(colp[(iy - 1) * TS])) == v) { ++cy; --iy; }
+        const double t = (double)(cx + cy);
+        wsum += (double)cx * (less + (t + 1.0) / 2.0);
+        tie += t * t * t - t;
+        less += t;
+    }
+    return make_double2(wsum, tie);
+}
+
 // C6-C9 for one site held by one thread: priors, posterior, top-2, rank-sum pieces, record.
 // SORTED: the column holds the site's keys in canonical order (rank-sum by one merge).
 template <bool DBG, bool SORTED, bool INL>
@@ -911,25 +950,9 @@ __device__ __forceinline__ void thread_finish(const CallArgs& A, const double* l
     const int a1 = geno_a1(t1), a2 = geno_a2(t1);
     double wsum = 0.0, tie = 0.0;
     if (SORTED && a1 != a2 && (A.flags & GSNP_RANK_SUM) && f16(cu, a1) && f16(cu, a2)) {
-        // The column is in canonical order: each allele's keys are one run with qualities
-        // descending, so the pooled mid-ranks come from one merge from the low-quality ends.
-        uint32_t sx = 0, sy = 0;
-        for (int b = 0; b < a1; ++b) sx += f16(cu, b);
-        for (int b = 0; b < a2; ++b) sy += f16(cu, b);
-        uint32_t ix = sx + f16(cu, a1), iy = sy + f16(cu, a2);
-        double less = 0.0;
-        while (ix > sx || iy > sy) {
-            const uint32_t qx = ix > sx ? key_q(COLKEY(colp[(ix - 1) * TS])) : 99u;
-            const uint32_t qy = iy > sy ? key_q(COLKEY(colp[(iy - 1) * TS])) : 99u;
-            const uint32_t v = min(qx, qy);
-            uint32_t cx = 0, cy = 0;
-            while (ix > sx && key_q(COLKEY(colp[(ix - 1) * TS])) == v) { ++cx; --ix; }
-            while (iy > sy && key_q(COLKEY(colp[(iy - 1) * TS])) == v) { ++cy; --iy; }
-            const double t = (double)(cx + cy);
-            wsum += (double)cx * (less + (t + 1.0) / 2.0);
-            tie += t * t * t - t;
-            less += t;
-        }
+        const double2 wt = rank_pieces_sorted(colp, cu, a1, a2);
+        wsum = wt.x;
+        tie = wt.y;
     }
     if (!SORTED && a1 != a2 && (A.flags & GSNP_RANK_SUM) && f16(cu, a1) && f16(cu, a2)) {
         // column in chunk order: pooled mid-ranks by pairwise counts (het calls only)
@@ -1565,6 +1588,9 @@ struct BigSite {
 // independently (no CTA barrier): counting + base_word gather (site-major, no atomics), then
 // thread-per-site sort + likelihood + posterior + record; its sites with more than 32 keys
 // follow on the warp paths; beyond 1024 keys they go to k_big_sites.
+#ifndef GSNP_REC_OOL
+#define GSNP_REC_OOL 0
+#endif
 #ifndef GSNP_CALL_MINB
 #define GSNP_CALL_MINB 3
 #endif
@@ -1644,7 +1670,11 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
     bool slow_pcr = false, have_minus = false;
     int run_pos = INT32_MIN;
     uint32_t run_start = 0;
+#if GSNP_END64
     int64_t last_end = 0, last_end_pos = 0;
+#else
+    int last_end = 0, last_end_pos = 0;      // read starts relative to g0 fit 32 bits (|pk| < 2^30)
+#endif
     int err = 0;
     uint32_t* dbg_built = nullptr;
     if (DBG && A.dbg_keys_built) dbg_built = A.dbg_keys_built + (active ? A.dbg_off[site - A.w0] : 0);
@@ -1713,7 +1743,11 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
                     }
                 }
                 if (!one_len) {       // '-' ends must rise between start runs, else recount pcr
+#if GSNP_END64
                     const int64_t e = (int64_t)pk[u] + lk - 1;
+#else
+                    const int e = pk[u] + (int)lk - 1;
+#endif
                     const bool minus = use && sk;
                     slow_pcr |= minus && have_minus &&
                                 (e < last_end || (e == last_end && pk[u] != last_end_pos));
@@ -1737,11 +1771,11 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
     // the deep kernel also keeps 33..128-key sites on the thread path (chunked sort + merge)
     const bool small = active && n <= COLS;
     const bool mid = CC > COLS && active && n > COLS && n <= CC && !slow_pcr;
-    const uint32_t maxn = __reduce_max_sync(FULL, small ? n : 0u);
     if (small) {
-        if (CC == COLS && maxn <= 16) sort_column<16>(colp, n);   // (one network in the deeper
-        else sort_column<32>(colp, n);                           //  kernels: instruction cache)
-        thread_site<DBG, CC == COLS>(A, adj, lp_s, rt, colp, site, n, slow_pcr, ca0, ca1, ca2, ca3, rep);
+        sort_column<32>(colp, n);     // one network for every n <= 32: a second (16-key) network
+                                      // measured 1.4% slower at C2 (instruction cache)
+        thread_site<DBG, CC == COLS && !GSNP_REC_OOL>(A, adj, lp_s, rt, colp, site, n, slow_pcr, ca0, ca1,
+                                                     ca2, ca3, rep);
     } else if (mid) {
         thread_site_deep<DBG, CC / 32>(A, adj, lp_s, rt, colp, site, n, ca0, ca1, ca2, ca3, rep);
     }

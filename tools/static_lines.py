@@ -9,7 +9,7 @@ import tempfile
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 name = sys.argv[1] if len(sys.argv) > 1 else "_ZN8gsnp_dev11k_call_tileILb0ELi32E"
 top = int(sys.argv[2]) if len(sys.argv) > 2 else 30
-lib = os.environ.get("GSNP_LIB") or os.path.join(ROOT, "paper_conf_icpp_luzlwfl11_b200", "libgsnp.so")
+lib = os.path.abspath(os.environ.get("GSNP_LIB") or "") if os.environ.get("GSNP_LIB") else os.path.join(ROOT, "paper_conf_icpp_luzlwfl11_b200", "libgsnp.so")
 d = tempfile.mkdtemp()
 subprocess.run(["cuobjdump", "-xelf", "all", lib], cwd=d, capture_output=True)
 txt = ""
