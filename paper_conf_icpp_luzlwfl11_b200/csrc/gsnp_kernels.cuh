@@ -1767,7 +1767,7 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
         continue;
     }
 
-    // ---- thread-per-site sort (in-register network sized per warp: 16 / 32) + likelihood;
+    // ---- thread-per-site sort (in-register 32-key network) + likelihood;
     // the deep kernel also keeps 33..128-key sites on the thread path (chunked sort + merge)
     const bool small = active && n <= COLS;
     const bool mid = CC > COLS && active && n > COLS && n <= CC && !slow_pcr;
