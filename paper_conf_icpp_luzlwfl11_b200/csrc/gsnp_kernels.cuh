@@ -80,6 +80,12 @@ struct CallArgs {
     int count_only;
 };
 
+// x << s with PTX semantics: shifts of 32 or more give 0
+__device__ __forceinline__ uint32_t shl_clamp(uint32_t x, uint32_t s) {
+    uint32_t r;
+    asm("shl.b32 %0, %1, %2;" : "=r"(r) : "r"(x), "r"(s));
+    return r;
+}
 __device__ __forceinline__ uint32_t lanemask_lt() {
     uint32_t m;
     asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
@@ -1676,6 +1682,7 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
     int last_end = 0, last_end_pos = 0;      // read starts relative to g0 fit 32 bits (|pk| < 2^30)
 #endif
     int err = 0;
+    uint32_t bmax = 0, qmx = 0;                              // largest base code / quality seen
     uint32_t* dbg_built = nullptr;
     if (DBG && A.dbg_keys_built) dbg_built = A.dbg_keys_built + (active ? A.dbg_off[site - A.w0] : 0);
     // byte arrays addressed from the warp's first read with 32-bit offsets: the bases of the
@@ -1717,10 +1724,10 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
             for (int u = 0; u < GB; ++u) {
                 const uint32_t b = bb[u], q = qq[u];
                 const uint32_t lk = mk[u] & 511u, sk = (mk[u] >> 9) & 1u, hk = mk[u] >> 10;
-                const bool cov = lk != 0;
-                err |= (cov && (b > 4 || q > (uint32_t)A.q_max)) ? ERR_RANGE : 0;
+                bmax = max(bmax, b);                             // range checks after the group
+                qmx = max(qmx, q);                               // (uncovered: b = 4, q = 0)
                 const bool nb = b < 4;                           // a non-N aligned base
-                cpack += nb ? 1u << (8 * b) : 0u;
+                cpack += shl_clamp(1u, 8 * b);                   // 0 for N (shift 32)
                 rep += nb ? hk : 0u;
                 const bool use = nb && hk == 1;                  // uniquely aligned
                 const uint32_t i = ii[u];
@@ -1761,6 +1768,7 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
         }
         ca0 += cpack & 255u; ca1 += (cpack >> 8) & 255u; ca2 += (cpack >> 16) & 255u; ca3 += cpack >> 24;
     }
+    err |= (bmax > 4 || qmx > (uint32_t)A.q_max) ? ERR_RANGE : 0;
     if (err) atomicOr(A.err, err);
     if (DBG && A.count_only) {
         if (active) A.dbg_nuni[site - A.w0] = n;
