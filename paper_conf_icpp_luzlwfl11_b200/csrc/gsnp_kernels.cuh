@@ -1676,11 +1676,7 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
     bool slow_pcr = false, have_minus = false;
     int run_pos = INT32_MIN;
     uint32_t run_start = 0;
-#if GSNP_END64
-    int64_t last_end = 0, last_end_pos = 0;
-#else
     int last_end = 0, last_end_pos = 0;      // read starts relative to g0 fit 32 bits (|pk| < 2^30)
-#endif
     int err = 0;
     uint32_t bmax = 0, qmx = 0;                              // largest base code / quality seen
     uint32_t* dbg_built = nullptr;
@@ -1713,7 +1709,9 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
                 pk[u] = __shfl_sync(FULL, pr, k);
                 const uint32_t ok = __shfl_sync(FULL, o, k);
                 mk[u] = __shfl_sync(FULL, meta, k);
-                if (k0 + u >= nr) pk[u] = INT32_MAX / 2;       // past the batch: covers nothing
+                // past the batch: lanes k >= nr hold pr = INT32_MAX / 2 and meta = 0 already; only a
+                // GB that does not divide 32 can wrap k past 31 onto lane 0
+                if ((32 % GB) != 0 && k0 + u >= nr) pk[u] = INT32_MAX / 2;
                 ii[u] = (uint32_t)(lane_rel - pk[u]);           // huge unless 0 <= i < len
                 const bool cov = ii[u] < (mk[u] & 511u);
                 bb[u] = cov ? wbases[ok + ii[u]] : 4u;
@@ -1732,7 +1730,9 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
                 const bool use = nb && hk == 1;                  // uniquely aligned
                 const uint32_t i = ii[u];
                 const uint32_t cyc = sk ? lk - 1 - i : i;
-                const uint32_t key = b << 15 | ((63u - q) & 63u) << 9 | cyc << 1 | sk;
+                // (a quality above 63 is a range error of the call; its bits only reach the masked
+                // quality and base fields, never the coordinate)
+                const uint32_t key = b << 15 | (63u - q) << 9 | cyc << 1 | sk;
                 if (DBG && dbg_built && use) dbg_built[n] = key;
                 // pcr: keys sharing (base, strand, coord) come from reads with the same start
                 // ('+') or the same end ('-'); with equal starts they are one run of this
@@ -1750,11 +1750,7 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
                     }
                 }
                 if (!one_len) {       // '-' ends must rise between start runs, else recount pcr
-#if GSNP_END64
-                    const int64_t e = (int64_t)pk[u] + lk - 1;
-#else
                     const int e = pk[u] + (int)lk - 1;
-#endif
                     const bool minus = use && sk;
                     slow_pcr |= minus && have_minus &&
                                 (e < last_end || (e == last_end && pk[u] != last_end_pos));
