@@ -1182,23 +1182,32 @@ __device__ __forceinline__ void group_epilogue(const CallArgs& A, uint64_t site,
 // Warp gather of one site's unique non-N keys from the reads [ra, rb) into the warp slice (at
 // most cap keys are stored: a deeper site goes to k_big_sites, which gathers again); returns the
 // count.
+// The same pass counts every read's non-N base at the site (all hits: c[4], their hits in rp,
+// this lane's share; the caller reduces across the warp).
 __device__ __forceinline__ uint32_t warp_gather(const CallArgs& A, uint32_t* col, int warp,
-                                                uint64_t s, uint64_t ra, uint64_t rb, uint32_t cap) {
+                                                uint64_t s, uint64_t ra, uint64_t rb, uint32_t cap,
+                                                uint32_t (&c)[4], uint32_t& rp) {
     const int lane = threadIdx.x & 31;
     uint32_t m = 0;
     for (uint64_t r0 = ra; r0 < rb; r0 += 32) {
         const uint64_t r = r0 + lane;
         uint32_t key = KEY_INF;
-        if (r < rb && A.R.hits[r] == 1) {
-            const uint64_t i = s - A.R.pos[r];
+        if (r < rb) {
+            const uint64_t i = s - A.R.pos[r];               // huge when the read starts later
             const uint32_t l = A.R.len[r];
             if (i < l) {
                 const uint64_t bi = A.R.off[r] - A.R.off0 + i;
                 const uint32_t b = A.R.bases[bi];
                 if (b < 4) {
-                    const uint32_t st = A.R.strand[r];
-                    const uint32_t cyc = st ? l - 1 - (uint32_t)i : (uint32_t)i;
-                    key = b << 15 | (63u - A.R.quals[bi]) << 9 | cyc << 1 | st;
+                    const uint32_t h = A.R.hits[r];
+#pragma unroll
+                    for (int x = 0; x < 4; ++x) c[x] += b == (uint32_t)x;
+                    rp += h;
+                    if (h == 1) {
+                        const uint32_t st = A.R.strand[r];
+                        const uint32_t cyc = st ? l - 1 - (uint32_t)i : (uint32_t)i;
+                        key = b << 15 | (63u - A.R.quals[bi]) << 9 | cyc << 1 | st;
+                    }
                 }
             }
         }
@@ -1820,24 +1829,13 @@ __global__ void __launch_bounds__(NT) k_warp_sites(const __grid_constant__ CallA
         const uint64_t grp = (s - A.w0) / 32;
         const uint64_t ra = A.tile_ra[grp], rb = A.tile_rb[grp];
         uint32_t c[4] = {0, 0, 0, 0}, rp = 0;
-        for (uint64_t r = ra + lane; r < rb; r += 32) {
-            const uint64_t i = s - A.R.pos[r];                   // huge when the read starts later
-            if (i < A.R.len[r]) {
-                const uint32_t b = A.R.bases[A.R.off[r] - A.R.off0 + i];
-                if (b < 4) {
-#pragma unroll
-                    for (int x = 0; x < 4; ++x) c[x] += b == (uint32_t)x;
-                    rp += A.R.hits[r];
-                }
-            }
-        }
+        const uint32_t m = warp_gather(A, sm.col, warp, s, ra, rb, 32u * CC, c, rp);
 #pragma unroll
         for (int d = 16; d > 0; d >>= 1) {
 #pragma unroll
             for (int x = 0; x < 4; ++x) c[x] += __shfl_xor_sync(FULL, c[x], d);
             rp += __shfl_xor_sync(FULL, rp, d);
         }
-        const uint32_t m = warp_gather(A, sm.col, warp, s, ra, rb, 32u * CC);
         if (m > 32u * CC) {
             if (lane == 0) {
                 const uint32_t k = atomicAdd(big_n, 1u);
