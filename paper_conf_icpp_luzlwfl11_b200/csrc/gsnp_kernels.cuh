@@ -1642,11 +1642,14 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
     const uint64_t n_groups = (A.w1 - A.w0 + 31) / 32;
     // persistent warps: each takes the next group of 32 consecutive sites from a counter; the
     // next group's index and read range are fetched while the current one is processed
-    // groups are claimed GSNP_CLAIM at a time (fewer atomics on the one counter)
+    // groups are claimed GSNP_CLAIM at a time (fewer atomics on the one counter) when every warp
+    // gets many claims; a small window (the paper's 256 K sites: ~2 groups per warp) claims one
+    // at a time so no warp is left with a tail of several groups
+    const uint32_t claim = n_groups >= (uint64_t)8 * GSNP_CLAIM * gridDim.x * (NT / 32) ? GSNP_CLAIM : 1u;
     uint64_t nxt = 0, nra = 0, nrb = 0, claim_end = 0;
-    if (lane == 0) nxt = atomicAdd(work, (uint32_t)GSNP_CLAIM);
+    if (lane == 0) nxt = atomicAdd(work, claim);
     nxt = __shfl_sync(FULL, nxt, 0);
-    claim_end = nxt + GSNP_CLAIM;
+    claim_end = nxt + claim;
     if (nxt < n_groups) { nra = A.tile_ra[nxt]; nrb = A.tile_rb[nxt]; }
     for (;;) {
     const uint64_t grp = nxt;
@@ -1656,9 +1659,9 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
     if (grp + 1 < claim_end) {
         nxt = grp + 1;
     } else {
-        if (lane == 0) nxt = atomicAdd(work, (uint32_t)GSNP_CLAIM);
+        if (lane == 0) nxt = atomicAdd(work, claim);
         nxt = __shfl_sync(FULL, nxt, 0);
-        claim_end = nxt + GSNP_CLAIM;
+        claim_end = nxt + claim;
     }
     if (nxt < n_groups) { nra = A.tile_ra[nxt]; nrb = A.tile_rb[nxt]; }
     const uint64_t g0 = A.w0 + grp * 32;                     // first site of the group
