@@ -205,6 +205,7 @@ struct gsnp_ctx {
     }
     // window depth thresholds of the 64- / 128-slot k_call_tile instantiations (pick_variant)
     float mid_at = 24.0f, deep_at = 48.0f;
+    uint32_t epoch = 0;               // calls so far (k_prep's read-length flag)
     bool mid_adj_smem = false;        // the 64-slot kernel reads adj from L1/L2: 3 CTAs per SM
     size_t cal_budget = 0;            // k_calib_count shared-memory budget (0 = not yet sized)
     // per-stage timing (GSNP_TIMING)
@@ -503,18 +504,21 @@ gsnp_status prep_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t 
     const uint64_t n_groups = (w1 - w0 + 31) / 32;
     CK(ctx->tile_ra.ensure(n_groups));
     CK(ctx->tile_rb.ensure(n_groups));
-    CK(ctx->big_n.ensure(3));
+    CK(ctx->big_n.ensure(4));
+    const uint32_t epoch = ++ctx->epoch;               // k_prep's read-length flag (no reset)
     // one launch: validate the reads (ABI contract; the calling kernels return at once on a
     // violation), the per-group read ranges, and zero the window's work counters
     const uint32_t nbv = (uint32_t)((d.n + 255) / 256);
     ctx->begin();
     k_prep<<<(unsigned)(nbv + (n_groups + 255) / 256), 256, 0, s>>>(
         d, ctx->origin, ctx->n_sites, (int)ctx->prm.max_read_len, ctx->d_err.p, nbv, w0, w1, n_groups,
-        ctx->tile_ra.p, ctx->tile_rb.p, ctx->big_n.p);
+        ctx->tile_ra.p, ctx->tile_rb.p, ctx->big_n.p, epoch);
     ctx->end(GSNP_STAGE_RANGES);
     ctx->launches++;
     CK(cudaGetLastError());
     A.R = d;
+    A.len_flag = ctx->big_n.p + 3;
+    A.epoch = epoch;
     A.ref = ctx->ref_code;
     A.origin = ctx->origin;
     A.n_sites = ctx->n_sites;

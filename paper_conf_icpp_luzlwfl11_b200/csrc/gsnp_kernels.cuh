@@ -69,6 +69,8 @@ struct CallArgs {
     gsnp_record* out;                 // out[site - w0]
     int* err;
     float mid_at, deep_at;            // window depth thresholds of the 64- and 128-slot kernels
+    const uint32_t* len_flag;         // == epoch: not every read has the same length (k_prep)
+    uint32_t epoch;
     // debug (all may be null)
     uint32_t* dbg_nuni;               // count-only pass: unique keys per site
     const uint32_t* dbg_off;          // CSR offsets for the key dumps
@@ -128,13 +130,18 @@ __device__ __forceinline__ void validate_read(const DevReads& R, uint64_t r, uin
     if (e) atomicOr(err, e | ERR_VALID);
 }
 
+// counters[3]: set to `epoch` (this call's number) when some read's length differs from read 0's —
+// the calling kernels then check uniformity per group; no reset is needed between calls
 __global__ void k_prep(DevReads R, uint64_t origin, uint64_t n_sites, int L, int* err, uint32_t nbv,
                        uint64_t w0, uint64_t w1, uint64_t n_groups, uint64_t* ra, uint64_t* rb,
-                       uint32_t* counters) {
+                       uint32_t* counters, uint32_t epoch) {
     if (blockIdx.x == 0 && threadIdx.x < 3) counters[threadIdx.x] = 0;
     if (blockIdx.x < nbv) {
         const uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-        if (r < R.n) validate_read(R, r, origin, n_sites, L, err);
+        if (r < R.n) {
+            validate_read(R, r, origin, n_sites, L, err);
+            if (R.len[r] != R.len[0]) counters[3] = epoch;
+        }
         return;
     }
     const uint64_t g = (blockIdx.x - nbv) * (uint64_t)blockDim.x + threadIdx.x;
@@ -1640,6 +1647,7 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
     uint32_t* colp = sm.col + tid;                           // this lane's column
     __syncthreads();
     const uint64_t n_groups = (A.w1 - A.w0 + 31) / 32;
+    const bool all_one_len = *A.len_flag != A.epoch;          // every read has read 0's length
     // persistent warps: each takes the next group of 32 consecutive sites from a counter; the
     // next group's index and read range are fetched while the current one is processed
     // groups are claimed GSNP_CLAIM at a time (fewer atomics on the one counter) when every warp
@@ -1677,7 +1685,7 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
     // the range has the same length, '-' strand reads share a coordinate only within one start
     // run and the end tracking below is skipped.
     uint32_t one_len = 1;
-    {
+    if (!all_one_len) {                                       // some read's length differs
         const uint32_t L0 = wra < wrb ? A.R.len[wra] : 0u;
         for (uint64_t r0 = wra; r0 < wrb; r0 += 32) {          // warp-uniform trip count
             const uint64_t r = r0 + lane;
