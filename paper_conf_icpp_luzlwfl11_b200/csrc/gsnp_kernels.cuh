@@ -919,7 +919,9 @@ double2 rank_pieces_sorted(const uint32_t* colp, uint64_t cu, int a1, int a2) {
 
 // C6-C9 for one site held by one thread: priors, posterior, top-2, rank-sum pieces, record.
 // SORTED: the column holds the site's keys in canonical order (rank-sum by one merge).
-template <bool DBG, bool SORTED, bool INL>
+// HIST (unsorted columns of up to 128 keys): rank-sum pieces from quality histograms instead of
+// pairwise counts.
+template <bool DBG, bool SORTED, bool INL, bool HIST = false>
 // lps: the novel log10 prior rows (R6) staged in shared memory; rt: the site's reference byte
 // (code | known << 3), loaded when the site's group was taken.
 __device__ __forceinline__ void thread_finish(const CallArgs& A, const double* lps, uint32_t rt,
@@ -968,20 +970,46 @@ __device__ __forceinline__ void thread_finish(const CallArgs& A, const double* l
         tie = wt.y;
     }
     if (!SORTED && a1 != a2 && (A.flags & GSNP_RANK_SUM) && f16(cu, a1) && f16(cu, a2)) {
-        // column in chunk order: pooled mid-ranks by pairwise counts (het calls only)
-        for (uint32_t x = 0; x < n; ++x) {
-            const uint32_t xk = colp[x * TS] >> 8;
-            const uint32_t xb = key_base(xk), xq = key_q(xk);
-            if (xb != (uint32_t)a1 && xb != (uint32_t)a2) continue;
-            uint32_t less = 0, eq = 0;
-            for (uint32_t y = 0; y < n; ++y) {
-                const uint32_t yk = colp[y * TS] >> 8, yb = key_base(yk), yq = key_q(yk);
-                const bool yin = yb == (uint32_t)a1 || yb == (uint32_t)a2;
-                less += yin && yq < xq;
-                eq += yin && yq == xq;
+        if (HIST) {
+            // column in chunk order: pooled mid-ranks from the two alleles' quality histograms (6-bit
+            // qualities; counts of allele 1 / 2 in the low / high half of one word per quality), walked
+            // from the lowest quality as the sorted merge does — every term is an integer or a
+            // half-integer, so the sums are exact in either order
+            uint32_t hq[64];
+#pragma unroll
+            for (int q = 0; q < 64; ++q) hq[q] = 0;
+            for (uint32_t x = 0; x < n; ++x) {
+                const uint32_t xk = colp[x * TS] >> 8;
+                const uint32_t xb = key_base(xk), xq = key_q(xk);
+                if (xb == (uint32_t)a1) hq[xq] += 1u;
+                else if (xb == (uint32_t)a2) hq[xq] += 1u << 16;
             }
-            if (xb == (uint32_t)a1) wsum += (double)less + ((double)eq + 1.0) / 2.0;
-            tie += (double)eq * (double)eq - 1.0;
+            double less = 0.0;
+            for (int q = 0; q < 64; ++q) {
+                const uint32_t c1 = hq[q] & 0xFFFFu, t = c1 + (hq[q] >> 16);
+                if (t) {
+                    const double td = (double)t;
+                    wsum += (double)c1 * (less + (td + 1.0) / 2.0);
+                    tie += td * td * td - td;
+                    less += td;
+                }
+            }
+        } else {
+            // column in chunk order: pooled mid-ranks by pairwise counts (het calls only)
+            for (uint32_t x = 0; x < n; ++x) {
+                const uint32_t xk = colp[x * TS] >> 8;
+                const uint32_t xb = key_base(xk), xq = key_q(xk);
+                if (xb != (uint32_t)a1 && xb != (uint32_t)a2) continue;
+                uint32_t less = 0, eq = 0;
+                for (uint32_t y = 0; y < n; ++y) {
+                    const uint32_t yk = colp[y * TS] >> 8, yb = key_base(yk), yq = key_q(yk);
+                    const bool yin = yb == (uint32_t)a1 || yb == (uint32_t)a2;
+                    less += yin && yq < xq;
+                    eq += yin && yq == xq;
+                }
+                if (xb == (uint32_t)a1) wsum += (double)less + ((double)eq + 1.0) / 2.0;
+                tie += (double)eq * (double)eq - 1.0;
+            }
         }
     }
     if (DBG && (A.dbg_L10 || A.dbg_post10)) {
@@ -1144,7 +1172,8 @@ __device__ __forceinline__ void thread_site_deep(const CallArgs& A, const uint8_
 #pragma unroll
             for (int k = 0; k < 10; ++k) acc[k] += v[u][k];
     }
-    thread_finish<DBG, false, false>(A, lps, rt, colp, site, n, acc, cu, qs, ca0, ca1, ca2, ca3, rep);
+    thread_finish<DBG, false, false, (NCH >= 4)>(A, lps, rt, colp, site, n, acc, cu, qs, ca0, ca1, ca2,
+                                                 ca3, rep);
 }
 
 // ------------------------------------------------------------------------------------------
