@@ -1111,13 +1111,11 @@ __device__ __forceinline__ void thread_site_deep(const CallArgs& A, const uint8_
         const uint32_t cn = n > 32u * c ? min(32u, n - 32u * c) : 0u;
         if (cn) sort_column<32>(colp + (size_t)32 * c * TS, cn);
     }
-    uint32_t hi[NCH], he[NCH], hk[NCH];
+    // merge heads packed as (column word << 2) | chunk (words are unique and < 2^25), so one
+    // minimum gives the next key and its chunk; byte c of cur = position of chunk c's head
+    uint32_t hk[NCH], cur = 0;
 #pragma unroll
-    for (int c = 0; c < NCH; ++c) {
-        hi[c] = 32u * c;
-        he[c] = min(n, 32u * c + 32u);
-        hk[c] = hi[c] < he[c] ? colp[hi[c] * TS] : KEY_INF;
-    }
+    for (int c = 0; c < NCH; ++c) hk[c] = 32u * c < n ? colp[32u * c * TS] << 2 | (uint32_t)c : KEY_INF;
     uint32_t* dbg = nullptr;
     if (DBG && A.dbg_keys_sorted) dbg = A.dbg_keys_sorted + A.dbg_off[site - A.w0];
     double acc[10];
@@ -1138,12 +1136,15 @@ __device__ __forceinline__ void thread_site_deep(const CallArgs& A, const uint8_
             rowv[u] = 0xFFFFFFFFu;
             if (out0 + u < n) {
                 uint32_t best = hk[0];
-                int bc = 0;
 #pragma unroll
-                for (int c = 1; c < NCH; ++c) if (hk[c] < best) { best = hk[c]; bc = c; }
+                for (int c = 1; c < NCH; ++c) best = min(best, hk[c]);
+                const uint32_t bc = best & 3u;
+                const uint32_t ni = ((cur >> (8u * bc)) & 255u) + 1u, gi = 32u * bc + ni;
+                cur += 1u << (8u * bc);
+                const uint32_t nv = ni < 32u && gi < n ? colp[gi * TS] << 2 | bc : KEY_INF;
 #pragma unroll
-                for (int c = 0; c < NCH; ++c)
-                    if (c == bc) { ++hi[c]; hk[c] = hi[c] < he[c] ? colp[hi[c] * TS] : KEY_INF; }
+                for (int c = 0; c < NCH; ++c) hk[c] = (uint32_t)c == bc ? nv : hk[c];
+                best >>= 2;                                  // the column word
                 const uint32_t kk = best >> 8, b = key_base(kk), q = key_q(kk);
                 if (DBG && dbg) dbg[out0 + u] = kk;
                 const uint32_t pcr = (best & 255u) + 1u;
