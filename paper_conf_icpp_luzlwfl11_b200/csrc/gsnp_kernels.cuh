@@ -1640,6 +1640,9 @@ struct BigSite {
 // independently (no CTA barrier): counting + base_word gather (site-major, no atomics), then
 // thread-per-site sort + likelihood + posterior + record; its sites with more than 32 keys
 // follow on the warp paths; beyond 1024 keys they go to k_big_sites.
+#ifndef GSNP_MID_UNIFORM
+#define GSNP_MID_UNIFORM 1
+#endif
 #ifndef GSNP_REC_OOL
 #define GSNP_REC_OOL 0
 #endif
@@ -1823,8 +1826,14 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
 
     // ---- thread-per-site sort (in-register 32-key network) + likelihood;
     // the deep kernel also keeps 33..128-key sites on the thread path (chunked sort + merge)
-    const bool small = active && n <= COLS;
-    const bool mid = CC > COLS && active && n > COLS && n <= CC && !slow_pcr;
+    bool small = active && n <= COLS;
+    bool mid = CC > COLS && active && n > COLS && n <= CC && !slow_pcr;
+#if GSNP_MID_UNIFORM
+    // one path per warp: when any lane needs the chunked path, its small sites take it too (the
+    // chunked path visits the keys in the same canonical order, so the sums are the same) instead
+    // of the warp running both paths one after the other
+    if (CC > COLS && __any_sync(FULL, mid) && small && !slow_pcr) { small = false; mid = true; }
+#endif
     if (small) {
         sort_column<32>(colp, n);     // one network for every n <= 32: a second (16-key) network
                                       // measured 1.4% slower at C2 (instruction cache)
