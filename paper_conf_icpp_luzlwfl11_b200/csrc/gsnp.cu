@@ -153,6 +153,7 @@ struct gsnp_ctx {
     DevBuf<BigSite> big;
     DevBuf<uint32_t> big_n;
     DevBuf<uint32_t> wlist;
+    DevBuf<uint32_t> wlist2;       // k_list_sites' leftovers for k_warp_sites
     // dense ablation (§8(f) NEXT #3): base_occ of one chunk of sites + per-site all-hits counters
     DevBuf<uint8_t> dense_occ;
     DevBuf<uint32_t> dense_cnt;
@@ -504,7 +505,7 @@ gsnp_status prep_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t 
     const uint64_t n_groups = (w1 - w0 + 31) / 32;
     CK(ctx->tile_ra.ensure(n_groups));
     CK(ctx->tile_rb.ensure(n_groups));
-    CK(ctx->big_n.ensure(4));
+    CK(ctx->big_n.ensure(6));
     const uint32_t epoch = ++ctx->epoch;               // k_prep's read-length flag (no reset)
     // one launch: validate the reads (ABI contract; the calling kernels return at once on a
     // violation), the per-group read ranges, and zero the window's work counters
@@ -604,13 +605,28 @@ gsnp_status run_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t w
         ctx->launches++;
     }
     if (!A.count_only) {
-        // listed sites (n > 32 keys, or beyond the deep kernel's thread path): warp per site
+        // sites the 32-slot kernel listed (33..64 keys): thread per listed site, chunked thread path
+        CK(ctx->wlist2.ensure(w1 - w0));
+        auto lk = dbg ? k_list_sites<true> : k_list_sites<false>;
+        const size_t lsm = (size_t)4 * COLS_MID * TS;
+        const int lper = ctx->occupancy(reinterpret_cast<const void*>(lk), NT, lsm);
+        if (lper < 0) return fail(ctx, GSNP_E_CUDA, "k_list_sites: shared memory %zu B", lsm);
+        ctx->begin();
+        lk<<<(unsigned)(ctx->num_sms * std::max(lper, 1)), NT, lsm, s>>>(A, ctx->wlist.p, ctx->big_n.p + 2,
+                                                                       ctx->wlist2.p, ctx->big_n.p + 4,
+                                                                       ctx->big_n.p + 5);
+        ctx->end(GSNP_STAGE_WARP);
+        ctx->launches++;
+        CK(cudaGetLastError());
+        // what is left (n > 64 keys, '-' end recounts, or beyond the deep kernels' thread paths):
+        // warp per site
         auto wk = k_warp_sites<COLS>;
         const size_t wsm = call_smem_bytes(A.L, 0, COLS, nullptr, nullptr);
         const int wper = ctx->occupancy(reinterpret_cast<const void*>(wk), NT, wsm);
         if (wper < 0) return fail(ctx, GSNP_E_CUDA, "k_warp_sites: shared memory %zu B", wsm);
         ctx->begin();
         wk<<<(unsigned)(ctx->num_sms * std::max(wper, 1)), NT, wsm, s>>>(A, ctx->wlist.p, ctx->big_n.p + 2,
+                                                                       ctx->wlist2.p, ctx->big_n.p + 4,
                                                                        ctx->big.p, ctx->big_n.p, big_cap);
         ctx->end(GSNP_STAGE_WARP);
         ctx->launches++;
@@ -1632,7 +1648,7 @@ void gsnp_destroy(gsnp_ctx* ctx) {
     ctx->ref.release(); ctx->known_pos.release(); ctx->known_lp.release();
     ctx->adj.release(); ctx->LP.release(); ctx->rank_cdf.release(); ctx->T.release(); ctx->d_err.release();
     ctx->d_counts.release(); ctx->tile_ra.release(); ctx->tile_rb.release(); ctx->rec.release();
-    ctx->big.release(); ctx->big_n.release(); ctx->wlist.release();
+    ctx->big.release(); ctx->big_n.release(); ctx->wlist.release(); ctx->wlist2.release();
     ctx->dense_occ.release(); ctx->dense_cnt.release();
     ctx->p_text.release(); ctx->p_chr.release(); ctx->p_cnt.release(); ctx->p_ls.release();
     ctx->p_meta.release(); ctx->p_pos.release(); ctx->p_ridx.release(); ctx->p_boff.release();

@@ -135,7 +135,7 @@ __device__ __forceinline__ void validate_read(const DevReads& R, uint64_t r, uin
 __global__ void k_prep(DevReads R, uint64_t origin, uint64_t n_sites, int L, int* err, uint32_t nbv,
                        uint64_t w0, uint64_t w1, uint64_t n_groups, uint64_t* ra, uint64_t* rb,
                        uint32_t* counters, uint32_t epoch) {
-    if (blockIdx.x == 0 && threadIdx.x < 3) counters[threadIdx.x] = 0;
+    if (blockIdx.x == 0 && (threadIdx.x < 3 || threadIdx.x == 4 || threadIdx.x == 5)) counters[threadIdx.x] = 0;
     if (blockIdx.x < nbv) {
         const uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
         if (r < R.n) {
@@ -1857,15 +1857,92 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
     }  // persistent loop
 }
 
+// Sites listed by the 32-slot k_call_tile (more than 32 unique keys): one thread per listed site,
+// 32 listed sites per warp.  Each thread walks its site's group read range (as the gather does,
+// reads in position order, so the same pcr runs and '-' end checks apply), gathers the site's keys
+// into its own 64-slot column and runs the chunked thread path; sites with more than 64 keys or a
+// '-' end recount go on to k_warp_sites through the second list.  (Windows called by the 64- and
+// 128-slot kernels return at once: their lists hold only sites beyond those kernels' slots.)
+template <bool DBG>
+__global__ void __launch_bounds__(NT, 3) k_list_sites(const __grid_constant__ CallArgs A, const uint32_t* wlist,
+                                                      const uint32_t* wlist_n, uint32_t* wlist2,
+                                                      uint32_t* wlist2_n, uint32_t* work) {
+    if (reads_invalid(A.err) || pick_variant(A) != 0) return;
+    extern __shared__ __align__(16) unsigned char smem[];
+    __shared__ double lp_s[50];
+    const int tid = threadIdx.x, lane = tid & 31;
+    for (int i = tid; i < 50; i += NT) lp_s[i] = A.LP[i];
+    __syncthreads();
+    uint32_t* colp = reinterpret_cast<uint32_t*>(smem) + tid;          // [COLS_MID][TS]
+    const uint32_t count = *wlist_n;
+    const bool all_one_len = *A.len_flag != A.epoch;
+    for (;;) {
+        uint32_t j0 = 0;
+        if (lane == 0) j0 = atomicAdd(work, 32u);
+        j0 = __shfl_sync(FULL, j0, 0);
+        if (j0 >= count) break;
+        const uint32_t j = j0 + lane;
+        const bool active = j < count;
+        const uint64_t site = A.w0 + (active ? wlist[j] : 0u);
+        const uint64_t grp = (site - A.w0) / 32;
+        const uint64_t ra = A.tile_ra[grp], rb = active ? A.tile_rb[grp] : ra;
+        const uint32_t rt = A.ref[site - A.origin];
+        uint32_t ca0 = 0, ca1 = 0, ca2 = 0, ca3 = 0, rep = 0, n = 0, run_start = 0;
+        uint64_t run_pos = ~0ull, last_end = 0, last_end_pos = 0;
+        bool slow_pcr = false, have_minus = false;
+        for (uint64_t r = ra; r < rb; ++r) {
+            const uint64_t pos = A.R.pos[r];
+            if (pos != run_pos) { run_pos = pos; run_start = n; }
+            const uint64_t i = site - pos;                    // huge when the read starts later
+            const uint32_t l = A.R.len[r];
+            if (i >= l) continue;
+            const uint64_t bi = A.R.off[r] - A.R.off0 + i;
+            const uint32_t b = A.R.bases[bi];
+            if (b >= 4) continue;                             // (range errors: the gather checked)
+            const uint32_t h = A.R.hits[r];
+            ca0 += b == 0; ca1 += b == 1; ca2 += b == 2; ca3 += b == 3;
+            rep += h;
+            if (h != 1) continue;
+            const uint32_t q = A.R.quals[bi], st = A.R.strand[r];
+            const uint32_t cyc = st ? l - 1 - (uint32_t)i : (uint32_t)i;
+            const uint32_t key = b << 15 | (63u - q) << 9 | cyc << 1 | st;
+            uint32_t pcr1 = 0;                                // pcr - 1 as in the gather (R3)
+            const uint32_t jend = min(n, (uint32_t)COLS_MID);
+            for (uint32_t k = run_start; k < jend; ++k) {
+                const uint32_t kj = colp[k * TS];
+                if ((((kj >> 8) ^ key) & KEY_BSLOT) == 0) {
+                    if (key_q(kj >> 8) >= q) ++pcr1;
+                    else if ((kj & 255u) < 255u) colp[k * TS] = kj + 1;
+                }
+            }
+            if (!all_one_len && st) {                         // '-' ends must rise between runs
+                const uint64_t e = pos + l - 1;
+                slow_pcr |= have_minus && (e < last_end || (e == last_end && pos != last_end_pos));
+                last_end = e;
+                last_end_pos = pos;
+                have_minus = true;
+            }
+            if (n < (uint32_t)COLS_MID) colp[n * TS] = key << 8 | min(pcr1, 255u);
+            ++n;
+        }
+        const bool ok = active && n <= (uint32_t)COLS_MID && !slow_pcr;
+        if (active && !ok) wlist2[atomicAdd(wlist2_n, 1u)] = wlist[j];
+        if (ok) thread_site_deep<DBG, COLS_MID / 32>(A, A.adj, lp_s, rt, colp, site, n, ca0, ca1, ca2, ca3, rep);
+        __syncwarp();
+    }
+}
+
 // Sites listed by k_call_tile (n > COLS keys, or n > CC / '-' ends out of order on the deep
 // kernel): one warp per site.  The warp recounts the site's all-hits counters over its group's
 // read range, re-gathers the unique keys into its slice of the col region and runs the warp
 // paths (n <= 32*CC) or hands the site to k_big_sites.
 template <int CC>
 __global__ void __launch_bounds__(NT) k_warp_sites(const __grid_constant__ CallArgs A, const uint32_t* wlist,
-                                                   const uint32_t* wlist_n, BigSite* big,
+                                                   const uint32_t* wlist_n, const uint32_t* wlist2,
+                                                   const uint32_t* wlist2_n, BigSite* big,
                                                    uint32_t* big_n, uint32_t big_cap) {
     if (reads_invalid(A.err)) return;
+    if (pick_variant(A) == 0) { wlist = wlist2; wlist_n = wlist2_n; }   // k_list_sites' leftovers
     extern __shared__ __align__(16) unsigned char smem[];
     TileSmem sm;
     call_smem_bytes(A.L, 0, CC, &sm, smem);
