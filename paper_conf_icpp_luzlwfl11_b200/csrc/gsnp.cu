@@ -205,7 +205,10 @@ struct gsnp_ctx {
         return per;
     }
     // window depth thresholds of the 64- / 128-slot k_call_tile instantiations (pick_variant)
-    float mid_at = 24.0f, deep_at = 48.0f;
+    // window mean depth (reads x L / sites) at which the 64- / 128-slot kernels take over; the 32-slot
+    // kernel + k_list_sites wins below ~29.5 (tools/thr_probe.sh: 10.7 vs 11.4 ms at 27.6, 14.8 vs
+    // 12.4 at 31.3 per 24 M sites)
+    float mid_at = 29.5f, deep_at = 48.0f;
     uint32_t epoch = 0;               // calls so far (k_prep's read-length flag)
     bool mid_adj_smem = false;        // the 64-slot kernel reads adj from L1/L2: 3 CTAs per SM
     size_t cal_budget = 0;            // k_calib_count shared-memory budget (0 = not yet sized)

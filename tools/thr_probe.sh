@@ -1,8 +1,6 @@
-# k_call_tile variant thresholds: per-call stage ms (call_tile sums its three instantiations)
-for i in 1 2; do
-  for pair in "C2 48000000|" "C2 48000000|GSNP_MID_AT=10" "C3 48000000|" "C3 48000000|GSNP_MID_AT=40"; do
-    cfg=${pair%%|*}; env=${pair#*|}
-    echo "$cfg [$env] $(env $env python tools/profile_call.py $cfg 3 2>/dev/null | tail -1 | python -c "
-import sys; d=eval(sys.stdin.read()); print({k: round(v[0]/3, 3) for k, v in d.items() if k in ('call_tile','warp_sites','big_sites')})")"
+# 32-slot (+ k_list_sites) vs 64-slot kernel by depth: per-call ms of call + warp stages
+for d in 26 30 34 38 42 48; do
+  for env in "GSNP_MID_AT=200" "GSNP_MID_AT=1"; do
+    echo "C3 depth $d [$env] $(env $env python tools/profile_depth.py C3 $d 24000000 2 2>/dev/null | tail -1)"
   done
 done
