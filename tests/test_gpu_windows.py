@@ -46,10 +46,11 @@ def test_async_windows_equal_one_call(cfg, win):
 
 
 def test_variants_give_identical_records():
-    """C3-like 30X input called as one window (the 64-slot kernel) and as windows small enough
-    that the overlapping reads' estimate picks the 128-slot kernel (64 sites: (64 + 99) / 64 x the
-    depth) — at this depth every site stays on a thread path in both, where keys are summed in
-    canonical order, so the records are byte-identical."""
+    """C3-like 30X input (mean depth estimate 27.6) called as one window (the 32-slot kernel, its
+    33-64-key sites through k_list_sites) and as windows small enough that the overlapping reads'
+    estimate picks the 64-slot kernel (500 sites: (500 + 99) / 500 x 27.6 = 33) or the 128-slot
+    kernel (64 sites: 70) — at this depth every site stays on a thread path in all three, where
+    keys are summed in canonical order, so the records are byte-identical."""
     import torch
     w = synth.generate("C3", n_sites=2_000_000)
     lo, hi = w["region"]
@@ -59,7 +60,7 @@ def test_variants_give_identical_records():
         one = torch.empty(40 * (hi - lo), dtype=torch.uint8, device="cuda")
         ctx.call(dev, lo, hi, one)
         r_all = gsnp.make_reads(dev)
-        for win in (64, 5_000, 300_000):
+        for win in (64, 500, 5_000, 300_000):
             many = torch.zeros_like(one)
             for a in range(lo, hi, win):            # all reads passed: small windows look deep
                 b = min(hi, a + win)
