@@ -1890,20 +1890,24 @@ __global__ void __launch_bounds__(NT, 3) k_list_sites(const __grid_constant__ Ca
         uint32_t ca0 = 0, ca1 = 0, ca2 = 0, ca3 = 0, rep = 0, n = 0, run_start = 0;
         uint64_t run_pos = ~0ull, last_end = 0, last_end_pos = 0;
         bool slow_pcr = false, have_minus = false;
+        // read r's metadata is loaded one iteration ahead, so each read costs one round trip (its
+        // bytes) instead of two
+        uint64_t npos = ra < rb ? A.R.pos[ra] : 0, noff = ra < rb ? A.R.off[ra] : 0;
+        uint32_t nlen = ra < rb ? A.R.len[ra] : 0u;
         for (uint64_t r = ra; r < rb; ++r) {
-            const uint64_t pos = A.R.pos[r];
+            const uint64_t pos = npos, off = noff;
+            const uint32_t l = nlen;
+            if (r + 1 < rb) { npos = A.R.pos[r + 1]; noff = A.R.off[r + 1]; nlen = A.R.len[r + 1]; }
             if (pos != run_pos) { run_pos = pos; run_start = n; }
             const uint64_t i = site - pos;                    // huge when the read starts later
-            const uint32_t l = A.R.len[r];
             if (i >= l) continue;
-            const uint64_t bi = A.R.off[r] - A.R.off0 + i;
-            const uint32_t b = A.R.bases[bi];
+            const uint64_t bi = off - A.R.off0 + i;
+            // the read's bytes and flags in one round
+            const uint32_t b = A.R.bases[bi], q = A.R.quals[bi], h = A.R.hits[r], st = A.R.strand[r];
             if (b >= 4) continue;                             // (range errors: the gather checked)
-            const uint32_t h = A.R.hits[r];
             ca0 += b == 0; ca1 += b == 1; ca2 += b == 2; ca3 += b == 3;
             rep += h;
             if (h != 1) continue;
-            const uint32_t q = A.R.quals[bi], st = A.R.strand[r];
             const uint32_t cyc = st ? l - 1 - (uint32_t)i : (uint32_t)i;
             const uint32_t key = b << 15 | (63u - q) << 9 | cyc << 1 | st;
             uint32_t pcr1 = 0;                                // pcr - 1 as in the gather (R3)
