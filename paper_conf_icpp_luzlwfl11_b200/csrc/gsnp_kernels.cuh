@@ -1863,18 +1863,24 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
 // into its own 64-slot column and runs the chunked thread path; sites with more than 64 keys or a
 // '-' end recount go on to k_warp_sites through the second list.  (Windows called by the 64- and
 // 128-slot kernels return at once: their lists hold only sites beyond those kernels' slots.)
+// Below LIST_MIN listed sites the warp path takes them all: a thread walks its site's ~40 reads one
+// round trip after another (~60 us whatever the count), while a warp per site finishes one site in
+// ~14 us with every warp of the GPU in parallel (256 K-site windows list ~600 sites).
+constexpr uint32_t LIST_MIN = 16384;
 template <bool DBG>
 __global__ void __launch_bounds__(NT, 3) k_list_sites(const __grid_constant__ CallArgs A, const uint32_t* wlist,
                                                       const uint32_t* wlist_n, uint32_t* wlist2,
                                                       uint32_t* wlist2_n, uint32_t* work) {
     if (reads_invalid(A.err) || pick_variant(A) != 0) return;
+    const uint32_t count = *wlist_n;
+    if (count < LIST_MIN) return;                       // a short list: the warp path is quicker
+    if ((uint64_t)blockIdx.x * NT >= count) return;
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ double lp_s[50];
     const int tid = threadIdx.x, lane = tid & 31;
     for (int i = tid; i < 50; i += NT) lp_s[i] = A.LP[i];
     __syncthreads();
     uint32_t* colp = reinterpret_cast<uint32_t*>(smem) + tid;          // [COLS_MID][TS]
-    const uint32_t count = *wlist_n;
     const bool all_one_len = *A.len_flag != A.epoch;
     for (;;) {
         uint32_t j0 = 0;
@@ -1946,7 +1952,9 @@ __global__ void __launch_bounds__(NT) k_warp_sites(const __grid_constant__ CallA
                                                    const uint32_t* wlist2_n, BigSite* big,
                                                    uint32_t* big_n, uint32_t big_cap) {
     if (reads_invalid(A.err)) return;
-    if (pick_variant(A) == 0) { wlist = wlist2; wlist_n = wlist2_n; }   // k_list_sites' leftovers
+    if (pick_variant(A) == 0 && *wlist_n >= LIST_MIN) { wlist = wlist2; wlist_n = wlist2_n; }   // k_list_sites' leftovers
+    const uint32_t count = *wlist_n;
+    if ((uint64_t)blockIdx.x * NW >= count) return;     // one warp per listed site
     extern __shared__ __align__(16) unsigned char smem[];
     TileSmem sm;
     call_smem_bytes(A.L, 0, CC, &sm, smem);
@@ -1954,7 +1962,6 @@ __global__ void __launch_bounds__(NT) k_warp_sites(const __grid_constant__ CallA
     uint8_t* myslot = sm.slotcnt + warp * 8 * A.L;
     for (int i = lane; i < 2 * A.L; i += 32) reinterpret_cast<uint32_t*>(myslot)[i] = 0;
     __syncwarp();
-    const uint32_t count = *wlist_n;
     for (uint32_t j = blockIdx.x * NW + warp; j < count; j += gridDim.x * NW) {
         const uint64_t s = A.w0 + wlist[j];
         const uint64_t grp = (s - A.w0) / 32;
@@ -1994,8 +2001,9 @@ __global__ void __launch_bounds__(NT) k_big_sites(const __grid_constant__ CallAr
     uint32_t* buf = reinterpret_cast<uint32_t*>(smem);
     uint8_t* slotcnt = smem + 4 * (size_t)cap;
     const int tid = threadIdx.x;
-    for (int i = tid; i < 2 * A.L; i += NT) reinterpret_cast<uint32_t*>(slotcnt)[i] = 0;
     const uint32_t count = *big_n;
+    if (blockIdx.x >= count) return;                    // one CTA per listed site
+    for (int i = tid; i < 2 * A.L; i += NT) reinterpret_cast<uint32_t*>(slotcnt)[i] = 0;
     for (uint32_t j = blockIdx.x; j < count; j += gridDim.x) {
         const BigSite bs = big[j];
         if (bs.n > cap) {
