@@ -210,6 +210,7 @@ struct gsnp_ctx {
     // 12.4 at 31.3 per 24 M sites)
     float mid_at = 29.5f, deep_at = 48.0f;
     uint32_t epoch = 0;               // calls so far (k_prep's read-length flag)
+    uint32_t list_min = 16384;        // k_list_sites below this many listed sites: warp path instead
     bool mid_adj_smem = false;        // the 64-slot kernel reads adj from L1/L2: 3 CTAs per SM
     size_t cal_budget = 0;            // k_calib_count shared-memory budget (0 = not yet sized)
     // per-stage timing (GSNP_TIMING)
@@ -523,6 +524,7 @@ gsnp_status prep_window(gsnp_ctx* ctx, const DevReads& d, uint64_t w0, uint64_t 
     A.R = d;
     A.len_flag = ctx->big_n.p + 3;
     A.epoch = epoch;
+    A.list_min = ctx->list_min;
     A.ref = ctx->ref_code;
     A.origin = ctx->origin;
     A.n_sites = ctx->n_sites;
@@ -912,6 +914,7 @@ gsnp_status gsnp_create(const gsnp_reference* ref, const gsnp_priors* priors,
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, params->device);
         ctx->num_sms = sms > 0 ? sms : 148;
         if (const char* e = getenv("GSNP_MID_AT")) ctx->mid_at = (float)atof(e);
+        if (const char* e = getenv("GSNP_LIST_MIN")) ctx->list_min = (uint32_t)strtoul(e, nullptr, 10);
         if (const char* e = getenv("GSNP_DEEP_AT")) ctx->deep_at = (float)atof(e);
         if (const char* e = getenv("GSNP_MID_ADJ_SMEM")) ctx->mid_adj_smem = atoi(e) != 0;
     }

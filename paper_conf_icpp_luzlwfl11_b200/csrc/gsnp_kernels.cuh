@@ -71,6 +71,7 @@ struct CallArgs {
     float mid_at, deep_at;            // window depth thresholds of the 64- and 128-slot kernels
     const uint32_t* len_flag;         // == epoch: not every read has the same length (k_prep)
     uint32_t epoch;
+    uint32_t list_min;                // listed sites below this count take the warp path
     // debug (all may be null)
     uint32_t* dbg_nuni;               // count-only pass: unique keys per site
     const uint32_t* dbg_off;          // CSR offsets for the key dumps
@@ -1863,17 +1864,17 @@ k_call_tile(const __grid_constant__ CallArgs A, uint32_t* wlist, uint32_t* wlist
 // into its own 64-slot column and runs the chunked thread path; sites with more than 64 keys or a
 // '-' end recount go on to k_warp_sites through the second list.  (Windows called by the 64- and
 // 128-slot kernels return at once: their lists hold only sites beyond those kernels' slots.)
-// Below LIST_MIN listed sites the warp path takes them all: a thread walks its site's ~40 reads one
-// round trip after another (~60 us whatever the count), while a warp per site finishes one site in
-// ~14 us with every warp of the GPU in parallel (256 K-site windows list ~600 sites).
-constexpr uint32_t LIST_MIN = 16384;
+// Below A.list_min listed sites (default 16384; GSNP_LIST_MIN) the warp path takes them all: a
+// thread walks its site's ~40 reads one round trip after another (~60 us whatever the count), while
+// a warp per site finishes one site in ~14 us with every warp of the GPU in parallel (256 K-site
+// windows list ~600 sites).
 template <bool DBG>
 __global__ void __launch_bounds__(NT, 3) k_list_sites(const __grid_constant__ CallArgs A, const uint32_t* wlist,
                                                       const uint32_t* wlist_n, uint32_t* wlist2,
                                                       uint32_t* wlist2_n, uint32_t* work) {
     if (reads_invalid(A.err) || pick_variant(A) != 0) return;
     const uint32_t count = *wlist_n;
-    if (count < LIST_MIN) return;                       // a short list: the warp path is quicker
+    if (count < A.list_min) return;                     // a short list: the warp path is quicker
     if ((uint64_t)blockIdx.x * NT >= count) return;
     extern __shared__ __align__(16) unsigned char smem[];
     __shared__ double lp_s[50];
@@ -1952,7 +1953,7 @@ __global__ void __launch_bounds__(NT) k_warp_sites(const __grid_constant__ CallA
                                                    const uint32_t* wlist2_n, BigSite* big,
                                                    uint32_t* big_n, uint32_t big_cap) {
     if (reads_invalid(A.err)) return;
-    if (pick_variant(A) == 0 && *wlist_n >= LIST_MIN) { wlist = wlist2; wlist_n = wlist2_n; }   // k_list_sites' leftovers
+    if (pick_variant(A) == 0 && *wlist_n >= A.list_min) { wlist = wlist2; wlist_n = wlist2_n; }   // k_list_sites' leftovers
     const uint32_t count = *wlist_n;
     if ((uint64_t)blockIdx.x * NW >= count) return;     // one warp per listed site
     extern __shared__ __align__(16) unsigned char smem[];

@@ -287,3 +287,24 @@ def test_unaligned_device_reads_calibrate_and_call(c1):
         ctx.calibrate_finalize(counts)
         got = ctx.call(dev, int(w["origin"]), int(w["origin"]) + len(w["ref"]))
     compare(w, got, rec, c1[4]["L10"])
+
+
+@pytest.mark.parametrize("case", ["26x_dups", "40x_32slot", "pile"])
+def test_listed_sites_thread_path_parity(case, monkeypatch):
+    """k_list_sites (the 32-slot kernel's sites with 33-64 unique keys, one thread per site,
+    chunked thread path) on small inputs: GSNP_LIST_MIN=0 sends every list through it (by default
+    lists under 16 K sites take the warp path).  At 40X with the 32-slot kernel forced
+    (GSNP_MID_AT) and in a 700-read pile, sites beyond 64 keys go on to the warp and CTA paths
+    through the second list."""
+    monkeypatch.setenv("GSNP_LIST_MIN", "0")
+    if case == "26x_dups":
+        w, win = synth.generate("C1", n_sites=6_000, depth=26.0, dup_rate=0.1, seed=26), (0, 6_000)
+    elif case == "40x_32slot":
+        monkeypatch.setenv("GSNP_MID_AT", "1000")
+        w, win = synth.generate("C1", n_sites=6_000, depth=40.0, dup_rate=0.1, seed=40), (0, 6_000)
+    else:
+        w, win = _pile_workload(700, seed=7), (150, 450)
+    C, p, _, _ = _oracle_all(w, w0=0, w1=1)
+    with _ctx(w) as ctx:
+        ctx.calibrate(w)
+        _check_window(ctx, w, win[0], win[1], C, p)
